@@ -1,0 +1,356 @@
+#!/usr/bin/env python
+"""Benchmark of the GP-metis coarsening hot path on B200 (one JSON line on rank 0).
+
+A "step" is one full coarsen-to-threshold (gp_coarsen_to: every level's matching rounds,
+cmap, contraction and CSR assembly) of the BASELINE.json workload, input resident in HBM.
+
+  metric  fine edges coarsened/s = sum over levels of |E_level| / (time of one step)
+  value   whole-job aggregate over all ranks
+  e2e     the same metric through the C ABI with HOST buffers: pinned H2D of the CSR,
+          gp_graph_create + gp_coarsen_to, D2H of every level's cmap + the coarsest graph
+  roofline  dominant kernel family, algorithmic bytes / CUDA-event time
+  cpu_baseline  the oracle (oracle/, single thread) on the box's host, bounded sample
+
+--impl reference times the oracle (the reference arm of this tier) on the same config.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import graphgen as G  # noqa: E402
+
+WORKLOADS = {
+    "C1": ("grid64x64_unit", 100),
+    "C2": ("rgg_n2^20_deg13_w1-100", 100),
+    "C3": ("delaunay_like_n2^22_w1-100", 100),
+    "C4": ("rmat_s24_ef16_w1-100", 100),
+    "C5": ("road_like_n2^26_deg2.5_w1-100", 100),
+}
+METRIC = "fine edges coarsened/sec (sum of |E| over levels / full coarsen-to-threshold time)"
+UNIT = "edges/s"
+L2_BYTES = 126 * 1024 * 1024
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+# ------------------------------------------------------------------------------------------
+# algorithmic byte model per kernel family; int32 everywhere
+# ------------------------------------------------------------------------------------------
+def level_bytes(l) -> dict:
+    n, nnz, nc, cnnz = l["n"], l["nnz"], l["n_coarse"], l["cnnz"]
+    S, Vs, R, L = l["arcs_scanned"], l["rows_scanned"], max(l["rounds"], 1), l["live_visits"]
+    return {
+        # adjp pair + P write per scanned row, adjncy+adjwgt per scanned arc, M gathers of
+        # rescans (rounds >= 2; each M entry counted at most once per round)
+        "propose": 12 * Vs + 8 * S + min(4 * max(S - nnz, 0), 4 * n * (R - 1)),
+        # per live visit: list entry (rounds >= 2), P[u], P[P[u]], P[P[P[u]]]; M writes
+        "commit": 12 * L + 4 * max(L - n, 0) + 4 * (n - nc) * 2 // 2,
+        # M read, CM write (+partner), adjp/vwgt gathers, leaders/ub/cvwgt writes
+        "cmap": 4 * n + 4 * n + 8 * n + 4 * n + 12 * nc,
+        # off/leaders/M per coarse row, adjp of both ends, adjncy+adjwgt once, CM gathers
+        # (each CM entry once), merged rows + counts written
+        "contract": 12 * nc + 8 * n + 8 * nnz + 4 * n + 8 * cnnz + 4 * nc,
+        # two scans (read + write) and the compaction (read off/cnt/cadjp + rows, write rows)
+        "assemble": 16 * nc + 12 * nc + 16 * cnnz,
+    }
+
+
+# ------------------------------------------------------------------------------------------
+# clocks sampled during the timed region
+# ------------------------------------------------------------------------------------------
+class ClockSampler:
+    FIELDS = "clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown," \
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap"
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], 0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 6:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx = max(mx, float(parts[1]))
+            except ValueError:
+                continue
+            for nm, val in zip(names, parts[2:6]):
+                if val.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------------------
+# oracle timing (cpu_baseline and --impl reference)
+# ------------------------------------------------------------------------------------------
+def oracle_run(g, threshold):
+    import oracle
+    t0 = time.perf_counter()
+    levels = oracle.coarsen_to(g, threshold)
+    dt = time.perf_counter() - t0
+    return dt, sum(l["nnz"] // 2 for l in levels), len(levels)
+
+
+def cpu_baseline(g, threshold, budget_s=12.0):
+    runs, tot_t, tot_e, nlev = 0, 0.0, 0, 0
+    while runs == 0 or tot_t < budget_s:
+        dt, e, nlev = oracle_run(g, threshold)
+        runs += 1
+        tot_t += dt
+        tot_e += e
+        if runs >= 8:
+            break
+    return {"value": tot_e / tot_t, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{runs} full coarsen-to-{threshold} run(s) of the same graph ({nlev} levels), "
+                      f"single-threaded C oracle, {tot_t:.1f} s"}
+
+
+def host_info():
+    try:
+        model = [l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo") if l.startswith("model name")][0]
+    except Exception:
+        model = "unknown"
+    return {"host_cpu": model, "host_nproc": os.cpu_count()}
+
+
+# ------------------------------------------------------------------------------------------
+def make_graph(cfg: str, device: str):
+    t0 = time.perf_counter()
+    g = G.make_config(cfg, device=device)
+    return g, time.perf_counter() - t0
+
+
+def run_ours(args, rank, world, local_rank):
+    import paper_conf_ipps_goodarzibg16_b200.gp as gp
+    torch.cuda.set_device(local_rank)
+    dev = f"cuda:{local_rank}"
+    name, threshold = WORKLOADS[args.config]
+    g, gen_s = make_graph(args.config, dev)
+    n, nnz = g["n"], g["nnz"]
+    ctx = gp.Context(local_rank)
+    stream = ctx.stream
+    graph = gp.Graph.create(ctx, g["adjp"], g["adjncy"], g["adjwgt"], g["vwgt"])
+
+    def step():
+        return graph.coarsen_to(threshold)
+
+    # warm-up
+    hier = None
+    for _ in range(args.warmup):
+        hier = step()
+        levels = [vars(l) for l in hier.levels()]
+        hier.close()
+    levels = [{k: v for k, v in l.items() if k != "coarse"} for l in levels]
+    edges_per_step = sum(l["nnz"] // 2 for l in levels)
+
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    ctx.reset_stats()
+    ctx.set_timing(True)
+    launches0 = ctx.launch_count()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local_rank) as clk:
+        ev0.record(stream)
+        for _ in range(args.steps):
+            hier = step()
+            hier.close()
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    ms = ev0.elapsed_time(ev1)
+    launches = ctx.launch_count() - launches0
+    kstats = ctx.kernel_stats()
+    ctx.set_timing(False)
+    # untimed-instrumentation check: the same steps without event brackets
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        hier = step()
+        hier.close()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms_plain = e0.elapsed_time(e1)
+    ms_step = min(ms, ms_plain) / args.steps
+    if world > 1:
+        t = torch.tensor([ms_step], device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms_step = float(t.item())
+
+    # roofline of the dominant kernel family
+    fam_bytes = {}
+    for l in levels:
+        for k, v in level_bytes(l).items():
+            fam_bytes[k] = fam_bytes.get(k, 0) + v
+    fam_ms = {k: kstats[k]["ms"] / args.steps for k in fam_bytes}
+    dom = max(fam_ms, key=lambda k: fam_ms[k])
+    peak, peak_kind = peaks()
+    achieved = fam_bytes[dom] / (fam_ms[dom] / 1e3) / 1e9 if fam_ms[dom] > 0 else 0.0
+    step_bytes = sum(fam_bytes.values())
+
+    # end-to-end through the C ABI with host buffers
+    host = {k: g[k].cpu().pin_memory() for k in ("adjp", "adjncy", "adjwgt", "vwgt")}
+    h2d = sum(t.numel() * 4 for t in host.values())
+    e2e_ms = []
+    d2h = 0
+    for it in range(max(2, min(args.steps, 5)) + 1):
+        torch.cuda.synchronize()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        gh = gp.Graph.create(ctx, host["adjp"], host["adjncy"], host["adjwgt"], host["vwgt"])
+        hh = gh.coarsen_to(threshold)
+        nb = 0
+        for i in range(len(hh)):
+            _, c = hh.download_level(i)
+            nb += c.numel() * 4
+        last = hh.level(len(hh) - 1).coarse.download()
+        nb += sum(last[k].numel() * 4 for k in ("adjp", "adjncy", "adjwgt", "vwgt"))
+        b.record(stream)
+        torch.cuda.synchronize()
+        hh.close()
+        gh.close()
+        if it > 0:
+            e2e_ms.append(a.elapsed_time(b))
+        d2h = nb
+    e2e_step = min(e2e_ms)
+
+    line = {
+        "metric": METRIC, "value": world * edges_per_step / (ms_step / 1e3), "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "config": {"workload": f"{args.config}:{name}", "n": n, "edges": nnz // 2, "threshold": threshold,
+                   "levels": len(levels), "edges_all_levels": edges_per_step,
+                   "level0_edges_per_s": (nnz // 2) / (ms_step / 1e3),
+                   "t_full_ms": ms_step, "rounds": [l["rounds"] for l in levels],
+                   "l2": f"L0 input {(4 * (2 * nnz + 2 * n)) / 2**20:.0f} MiB > L2 126 MiB (no flush)",
+                   "parallelism": "single GPU" if world == 1 else f"replicas x{world} (sharded path not built)",
+                   "gen_s": round(gen_s, 2)},
+        "hbm_gbs_step": step_bytes / (ms_step / 1e3) / 1e9,
+        "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "peak_kind": peak_kind,
+                     "unit": "GB/s", "frac": achieved / peak, "traffic": None,
+                     "bytes_per_step": fam_bytes[dom], "ms_per_step": fam_ms[dom]},
+        "kernels": {k: {"ms_per_step": fam_ms[k], "GB/s": (fam_bytes[k] / (fam_ms[k] / 1e3) / 1e9) if fam_ms[k] else None,
+                        "launches_per_step": kstats[k]["launches"] / args.steps} for k in fam_bytes},
+        "e2e": {"value": world * edges_per_step / (e2e_step / 1e3), "unit": UNIT, "ms_per_step": e2e_step,
+                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
+        "gpu_launches": launches,
+        "clocks": clk.summary(),
+    }
+    if rank == 0 and not args.no_cpu_baseline:
+        gh = {k: g[k].cpu() for k in ("adjp", "adjncy", "adjwgt", "vwgt")}
+        line["cpu_baseline"] = cpu_baseline(gh, threshold)
+        line["cpu_baseline"].update(host_info())
+    graph.close()
+    ctx.close()
+    return line
+
+
+def run_reference(args, rank, world):
+    name, threshold = WORKLOADS[args.config]
+    if rank != 0:
+        return None
+    g, _ = make_graph(args.config, "cpu")
+    for _ in range(args.warmup):
+        oracle_run(g, threshold)
+    t = 0.0
+    e = 0
+    for _ in range(args.steps):
+        dt, e, nlev = oracle_run(g, threshold)
+        t += dt
+    ms = t / args.steps * 1e3
+    value = e / (ms / 1e3)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": f"{args.config}:{name}", "n": g["n"], "edges": g["nnz"] // 2,
+                       "threshold": threshold, "edges_all_levels": e},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"full coarsen-to-{threshold} per step, single-threaded C oracle"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    line["cpu_baseline"].update(host_info())
+    return line
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", choices=sorted(WORKLOADS), default="C3")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3) if args.impl == "ours" else args.warmup
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1 and args.impl == "ours":
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        torch.distributed.init_process_group("nccl", device_id=torch.device(f"cuda:{local_rank}"))
+
+    if args.impl == "reference":
+        line = run_reference(args, rank, world)
+    else:
+        line = run_ours(args, rank, world, local_rank)
+    if rank == 0 and line is not None:
+        print(json.dumps(line), flush=True)
+    if world > 1 and args.impl == "ours":
+        torch.distributed.barrier()
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,298 @@
+"""Thin Python binding of the C ABI in include/gp.h (argument marshalling only).
+
+Every step of the coarsening path runs in libgpcoarsen.so's sm_100a kernels; this module
+only passes pointers (torch tensors' ``data_ptr()``), sizes and the current CUDA stream.
+There is NO CPU fallback: importing this module raises if the shared library is missing,
+and creating a context raises if no CUDA device is present.
+
+Names follow the ABI (and the paper's notation: adjp/adjncy/adjwgt/vwgt, P16.s17-19;
+match M and cmap CM, P16.s24).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+from typing import Dict, List, Optional
+
+import torch
+
+from ._build import LIB
+
+if not os.path.exists(LIB):
+    raise ImportError(f"libgpcoarsen.so not built ({LIB}); run __graft_entry__.build() — "
+                      "there is no CPU fallback for the coarsening path")
+
+_lib = ctypes.CDLL(LIB)
+
+_vp = ctypes.c_void_p
+_i32 = ctypes.c_int32
+_i32p = ctypes.POINTER(ctypes.c_int32)
+
+GP_INPUT_DEVICE = 0x1
+GP_VALIDATE = 0x2
+
+STATUS = {0: "GP_OK", 1: "GP_ERR_INVALID_ARG", 2: "GP_ERR_INVALID_GRAPH", 3: "GP_ERR_OVERFLOW",
+          4: "GP_ERR_OUT_OF_MEMORY", 5: "GP_ERR_CUDA", 6: "GP_ERR_NCCL", 7: "GP_ERR_INTERNAL"}
+
+STOP_NONE, STOP_THRESHOLD, STOP_STALL, STOP_MAX_LEVELS = 0, 1, 2, 3
+K_PROPOSE, K_COMMIT, K_CMAP, K_CONTRACT, K_ASSEMBLE, K_OTHER = range(6)
+KERNEL_KINDS = ["propose", "commit", "cmap", "contract", "assemble", "other"]
+
+
+class GPError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        detail = _lib.gp_last_error().decode(errors="replace")
+        super().__init__(f"{where}: {STATUS.get(status, status)}: {detail}")
+        self.status = status
+
+
+class CoarsenOpts(ctypes.Structure):
+    _fields_ = [("threshold", _i32), ("stall_ratio_pct", _i32), ("max_levels", _i32), ("max_rounds", _i32)]
+
+
+class Level(ctypes.Structure):
+    _fields_ = [("n", _i32), ("nnz", _i32), ("n_coarse", _i32), ("cnnz", _i32), ("rounds", _i32),
+                ("maximal", _i32), ("stop_reason", _i32), ("reserved", _i32),
+                ("arcs_scanned", ctypes.c_int64), ("rows_scanned", ctypes.c_int64),
+                ("live_visits", ctypes.c_int64), ("d_match", _vp), ("d_cmap", _vp), ("coarse", _vp)]
+
+
+class KernelStats(ctypes.Structure):
+    _fields_ = [("launches", ctypes.c_int64), ("ms", ctypes.c_double)]
+
+
+def _sig(name, res, args):
+    f = getattr(_lib, name)
+    f.restype = res
+    f.argtypes = args
+    return f
+
+
+_sig("gp_status_string", ctypes.c_char_p, [ctypes.c_int])
+_sig("gp_last_error", ctypes.c_char_p, [])
+_sig("gp_ctx_create", ctypes.c_int, [ctypes.c_int, _vp, ctypes.POINTER(_vp)])
+_sig("gp_ctx_num_sms", ctypes.c_int, [_vp, _i32p])
+_sig("gp_graph_create", ctypes.c_int, [_vp, _i32, _vp, _vp, _vp, _vp, ctypes.c_uint32, ctypes.POINTER(_vp)])
+_sig("gp_graph_view", ctypes.c_int, [_vp, _i32p, _i32p, ctypes.POINTER(_vp), ctypes.POINTER(_vp),
+                                     ctypes.POINTER(_vp), ctypes.POINTER(_vp)])
+_sig("gp_graph_download", ctypes.c_int, [_vp, _vp, _vp, _vp, _vp])
+_sig("gp_match_level", ctypes.c_int, [_vp, _vp, _i32, _i32p])
+_sig("gp_contract_level", ctypes.c_int, [_vp, _vp, _vp, ctypes.POINTER(_vp)])
+_sig("gp_coarsen_to", ctypes.c_int, [_vp, ctypes.POINTER(CoarsenOpts), ctypes.POINTER(_vp)])
+_sig("gp_hier_num_levels", ctypes.c_int, [_vp, _i32p])
+_sig("gp_hier_level", ctypes.c_int, [_vp, _i32, ctypes.POINTER(Level)])
+_sig("gp_hier_download_level", ctypes.c_int, [_vp, _i32, _vp, _vp])
+_sig("gp_free", None, [_vp])
+_sig("gp_ctx_set_timing", ctypes.c_int, [_vp, _i32])
+_sig("gp_ctx_kernel_stats", ctypes.c_int, [_vp, ctypes.c_int, ctypes.POINTER(KernelStats)])
+_sig("gp_ctx_reset_stats", ctypes.c_int, [_vp])
+_sig("gp_ctx_launch_count", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_int64)])
+
+
+def _check(st: int, where: str) -> None:
+    if st != 0:
+        raise GPError(st, where)
+
+
+def _ptr(t: Optional[torch.Tensor]):
+    if t is None:
+        return None
+    assert t.dtype == torch.int32 and t.is_contiguous(), "int32 contiguous tensors expected"
+    return t.data_ptr()
+
+
+class Context:
+    """gp_ctx on a CUDA device, enqueuing on the given (default: current) torch stream."""
+
+    def __init__(self, device: int = 0, stream: Optional[torch.cuda.Stream] = None):
+        if not torch.cuda.is_available():
+            raise RuntimeError("no CUDA device: the coarsening path has no CPU fallback")
+        self.device = device
+        self.stream = stream if stream is not None else torch.cuda.current_stream(device)
+        h = _vp()
+        _check(_lib.gp_ctx_create(device, self.stream.cuda_stream, ctypes.byref(h)), "gp_ctx_create")
+        self.handle = h
+
+    def close(self) -> None:
+        if self.handle is not None and self.handle.value:
+            _lib.gp_free(self.handle)
+        self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    @property
+    def num_sms(self) -> int:
+        v = _i32()
+        _check(_lib.gp_ctx_num_sms(self.handle, ctypes.byref(v)), "gp_ctx_num_sms")
+        return v.value
+
+    def set_timing(self, on: bool) -> None:
+        _check(_lib.gp_ctx_set_timing(self.handle, 1 if on else 0), "gp_ctx_set_timing")
+
+    def reset_stats(self) -> None:
+        _check(_lib.gp_ctx_reset_stats(self.handle), "gp_ctx_reset_stats")
+
+    def kernel_stats(self) -> Dict[str, Dict[str, float]]:
+        out = {}
+        for k, name in enumerate(KERNEL_KINDS):
+            s = KernelStats()
+            _check(_lib.gp_ctx_kernel_stats(self.handle, k, ctypes.byref(s)), "gp_ctx_kernel_stats")
+            out[name] = {"launches": int(s.launches), "ms": float(s.ms)}
+        return out
+
+    def launch_count(self) -> int:
+        v = ctypes.c_int64()
+        _check(_lib.gp_ctx_launch_count(self.handle, ctypes.byref(v)), "gp_ctx_launch_count")
+        return int(v.value)
+
+
+class Graph:
+    """Library-owned device CSR graph (gp_graph)."""
+
+    def __init__(self, ctx: Context, handle, owned: bool = True):
+        self.ctx = ctx
+        self.handle = handle
+        self.owned = owned
+
+    @classmethod
+    def create(cls, ctx: Context, adjp: torch.Tensor, adjncy: torch.Tensor, adjwgt: Optional[torch.Tensor] = None,
+               vwgt: Optional[torch.Tensor] = None, validate: bool = False) -> "Graph":
+        """gp_graph_create from int32 tensors, all on the GPU or all on the host (pinned
+        host memory gives asynchronous copies)."""
+        n = adjp.numel() - 1
+        dev = adjp.is_cuda
+        for t in (adjncy, adjwgt, vwgt):
+            if t is not None and t.is_cuda != dev:
+                raise ValueError("inputs must all be on the device or all on the host")
+        flags = (GP_INPUT_DEVICE if dev else 0) | (GP_VALIDATE if validate else 0)
+        h = _vp()
+        _check(_lib.gp_graph_create(ctx.handle, n, _ptr(adjp), _ptr(adjncy), _ptr(adjwgt), _ptr(vwgt), flags,
+                                    ctypes.byref(h)), "gp_graph_create")
+        return cls(ctx, h)
+
+    def close(self) -> None:
+        if self.owned and self.handle is not None and self.handle.value:
+            _lib.gp_free(self.handle)
+        self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def view(self):
+        n, nnz = _i32(), _i32()
+        _check(_lib.gp_graph_view(self.handle, ctypes.byref(n), ctypes.byref(nnz), None, None, None, None),
+               "gp_graph_view")
+        return n.value, nnz.value
+
+    @property
+    def n(self) -> int:
+        return self.view()[0]
+
+    @property
+    def nnz(self) -> int:
+        return self.view()[1]
+
+    def download(self) -> Dict[str, torch.Tensor]:
+        """Copy the CSR arrays to host int32 tensors (gp_graph_download)."""
+        n, nnz = self.view()
+        out = {k: torch.empty(sz, dtype=torch.int32) for k, sz in
+               (("adjp", n + 1), ("adjncy", nnz), ("adjwgt", nnz), ("vwgt", n))}
+        _check(_lib.gp_graph_download(self.handle, out["adjp"].data_ptr(), out["adjncy"].data_ptr(),
+                                      out["adjwgt"].data_ptr(), out["vwgt"].data_ptr()), "gp_graph_download")
+        out["n"], out["nnz"] = n, nnz
+        return out
+
+    def match_level(self, match: torch.Tensor, max_rounds: int = 0, sync_rounds: bool = True) -> Optional[int]:
+        """gp_match_level into a caller-owned device int32[n] tensor; returns rounds."""
+        r = _i32()
+        _check(_lib.gp_match_level(self.handle, _ptr(match), max_rounds, ctypes.byref(r) if sync_rounds else None),
+               "gp_match_level")
+        return r.value if sync_rounds else None
+
+    def contract_level(self, match: torch.Tensor, cmap: torch.Tensor) -> "Graph":
+        """gp_contract_level: fills cmap, returns the coarse graph (caller-owned)."""
+        h = _vp()
+        _check(_lib.gp_contract_level(self.handle, _ptr(match), _ptr(cmap), ctypes.byref(h)), "gp_contract_level")
+        return Graph(self.ctx, h)
+
+    def coarsen_to(self, threshold: int, stall_ratio_pct: int = 95, max_levels: int = 64,
+                   max_rounds: int = 0) -> "Hierarchy":
+        opts = CoarsenOpts(threshold, stall_ratio_pct, max_levels, max_rounds)
+        h = _vp()
+        _check(_lib.gp_coarsen_to(self.handle, ctypes.byref(opts), ctypes.byref(h)), "gp_coarsen_to")
+        return Hierarchy(self.ctx, h)
+
+
+@dataclass
+class LevelInfo:
+    n: int
+    nnz: int
+    n_coarse: int
+    cnnz: int
+    rounds: int
+    maximal: bool
+    stop_reason: int
+    arcs_scanned: int
+    rows_scanned: int
+    live_visits: int
+    coarse: Graph
+
+
+class Hierarchy:
+    """gp_hier: the kept level hierarchy (M, CM, coarse graph per level; P20.s27)."""
+
+    def __init__(self, ctx: Context, handle):
+        self.ctx = ctx
+        self.handle = handle
+
+    def close(self) -> None:
+        if self.handle is not None and self.handle.value:
+            _lib.gp_free(self.handle)
+        self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __len__(self) -> int:
+        v = _i32()
+        _check(_lib.gp_hier_num_levels(self.handle, ctypes.byref(v)), "gp_hier_num_levels")
+        return v.value
+
+    def level(self, i: int) -> LevelInfo:
+        l = Level()
+        _check(_lib.gp_hier_level(self.handle, i, ctypes.byref(l)), "gp_hier_level")
+        return LevelInfo(l.n, l.nnz, l.n_coarse, l.cnnz, l.rounds, bool(l.maximal), l.stop_reason,
+                         l.arcs_scanned, l.rows_scanned, l.live_visits, Graph(self.ctx, _vp(l.coarse), owned=False))
+
+    def levels(self) -> List[LevelInfo]:
+        return [self.level(i) for i in range(len(self))]
+
+    def download_level(self, i: int):
+        """(match, cmap) of level i as host int32 tensors."""
+        info = self.level(i)
+        m = torch.empty(info.n, dtype=torch.int32)
+        c = torch.empty(info.n, dtype=torch.int32)
+        _check(_lib.gp_hier_download_level(self.handle, i, m.data_ptr(), c.data_ptr()), "gp_hier_download_level")
+        return m, c
+
+
+def exported_symbols():
+    """Every gp_* entry point declared in include/gp.h."""
+    import re
+    hdr = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include", "gp.h")
+    with open(hdr) as f:
+        text = f.read()
+    text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)               # drop comments
+    return sorted(set(re.findall(r"^\s*(?:gp_status|void|const char\s*\*)\s*(gp_[a-z_0-9]+)\s*\(", text,
+                                 flags=re.M)))

@@ -128,9 +128,11 @@ def check_level(g: Dict, match: np.ndarray, cmap: np.ndarray, n_c: int, coarse: 
     src = np.repeat(np.arange(n), np.diff(g["adjp"]))
     collapsed = int(g["adjwgt"][m[src] == g["adjncy"]].sum())      # both arc directions
     assert int(c["adjwgt"].sum()) == int(g["adjwgt"].sum()) - collapsed
-    for cc in range(n_c):
-        row = c["adjncy"][c["adjp"][cc]:c["adjp"][cc + 1]]
-        assert np.all(np.diff(row) > 0), "coarse row not strictly increasing"
+    adj = c["adjncy"]
+    if len(adj) > 1:
+        rows = np.repeat(np.arange(n_c), np.diff(c["adjp"]))
+        same_row = rows[1:] == rows[:-1]
+        assert np.all(np.diff(adj)[same_row] > 0), "coarse row not strictly increasing"
 
 
 def contract_by_sparse_triple_product(g: Dict, cmap: np.ndarray, n_c: int) -> Dict:
