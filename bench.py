@@ -56,22 +56,26 @@ def peaks():
 # algorithmic byte model per kernel family; int32 everywhere
 # ------------------------------------------------------------------------------------------
 def level_bytes(l) -> dict:
+    """Algorithmic HBM bytes of one level per kernel family.
+
+    match    (k_match_level: A1-A4, every round)
+      phase 0   adjp 4(n+1) + adjncy/adjwgt 8*nnz + P and M writes 8n
+      rounds    per live visit: list entry, P[u], P[p], P[q], one write, one append (24 B)
+      rescans   8 B per rescanned arc + adjp pair and P write per rescanned row (12 B)
+                + M gathers, each M entry counted at most once per round
+    contract (k_contract_level: A4 leftover + A5-A8)
+      C1        M 4n, CM 4n, adjp of leader+partner 8n, vwgt 4n, leaders/cvwgt/off 12 n_c
+      C2        off/leaders/M/cnt per coarse row 24 n_c, adjp 8n, adjncy+adjwgt 8 nnz,
+                CM gathers (each entry once) 4n, cadjp 4 n_c, cadjncy+cadjwgt 8 cnnz
+    """
     n, nnz, nc, cnnz = l["n"], l["nnz"], l["n_coarse"], l["cnnz"]
     S, Vs, R, L = l["arcs_scanned"], l["rows_scanned"], max(l["rounds"], 1), l["live_visits"]
-    return {
-        # adjp pair + P write per scanned row, adjncy+adjwgt per scanned arc, M gathers of
-        # rescans (rounds >= 2; each M entry counted at most once per round)
-        "propose": 12 * Vs + 8 * S + min(4 * max(S - nnz, 0), 4 * n * (R - 1)),
-        # per live visit: list entry (rounds >= 2), P[u], P[P[u]], P[P[P[u]]]; M writes
-        "commit": 12 * L + 4 * max(L - n, 0) + 4 * (n - nc) * 2 // 2,
-        # M read, CM write (+partner), adjp/vwgt gathers, leaders/ub/cvwgt writes
-        "cmap": 4 * n + 4 * n + 8 * n + 4 * n + 12 * nc,
-        # off/leaders/M per coarse row, adjp of both ends, adjncy+adjwgt once, CM gathers
-        # (each CM entry once), merged rows + counts written
-        "contract": 12 * nc + 8 * n + 8 * nnz + 4 * n + 8 * cnnz + 4 * nc,
-        # two scans (read + write) and the compaction (read off/cnt/cadjp + rows, write rows)
-        "assemble": 16 * nc + 12 * nc + 16 * cnnz,
-    }
+    rescan_arcs = max(S - nnz, 0)
+    rescan_rows = max(Vs - n, 0)
+    match = (4 * (n + 1) + 8 * nnz + 8 * n) + 24 * L + 8 * rescan_arcs + 12 * rescan_rows \
+        + min(4 * rescan_arcs, 4 * n * (R - 1))
+    contract = (20 * n + 12 * nc) + (24 * nc + 8 * n + 8 * nnz + 4 * n + 4 * nc + 8 * cnnz)
+    return {"match": match, "contract": contract}
 
 
 # ------------------------------------------------------------------------------------------
@@ -233,7 +237,8 @@ def run_ours(args, rank, world, local_rank):
     for l in levels:
         for k, v in level_bytes(l).items():
             fam_bytes[k] = fam_bytes.get(k, 0) + v
-    fam_ms = {k: kstats[k]["ms"] / args.steps for k in fam_bytes}
+    kfam = {"match": "propose", "contract": "contract"}   # gp_kernel_kind of each family
+    fam_ms = {k: kstats[kfam[k]]["ms"] / args.steps for k in fam_bytes}
     dom = max(fam_ms, key=lambda k: fam_ms[k])
     peak, peak_kind = peaks()
     achieved = fam_bytes[dom] / (fam_ms[dom] / 1e3) / 1e9 if fam_ms[dom] > 0 else 0.0
@@ -282,7 +287,7 @@ def run_ours(args, rank, world, local_rank):
                      "unit": "GB/s", "frac": achieved / peak, "traffic": None,
                      "bytes_per_step": fam_bytes[dom], "ms_per_step": fam_ms[dom]},
         "kernels": {k: {"ms_per_step": fam_ms[k], "GB/s": (fam_bytes[k] / (fam_ms[k] / 1e3) / 1e9) if fam_ms[k] else None,
-                        "launches_per_step": kstats[k]["launches"] / args.steps} for k in fam_bytes},
+                        "launches_per_step": kstats[kfam[k]]["launches"] / args.steps} for k in fam_bytes},
         "e2e": {"value": world * edges_per_step / (e2e_step / 1e3), "unit": UNIT, "ms_per_step": e2e_step,
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
         "gpu_launches": launches,

@@ -1,22 +1,28 @@
-// contract.cu -- A4 leftover + A5 cmap + A6 sizing + A7 merge + A8 coarse CSR assembly.
+// contract.cu -- A4 leftover + A5 cmap + A6 sizing + A7 merge + A8 coarse CSR assembly of
+// one level in ONE persistent cooperative kernel.
 //
-// Paper: the mapping array CM is built by four kernels (flag u<=M[u], CUB inclusive scan,
-// subtract one, partner copy; P18.s16-27).  Contraction sizes each thread's output by the
-// pair's degree sum (P20.s5-11), merges the two neighbour lists by quicksort + duplicate
-// removal or by a per-thread hash table (P20.s14-21), counts, scans again and copies the
-// rows into the final arrays (P20.s22-26).
+// Paper: CM is built by four kernels (flag u<=M[u], CUB inclusive scan, subtract one,
+// partner copy; P18.s16-27).  Contraction sizes each thread's output by the pair's degree
+// sum (P20.s5-11), merges the two neighbour lists by quicksort + duplicate removal or a
+// per-thread hash table (P20.s14-21), counts, scans again and copies the rows into the
+// final arrays (P20.s22-26).
 //
 // B200 design:
-//  * A4+A5+A6 are ONE single-pass kernel (decoupled look-back scan over the leader flags):
-//    the leftover self-match, the exclusive scan (= the paper's inclusive scan minus one),
-//    the leader list, the partner's CM (written by its leader, so no second pass), the
-//    coarse vertex weight and the merged-row upper bound are all produced in one read of M.
-//  * A7 bins coarse rows by their upper bound: <= 16 entries are merged by one thread in
-//    registers (bitonic network + run-length sum); <= 256 by a warp in shared memory;
-//    <= 8192 by a CTA in shared memory; longer (R-MAT hubs) by a CTA in global scratch.
-//    Rows are emitted in ascending coarse id (R10) with weights of repeated coarse
-//    neighbours summed (R8) and the collapsed edge dropped (R9).
-//  * A8: look-back scan of the merged counts + compaction into the final arrays.
+//  C1  one decoupled look-back pass over u in [0,n): leftover self-match, leader flags,
+//      exclusive scan (= the paper's inclusive scan minus one), leader list, the partner's
+//      CM (written by its leader: no second pass), cvwgt, and the exclusive prefix `off`
+//      of the merged-row upper bounds ub = deg(u) + deg(partner) (P20.s6-8).  Coarse rows
+//      are cut into tiles of kTileArcs upper-bound entries; C1 also records each tile's
+//      first row.
+//  C1b (only if some ub > kTileArcs, e.g. R-MAT hubs) such rows are merged by a whole CTA
+//      in global scratch.
+//  C2  one pass over the tiles in order: every row of the tile is merged into the tile's
+//      shared-memory slots (ub <= 16: one thread, registers + bitonic network; longer: one
+//      warp, shared-memory bitonic sort), counted, the tile total gets its global prefix
+//      by decoupled look-back, and the rows are written straight into the final compact
+//      cadjp/cadjncy/cadjwgt (no temporary arrays, no second scan, no copy kernel).
+//  Rows come out sorted by coarse id (R10) with repeated coarse neighbours summed (R8) and
+//  the collapsed edge dropped (R9).
 #include <cuda_runtime.h>
 
 #include "device_util.cuh"
@@ -24,148 +30,126 @@
 
 namespace gp {
 
-constexpr int kScanItems = 8;
-constexpr int kTile = kBlock * kScanItems;  // 2048 elements per look-back tile
-constexpr int kNet = 16;                    // thread-bin capacity
-constexpr int kWarpCap = 256;               // warp-bin capacity (entries)
-constexpr int kCtaCap = 8192;               // CTA-bin capacity (entries, 64 KB smem)
+constexpr int kCNT = 512;              // threads per CTA
+constexpr int kCItems = 8;             // vertices per thread per C1 tile
+constexpr int kCTileV = kCNT * kCItems;  // 4096 vertices per C1 tile
+constexpr int kTileArcs = 4096;        // C2 tile budget (upper-bound entries); rows with a
+                                       // larger bound are merged by C1b
+constexpr int kTileBuf = 2 * kTileArcs;  // a row starting inside the budget ends within 2x
+constexpr int kNet = 16;               // one-thread merge capacity
 constexpr unsigned long long kMaxKey = ~0ull;
 
-struct ContractBufs {
-    int32_t *leaders, *ub, *off, *cnt;
-    int32_t *binW, *binC, *binG;
-    int32_t *tadj, *tw;           // merged rows at off[c] (P20.s11-13 "temporary" arrays)
-    unsigned long long *gkeys;    // global-bin sort space at off[c]
+struct ContractArgs {
+    const SizeRec *in;  // device: sizes + stop flag of this level's graph
+    const int32_t *adjp, *adjncy, *adjwgt, *vwgt;
+    int32_t *M, *CM;
+    int32_t *leaders, *off, *cnt, *tile_start, *huge;
+    unsigned long long *gkeys;  // C1b scratch (nnz entries)
+    unsigned long long *st1;    // C1 look-back status (4 words per tile)
+    unsigned long long *st2;    // C2 look-back status (2 words per tile)
+    uint32_t epoch;
+    int32_t *cadjp, *cadjncy, *cadjwgt, *cvwgt;  // coarse graph (upper-bound sized)
+    ContractCtl *ctl;
+    SizeRec *out;  // device: sizes + stop decision of the coarse graph
+    int32_t apply_leftover;
+    int32_t threshold, stall_pct, level, max_levels;
+    LevelReport *report;  // mapped host memory (may be null)
+};
+
+struct ContractSmem {
+    unsigned long long buf[kTileBuf];
+    int32_t scan[40];
+    int32_t tile, prefix, len;
+    unsigned long long prefix2;
+    int32_t wlen[kCNT / 32];
+    int32_t lead[kCNT], has[kCNT];
+    int32_t hub_c, hub_o;
 };
 
 // ---------------------------------------------------------------------------------------
-// A4 leftover + A5 cmap + A6 sizing: one decoupled look-back pass over u in [0, n)
+// look-back over V values per tile (V in {1,2}); words per tile: V aggregate + V inclusive;
+// a word is valid when its high half equals (epoch | 2^31).
 // ---------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kBlock) k_cmap_scan(int32_t n, const int32_t *__restrict__ adjp,
-                                                      const int32_t *__restrict__ vwgt, int32_t *__restrict__ M,
-                                                      int32_t *__restrict__ CM, ContractBufs b,
-                                                      int32_t *__restrict__ cvwgt, unsigned long long *status,
-                                                      uint32_t epoch, LevelCtl *ctl, int apply_leftover) {
-    __shared__ int32_t s_scan[33];
-    __shared__ int32_t s_tile, s_prefix;
-    const int ntiles = (n + kTile - 1) / kTile;
-    while (true) {
-        if (threadIdx.x == 0) s_tile = (int32_t)atomicAdd(&ctl->tile_ctr[0], 1u);
-        __syncthreads();
-        const int tile = s_tile;
-        __syncthreads();
-        if (tile >= ntiles) break;
-        const long long base = (long long)tile * kTile + (long long)threadIdx.x * kScanItems;
-        int32_t m[kScanItems];
-        int32_t cnt = 0;
+template <int V>
+__device__ __forceinline__ void lookback(unsigned long long *st, uint32_t epoch, int tile, const int32_t (&agg)[V],
+                                         int32_t (&prefix)[V]) {
+    const int l = threadIdx.x & 31;
+    const unsigned long long tag = ((unsigned long long)(epoch | 0x80000000u)) << 32;
+    unsigned long long *me = st + (size_t)tile * 2 * V;
 #pragma unroll
-        for (int i = 0; i < kScanItems; ++i) {
-            const long long u = base + i;
-            m[i] = -2;
-            if (u < n) {
-                m[i] = M[u];
-                if (m[i] == kFree && apply_leftover) {
-                    m[i] = (int32_t)u;  // leftover: matched to itself (P18.s12-13)
-                    M[u] = (int32_t)u;
-                }
-                cnt += (u <= m[i]) ? 1 : 0;  // leader flag (P18.s18, R7)
-            }
-        }
-        int32_t total;
-        int32_t excl = block_excl_scan<kBlock>(cnt, s_scan, total);
-        if (threadIdx.x < 32) {
-            int32_t pre = lookback_prefix(status, epoch, tile, total);
-            if (threadIdx.x == 0) s_prefix = pre;
-        }
-        __syncthreads();
-        int32_t c = s_prefix + excl;
-        if (tile == ntiles - 1 && threadIdx.x == 0) ctl->n_coarse = s_prefix + total;
+    for (int i = 0; i < V; ++i) prefix[i] = 0;
+    if (tile == 0) {
+        if (l == 0)
 #pragma unroll
-        for (int i = 0; i < kScanItems; ++i) {
-            const long long u = base + i;
-            if (u < n && u <= m[i]) {
-                const int32_t v = m[i];
-                CM[u] = c;                      // exclusive scan = inclusive - 1 (P18.s20-24)
-                b.leaders[c] = (int32_t)u;
-                int32_t d = adjp[u + 1] - adjp[u];
-                int32_t vw = vwgt[u];
-                if (v != u) {
-                    CM[v] = c;                  // partner copies its leader's id (P18.s26)
-                    d += adjp[v + 1] - adjp[v];  // sizing: deg(u) + deg(v) (P20.s6-8)
-                    vw += vwgt[v];               // w(c) = w(u) + w(v) (P12.s27)
-                }
-                b.ub[c] = d;
-                cvwgt[c] = vw;
-                ++c;
-            }
-        }
-        __syncthreads();
-    }
-}
-
-// ---------------------------------------------------------------------------------------
-// generic exclusive scan: out[i] = sum_{j<i} in[j] for i <= count, count read from device
-// ---------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kBlock) k_scan_excl(const int32_t *__restrict__ in, int32_t *__restrict__ out,
-                                                      const int32_t *count_ptr, int32_t *total_out,
-                                                      unsigned long long *status, uint32_t epoch,
-                                                      uint32_t *tile_ctr) {
-    __shared__ int32_t s_scan[33];
-    __shared__ int32_t s_tile, s_prefix;
-    const int32_t count = *count_ptr;
-    const int ntiles = count > 0 ? (count + kTile - 1) / kTile : 0;
-    if (count == 0) {
-        if (blockIdx.x == 0 && threadIdx.x == 0) {
-            out[0] = 0;
-            if (total_out) *total_out = 0;
-        }
+            for (int i = 0; i < V; ++i) lb_store(me + V + i, tag | (uint32_t)agg[i]);
         return;
     }
+    if (l == 0)
+#pragma unroll
+        for (int i = 0; i < V; ++i) lb_store(me + i, tag | (uint32_t)agg[i]);
+    int pred = tile - 1;
     while (true) {
-        if (threadIdx.x == 0) s_tile = (int32_t)atomicAdd(tile_ctr, 1u);
-        __syncthreads();
-        const int tile = s_tile;
-        __syncthreads();
-        if (tile >= ntiles) break;
-        const long long base = (long long)tile * kTile + (long long)threadIdx.x * kScanItems;
-        int32_t x[kScanItems];
-        int32_t sum = 0;
+        const int idx = pred - l;
+        int kind = 2;  // 2 inclusive, 1 aggregate (idx < 0 behaves as an inclusive 0)
+        int32_t val[V];
 #pragma unroll
-        for (int i = 0; i < kScanItems; ++i) {
-            x[i] = (base + i < count) ? in[base + i] : 0;
-            sum += x[i];
-        }
-        int32_t total;
-        int32_t excl = block_excl_scan<kBlock>(sum, s_scan, total);
-        if (threadIdx.x < 32) {
-            int32_t pre = lookback_prefix(status, epoch, tile, total);
-            if (threadIdx.x == 0) s_prefix = pre;
-        }
-        __syncthreads();
-        int32_t run = s_prefix + excl;
+        for (int i = 0; i < V; ++i) val[i] = 0;
+        if (idx >= 0) {
+            const unsigned long long *w = st + (size_t)idx * 2 * V;
+            const long long guard = spin_start();
+            while (true) {
+                spin_check(guard);
+                bool inc = true, ag = true;
+                unsigned long long wi[V], wa[V];
 #pragma unroll
-        for (int i = 0; i < kScanItems; ++i) {
-            if (base + i < count) out[base + i] = run;
-            run += x[i];
+                for (int i = 0; i < V; ++i) {
+                    wi[i] = lb_load(w + V + i);
+                    inc &= (wi[i] & 0xFFFFFFFF00000000ull) == tag;
+                }
+                if (inc) {
+#pragma unroll
+                    for (int i = 0; i < V; ++i) val[i] = (int32_t)(uint32_t)wi[i];
+                    kind = 2;
+                    break;
+                }
+#pragma unroll
+                for (int i = 0; i < V; ++i) {
+                    wa[i] = lb_load(w + i);
+                    ag &= (wa[i] & 0xFFFFFFFF00000000ull) == tag;
+                }
+                if (ag) {
+#pragma unroll
+                    for (int i = 0; i < V; ++i) val[i] = (int32_t)(uint32_t)wa[i];
+                    kind = 1;
+                    break;
+                }
+            }
         }
-        if (tile == ntiles - 1 && threadIdx.x == 0) {
-            out[count] = s_prefix + total;
-            if (total_out) *total_out = s_prefix + total;
+        const unsigned incl = __ballot_sync(0xffffffffu, kind == 2);
+        const int first = incl ? __ffs(incl) - 1 : 32;
+#pragma unroll
+        for (int i = 0; i < V; ++i) {
+            int32_t c = (l <= first) ? val[i] : 0;
+            c = warp_sum(c);
+            prefix[i] += c;
         }
-        __syncthreads();
+        if (incl) break;
+        pred -= 32;
     }
+    if (l == 0)
+#pragma unroll
+        for (int i = 0; i < V; ++i) lb_store(me + V + i, tag | (uint32_t)(prefix[i] + agg[i]));
 }
 
 // ---------------------------------------------------------------------------------------
-// A7 helpers
+// merge helpers
 // ---------------------------------------------------------------------------------------
-// coarse key of one arc: coarse neighbour id in the high word, edge weight in the low word
 __device__ __forceinline__ unsigned long long ckey(int32_t cx, int32_t w) {
     return ((unsigned long long)(uint32_t)cx << 32) | (uint32_t)w;
 }
 
 __device__ __forceinline__ void cswap(unsigned long long &a, unsigned long long &b) {
-    unsigned long long lo = a < b ? a : b, hi = a < b ? b : a;
+    const unsigned long long lo = a < b ? a : b, hi = a < b ? b : a;
     a = lo;
     b = hi;
 }
@@ -189,36 +173,34 @@ __device__ __forceinline__ void reg_sort(unsigned long long (&k)[N]) {
     }
 }
 
-// Sort len keys in place (any len) with the flip bitonic network; comparators whose
-// upper index is >= len are skipped (virtual +inf padding never moves).
-// Cooperative over `nthr` threads with index `tid`; `sync()` separates steps.
+// Sort len keys in place (any len) with the flip bitonic network; comparators whose upper
+// index is >= len are skipped (virtual +inf padding never moves).
 template <typename Sync>
 __device__ __forceinline__ void coop_sort(unsigned long long *keys, int len, int tid, int nthr, Sync sync) {
     int S = 1;
     while (S < len) S <<= 1;
     for (int size = 2; size <= S; size <<= 1) {
+        const int half = size >> 1;
         for (int i = tid; i < S / 2; i += nthr) {
-            // i-th comparator of the flip step: block of `size`, lower half index
-            const int blk = i / (size / 2), off = i % (size / 2);
-            const int a = blk * size + off, bb = blk * size + size - 1 - off;
-            if (bb < len) {
-                unsigned long long x = keys[a], y = keys[bb];
-                if (x > y) {
-                    keys[a] = y;
-                    keys[bb] = x;
+            const int blk = i / half, o = i % half;
+            const int x = blk * size + o, y = blk * size + size - 1 - o;
+            if (y < len) {
+                const unsigned long long p = keys[x], q = keys[y];
+                if (p > q) {
+                    keys[x] = q;
+                    keys[y] = p;
                 }
             }
         }
         sync();
         for (int j = size / 4; j > 0; j >>= 1) {
             for (int i = tid; i < S / 2; i += nthr) {
-                const int blk = i / j, off = i % j;
-                const int a = blk * 2 * j + off, bb = a + j;
-                if (bb < len) {
-                    unsigned long long x = keys[a], y = keys[bb];
-                    if (x > y) {
-                        keys[a] = y;
-                        keys[bb] = x;
+                const int x = (i / j) * 2 * j + (i % j), y = x + j;
+                if (y < len) {
+                    const unsigned long long p = keys[x], q = keys[y];
+                    if (p > q) {
+                        keys[x] = q;
+                        keys[y] = p;
                     }
                 }
             }
@@ -227,317 +209,454 @@ __device__ __forceinline__ void coop_sort(unsigned long long *keys, int len, int
     }
 }
 
-// run-length merge of sorted keys into (coarse id, summed weight); threads own contiguous
-// chunks; `scan(v, total)` returns the exclusive prefix of v over the cooperating threads.
-template <typename Scan>
-__device__ __forceinline__ int32_t coop_dedup(const unsigned long long *keys, int len, int tid, int nthr,
-                                              int32_t *out_adj, int32_t *out_w, Scan scan) {
+// In-place run-length merge of sorted (cx<<32|w) keys into (cx<<32|sum) at the front of
+// `keys`.  Thread `tid` owns the contiguous chunk [lo,hi); a run crossing chunk borders is
+// completed with the leading partial sums of the following chunks (`lead`/`has` scratch of
+// nthr entries each), so no thread reads outside its own chunk after any output write.
+// `scan(v, total)` = exclusive prefix over the group.  Sums fit int32 (R14).
+template <typename Scan, typename Sync>
+__device__ __forceinline__ int32_t coop_dedup(unsigned long long *keys, int len, int tid, int nthr, int32_t *lead,
+                                              int32_t *has, Scan scan, Sync sync) {
     const int per = (len + nthr - 1) / nthr;
     const int lo = min(len, tid * per), hi = min(len, lo + per);
-    int32_t heads = 0;
-    for (int i = lo; i < hi; ++i)
-        if (i == 0 || (keys[i] >> 32) != (keys[i - 1] >> 32)) ++heads;
-    int32_t total;
-    int32_t o = scan(heads, total);
+    int32_t heads = 0, lp = 0;
+    int first_head = hi;
     for (int i = lo; i < hi; ++i) {
-        const uint32_t cx = (uint32_t)(keys[i] >> 32);
-        if (i == 0 || (keys[i - 1] >> 32) != cx) {
-            int32_t s = (int32_t)(uint32_t)keys[i];
-            for (int k = i + 1; k < len && (uint32_t)(keys[k] >> 32) == cx; ++k) s += (int32_t)(uint32_t)keys[k];
-            out_adj[o] = (int32_t)cx;
-            out_w[o] = s;
-            ++o;
+        if (i == 0 || (keys[i] >> 32) != (keys[i - 1] >> 32)) {
+            if (heads == 0) first_head = i;
+            ++heads;
+        } else if (heads == 0) {
+            lp += (int32_t)(uint32_t)keys[i];  // continues the previous chunk's run
         }
     }
+    lead[tid] = lp;
+    has[tid] = heads;
+    sync();
+    int32_t total;
+    const int32_t first_o = scan(heads, total);
+    int32_t o = first_o;
+    int i = first_head;
+    while (i < hi) {
+        const uint32_t cx = (uint32_t)(keys[i] >> 32);
+        int32_t sum = (int32_t)(uint32_t)keys[i];
+        int k = i + 1;
+        while (k < hi && (uint32_t)(keys[k] >> 32) == cx) sum += (int32_t)(uint32_t)keys[k++];
+        if (k == hi)  // run reaches my chunk's end: add the following chunks' lead partials
+            for (int t = tid + 1; t < nthr; ++t) {
+                sum += lead[t];
+                if (has[t]) break;
+            }
+        keys[o++] = ((unsigned long long)cx << 32) | (uint32_t)sum;  // o <= i: never ahead of my reads
+        i = k;
+    }
+    sync();
     return total;
 }
 
 // ---------------------------------------------------------------------------------------
-// A7, thread bin (ub <= 16) + routing of longer rows to the warp / CTA / global bins
+// C1: leftover + cmap + cvwgt + ub prefix + tile starts
 // ---------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kBlock) k_merge_small(const int32_t *__restrict__ adjp,
-                                                        const int32_t *__restrict__ adjncy,
-                                                        const int32_t *__restrict__ adjwgt,
-                                                        const int32_t *__restrict__ M,
-                                                        const int32_t *__restrict__ CM, ContractBufs b,
-                                                        LevelCtl *ctl) {
-    const int32_t nc = ctl->n_coarse;
-    const long long stride = (long long)gridDim.x * blockDim.x;
-    for (long long base = (long long)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < nc; base += stride) {
-        const long long cc = base + (threadIdx.x & 31);
-        int32_t ub = 0, s0 = 0;
-        const bool valid = cc < nc;
-        if (valid) {
-            s0 = b.off[cc];
-            ub = b.off[cc + 1] - s0;
-        }
-        warp_append(b.binW, &ctl->n_big_w, valid && ub > kNet && ub <= kWarpCap, (int32_t)cc);
-        warp_append(b.binC, &ctl->n_big_c, valid && ub > kWarpCap && ub <= kCtaCap, (int32_t)cc);
-        warp_append(b.binG, &ctl->n_big_g, valid && ub > kCtaCap, (int32_t)cc);
-        if (!valid || ub > kNet) continue;
-        const int32_t c = (int32_t)cc;
-        const int32_t u = b.leaders[c];
-        const int32_t v = M[u];
-        const int32_t su = adjp[u], du = adjp[u + 1] - su;
-        const int32_t sv = (v != u) ? adjp[v] : 0;
-        unsigned long long k[kNet];
+__device__ void phase_c1(const ContractArgs &a, ContractSmem &sm, int32_t n, int32_t ntiles2) {
+    const int ntiles = (n + kCTileV - 1) / kCTileV;
+    while (true) {
+        if (threadIdx.x == 0) sm.tile = (int32_t)atomicAdd(&a.ctl->tile_ctr[0], 1u);
+        __syncthreads();
+        const int tile = sm.tile;
+        __syncthreads();
+        if (tile >= ntiles) break;
+        const long long base = (long long)tile * kCTileV + (long long)threadIdx.x * kCItems;
+        int32_t m[kCItems];
+        int32_t d[kCItems];
+        int32_t cnt = 0, ubs = 0;
 #pragma unroll
-        for (int i = 0; i < kNet; ++i) {
-            k[i] = kMaxKey;
-            if (i < ub) {
-                const int32_t j = (i < du) ? su + i : sv + (i - du);
-                const int32_t cx = CM[__ldg(adjncy + j)];
-                if (cx != c) k[i] = ckey(cx, __ldg(adjwgt + j));  // drop the collapsed edge (R9)
-            }
-        }
-        reg_sort<kNet>(k);
-        int32_t o = 0, prev = -1, acc = 0;
-#pragma unroll
-        for (int i = 0; i < kNet; ++i) {
-            if (k[i] != kMaxKey) {
-                const int32_t cx = (int32_t)(k[i] >> 32), w = (int32_t)(uint32_t)k[i];
-                if (cx == prev) {
-                    acc += w;  // repeated coarse neighbour: weights summed (R8, P12.s28)
-                } else {
-                    if (prev >= 0) {
-                        b.tadj[s0 + o] = prev;
-                        b.tw[s0 + o] = acc;
-                        ++o;
-                    }
-                    prev = cx;
-                    acc = w;
+        for (int i = 0; i < kCItems; ++i) {
+            const long long u = base + i;
+            m[i] = -2;
+            d[i] = 0;
+            if (u < n) {
+                m[i] = a.M[u];
+                if (m[i] == kFree && a.apply_leftover) {
+                    m[i] = (int32_t)u;  // leftover: matched to itself (P18.s12-13)
+                    a.M[u] = (int32_t)u;
+                }
+                if (u <= m[i]) {  // leader flag (P18.s18, R7)
+                    ++cnt;
+                    d[i] = __ldg(a.adjp + u + 1) - __ldg(a.adjp + u);
+                    if (m[i] != u) d[i] += __ldg(a.adjp + m[i] + 1) - __ldg(a.adjp + m[i]);  // P20.s6-8
+                    ubs += d[i];
                 }
             }
         }
-        if (prev >= 0) {
-            b.tadj[s0 + o] = prev;
-            b.tw[s0 + o] = acc;
-            ++o;
+        int32_t tc, tu;
+        const int32_t ec = block_excl_scan<kCNT>(cnt, sm.scan, tc);
+        const int32_t eu = block_excl_scan<kCNT>(ubs, sm.scan, tu);
+        if (threadIdx.x < 32) {
+            const int32_t agg[2] = {tc, tu};
+            int32_t pre[2];
+            lookback<2>(a.st1, a.epoch, tile, agg, pre);
+            if (threadIdx.x == 0) {
+                sm.prefix = pre[0];
+                sm.prefix2 = (unsigned long long)(uint32_t)pre[1];
+            }
         }
-        b.cnt[c] = o;
+        __syncthreads();
+        int32_t c = sm.prefix + ec;
+        int32_t o = (int32_t)sm.prefix2 + eu;
+        if (tile == 0 && threadIdx.x == 0) a.tile_start[0] = 0;
+        if (tile == ntiles - 1 && threadIdx.x == 0) {
+            const int32_t nc = sm.prefix + tc;
+            a.ctl->n_coarse = nc;
+            a.off[nc] = (int32_t)sm.prefix2 + tu;  // = nnz
+            a.tile_start[ntiles2] = nc;
+        }
+#pragma unroll
+        for (int i = 0; i < kCItems; ++i) {
+            const long long u = base + i;
+            if (u < n && u <= m[i]) {
+                const int32_t v = m[i];
+                a.CM[u] = c;                      // exclusive scan = inclusive - 1 (P18.s20-24)
+                a.leaders[c] = (int32_t)u;
+                int32_t vw = __ldg(a.vwgt + u);
+                if (v != u) {
+                    a.CM[v] = c;                  // partner copies its leader's id (P18.s26)
+                    vw += __ldg(a.vwgt + v);      // w(c) = w(u) + w(v) (P12.s27)
+                }
+                a.cvwgt[c] = vw;
+                a.off[c] = o;
+                // tile t starts at the first row with off >= t*kTileArcs: row c+1 for every t
+                // with off[c] < t*kTileArcs <= off[c+1]
+                for (int32_t t = o / kTileArcs + 1; t <= (o + d[i]) / kTileArcs && t < ntiles2; ++t)
+                    a.tile_start[t] = c + 1;
+                if (d[i] > kTileArcs) a.huge[atomicAdd(&a.ctl->n_huge, 1)] = c;
+                ++c;
+                o += d[i];
+            }
+        }
+        __syncthreads();
     }
 }
 
-// gather the (filtered) coarse keys of row c into dst[0..len), cooperative over a group;
-// returns len.  Order of the gathered keys is irrelevant (they are sorted next).
-template <typename Count>
-__device__ __forceinline__ void gather_row(const int32_t *adjp, const int32_t *adjncy, const int32_t *adjwgt,
-                                           const int32_t *M, const int32_t *CM, const int32_t *leaders, int32_t c,
-                                           int tid, int nthr, unsigned long long *dst, Count claim) {
-    const int32_t u = leaders[c];
-    const int32_t v = M[u];
+// ---------------------------------------------------------------------------------------
+// gather the coarse keys of row c (collapsed edge dropped) into dst via claim()
+// ---------------------------------------------------------------------------------------
+template <typename Claim>
+__device__ __forceinline__ void gather_row(const ContractArgs &a, int32_t c, int tid, int nthr,
+                                           unsigned long long *dst, Claim claim) {
+    const int32_t u = __ldcg(a.leaders + c);
+    const int32_t v = __ldcg(a.M + u);
     for (int side = 0; side < (v != u ? 2 : 1); ++side) {
         const int32_t y = side ? v : u;
-        const int32_t s = adjp[y], e = adjp[y + 1];
+        const int32_t s = __ldg(a.adjp + y), e = __ldg(a.adjp + y + 1);
         for (int32_t j = s + tid; j < e; j += nthr) {
-            const int32_t cx = CM[__ldg(adjncy + j)];
-            if (cx != c) dst[claim()] = ckey(cx, __ldg(adjwgt + j));
+            const int32_t cx = __ldcg(a.CM + __ldg(a.adjncy + j));
+            if (cx != c) dst[claim()] = ckey(cx, __ldg(a.adjwgt + j));  // drop the collapsed edge (R9)
         }
     }
 }
 
+// C1b: rows whose upper bound exceeds a tile: one CTA per row in global scratch
+__device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
+    for (int i = blockIdx.x; i < nh; i += gridDim.x) {
+        const int32_t c = a.huge[i];
+        unsigned long long *keys = a.gkeys + __ldcg(a.off + c);
+        if (threadIdx.x == 0) sm.len = 0;
+        __syncthreads();
+        gather_row(a, c, threadIdx.x, kCNT, keys, [&]() { return atomicAdd(&sm.len, 1); });
+        __syncthreads();
+        const int len = sm.len;
+        coop_sort(keys, len, threadIdx.x, kCNT, []() { __syncthreads(); });
+        const int32_t cnt = coop_dedup(
+            keys, len, threadIdx.x, kCNT, sm.lead, sm.has,
+            [&](int32_t v, int32_t &tot) { return block_excl_scan<kCNT>(v, sm.scan, tot); },
+            []() { __syncthreads(); });
+        if (threadIdx.x == 0) a.cnt[c] = cnt;
+        __syncthreads();
+    }
+}
+
 // ---------------------------------------------------------------------------------------
-// A7, warp bin (16 < ub <= 256): one warp per row, keys in shared memory
+// C2: tiled merge + assembly
 // ---------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kBlock) k_merge_warp(const int32_t *__restrict__ adjp,
-                                                       const int32_t *__restrict__ adjncy,
-                                                       const int32_t *__restrict__ adjwgt,
-                                                       const int32_t *__restrict__ M,
-                                                       const int32_t *__restrict__ CM, ContractBufs b,
-                                                       LevelCtl *ctl) {
-    __shared__ unsigned long long s_keys[kBlock / 32][kWarpCap];
-    __shared__ int32_t s_len[kBlock / 32];
+__device__ void phase_c2(const ContractArgs &a, ContractSmem &sm, int32_t nc, int32_t nnz, int32_t ntiles2) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    const int nW = ctl->n_big_w;
-    unsigned long long *keys = s_keys[wib];
-    for (int i = blockIdx.x * (kBlock / 32) + wib; i < nW; i += gridDim.x * (kBlock / 32)) {
-        const int32_t c = b.binW[i];
-        if (lane == 0) s_len[wib] = 0;
-        __syncwarp();
-        gather_row(adjp, adjncy, adjwgt, M, CM, b.leaders, c, lane, 32, keys,
-                   [&]() { return atomicAdd(&s_len[wib], 1); });
-        __syncwarp();
-        const int len = s_len[wib];
-        coop_sort(keys, len, lane, 32, []() { __syncwarp(); });
-        const int32_t s0 = b.off[c];
-        int32_t o = coop_dedup(keys, len, lane, 32, b.tadj + s0, b.tw + s0, [&](int32_t v, int32_t &tot) {
-            int32_t inc = warp_incl_scan(v);
-            tot = __shfl_sync(0xffffffffu, inc, 31);
-            return inc - v;
-        });
-        if (lane == 0) b.cnt[c] = o;
-        __syncwarp();
+    while (true) {
+        if (threadIdx.x == 0) sm.tile = (int32_t)atomicAdd(&a.ctl->tile_ctr[1], 1u);
+        __syncthreads();
+        const int tile = sm.tile;
+        __syncthreads();
+        if (tile >= ntiles2) break;
+        const int32_t r0 = __ldcg(a.tile_start + tile), r1 = __ldcg(a.tile_start + tile + 1);
+        const int32_t tbase = tile * kTileArcs;
+        // ---- pass 1: merge every row of the tile into its shared-memory slot, count ----
+        int32_t total = 0;
+        for (int32_t g0 = r0; g0 < r1; g0 += kCNT) {
+            const int32_t c = g0 + threadIdx.x;
+            int32_t ub = 0, slot = 0, cntc = 0;
+            bool warp_row = false;
+            if (c < r1) {
+                slot = __ldcg(a.off + c) - tbase;
+                ub = __ldcg(a.off + c + 1) - __ldcg(a.off + c);
+                if (ub > kTileArcs) {
+                    cntc = __ldcg(a.cnt + c);  // merged by C1b
+                } else if (ub > kNet) {
+                    warp_row = true;
+                } else if (ub > 0) {
+                    const int32_t u = __ldcg(a.leaders + c);
+                    const int32_t v = __ldcg(a.M + u);
+                    const int32_t su = __ldg(a.adjp + u), du = __ldg(a.adjp + u + 1) - su;
+                    const int32_t sv = (v != u) ? __ldg(a.adjp + v) : 0;
+                    unsigned long long k[kNet];
+#pragma unroll
+                    for (int i = 0; i < kNet; ++i) {
+                        k[i] = kMaxKey;
+                        if (i < ub) {
+                            const int32_t j = (i < du) ? su + i : sv + (i - du);
+                            const int32_t cx = __ldcg(a.CM + __ldg(a.adjncy + j));
+                            if (cx != c) k[i] = ckey(cx, __ldg(a.adjwgt + j));
+                        }
+                    }
+                    reg_sort<kNet>(k);
+                    int32_t prev = -1, acc = 0;
+#pragma unroll
+                    for (int i = 0; i < kNet; ++i) {
+                        if (k[i] != kMaxKey) {
+                            const int32_t cx = (int32_t)(k[i] >> 32), w = (int32_t)(uint32_t)k[i];
+                            if (cx == prev) {
+                                acc += w;  // repeated coarse neighbour: weights summed (R8, P12.s28)
+                            } else {
+                                if (prev >= 0) sm.buf[slot + cntc++] = ckey(prev, acc);
+                                prev = cx;
+                                acc = w;
+                            }
+                        }
+                    }
+                    if (prev >= 0) sm.buf[slot + cntc++] = ckey(prev, acc);
+                }
+            }
+            // rows longer than kNet: one warp each, in their shared-memory slot
+            unsigned mm = __ballot_sync(0xffffffffu, warp_row);
+            while (mm) {
+                const int src = __ffs(mm) - 1;
+                mm &= mm - 1;
+                const int32_t cw = __shfl_sync(0xffffffffu, c, src);
+                const int32_t sl = __shfl_sync(0xffffffffu, slot, src);
+                unsigned long long *keys = sm.buf + sl;
+                if (lane == 0) sm.wlen[wib] = 0;
+                __syncwarp();
+                gather_row(a, cw, lane, 32, keys, [&]() { return atomicAdd(&sm.wlen[wib], 1); });
+                __syncwarp();
+                const int len = sm.wlen[wib];
+                coop_sort(keys, len, lane, 32, []() { __syncwarp(); });
+                const int32_t cc = coop_dedup(
+                    keys, len, lane, 32, sm.lead + wib * 32, sm.has + wib * 32,
+                    [&](int32_t v, int32_t &tot) {
+                        const int32_t inc = warp_incl_scan(v);
+                        tot = __shfl_sync(0xffffffffu, inc, 31);
+                        return inc - v;
+                    },
+                    []() { __syncwarp(); });
+                if (lane == src) cntc = cc;
+            }
+            if (c < r1) a.cnt[c] = cntc;
+            int32_t part;
+            block_excl_scan<kCNT>(cntc, sm.scan, part);
+            total += part;
+        }
+        // ---- tile prefix by decoupled look-back ----
+        if (threadIdx.x < 32) {
+            const int32_t agg[1] = {total};
+            int32_t pre[1];
+            lookback<1>(a.st2, a.epoch, tile, agg, pre);
+            if (threadIdx.x == 0) sm.prefix = pre[0];
+        }
+        __syncthreads();
+        int32_t pos0 = sm.prefix;
+        if (tile == ntiles2 - 1 && threadIdx.x == 0) {
+            a.cadjp[nc] = pos0 + total;
+            a.ctl->cnnz = pos0 + total;
+        }
+        // ---- pass 2: cadjp and the rows, straight into the final arrays ----
+        for (int32_t g0 = r0; g0 < r1; g0 += kCNT) {
+            const int32_t c = g0 + threadIdx.x;
+            int32_t cntc = 0, ub = 0, slot = 0, o = 0;
+            if (c < r1) {
+                cntc = __ldcg(a.cnt + c);
+                slot = __ldcg(a.off + c) - tbase;
+                ub = __ldcg(a.off + c + 1) - __ldcg(a.off + c);
+            }
+            int32_t part;
+            const int32_t ex = block_excl_scan<kCNT>(cntc, sm.scan, part);
+            o = pos0 + ex;
+            if (c < r1) {
+                a.cadjp[c] = o;
+                if (ub <= kTileArcs) {
+                    for (int32_t j = 0; j < cntc; ++j) {
+                        const unsigned long long k = sm.buf[slot + j];
+                        a.cadjncy[o + j] = (int32_t)(k >> 32);
+                        a.cadjwgt[o + j] = (int32_t)(uint32_t)k;
+                    }
+                }
+            }
+            // a row merged by C1b (at most one per tile, its last row): copied by the CTA
+            if (threadIdx.x == 0) sm.hub_c = -1;
+            __syncthreads();
+            if (c < r1 && ub > kTileArcs) {
+                sm.hub_c = c;
+                sm.hub_o = o;
+            }
+            __syncthreads();
+            if (sm.hub_c >= 0) {
+                const int32_t hc = sm.hub_c, oc = sm.hub_o;
+                const unsigned long long *src = a.gkeys + __ldcg(a.off + hc);
+                const int32_t k = __ldcg(a.cnt + hc);
+                for (int32_t j = threadIdx.x; j < k; j += kCNT) {
+                    const unsigned long long kk = src[j];
+                    a.cadjncy[oc + j] = (int32_t)(kk >> 32);
+                    a.cadjwgt[oc + j] = (int32_t)(uint32_t)kk;
+                }
+            }
+            pos0 += part;
+        }
+        __syncthreads();
     }
 }
 
-// ---------------------------------------------------------------------------------------
-// A7, CTA bin (256 < ub <= 8192): one CTA per row, keys in (dynamic) shared memory
-// A7, global bin (ub > 8192, hubs): one CTA per row, keys in global scratch
-// ---------------------------------------------------------------------------------------
-template <bool kGlobal>
-__global__ void __launch_bounds__(kBlock) k_merge_cta(const int32_t *__restrict__ adjp,
-                                                      const int32_t *__restrict__ adjncy,
-                                                      const int32_t *__restrict__ adjwgt,
-                                                      const int32_t *__restrict__ M,
-                                                      const int32_t *__restrict__ CM, ContractBufs b,
-                                                      LevelCtl *ctl) {
-    extern __shared__ unsigned long long s_dyn[];
-    __shared__ int32_t s_scan[33];
-    __shared__ int32_t s_len;
-    const int nB = kGlobal ? ctl->n_big_g : ctl->n_big_c;
-    const int32_t *bin = kGlobal ? b.binG : b.binC;
-    for (int i = blockIdx.x; i < nB; i += gridDim.x) {
-        const int32_t c = bin[i];
-        const int32_t s0 = b.off[c];
-        unsigned long long *keys = kGlobal ? (b.gkeys + s0) : s_dyn;
-        if (threadIdx.x == 0) s_len = 0;
-        __syncthreads();
-        gather_row(adjp, adjncy, adjwgt, M, CM, b.leaders, c, threadIdx.x, kBlock, keys,
-                   [&]() { return atomicAdd(&s_len, 1); });
-        __syncthreads();
-        const int len = s_len;
-        coop_sort(keys, len, threadIdx.x, kBlock, []() { __syncthreads(); });
-        int32_t o = coop_dedup(keys, len, threadIdx.x, kBlock, b.tadj + s0, b.tw + s0,
-                               [&](int32_t v, int32_t &tot) { return block_excl_scan<kBlock>(v, s_scan, tot); });
-        if (threadIdx.x == 0) b.cnt[c] = o;
-        __syncthreads();
+__global__ void __launch_bounds__(kCNT, 2) k_contract_level(const __grid_constant__ ContractArgs a) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    ContractSmem &sm = *reinterpret_cast<ContractSmem *>(smem_raw);
+    ContractCtl *ctl = a.ctl;
+    const volatile SizeRec *in = a.in;
+    if (in->stop) {  // an earlier level ended the coarsening: propagate and leave
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            a.out->n = in->n;
+            a.out->nnz = in->nnz;
+            a.out->stop = 1;
+            a.out->stop_reason = in->stop_reason;
+            if (a.report) {
+                a.report->skipped = 1;
+                __threadfence_system();
+                *((volatile int32_t *)&a.report->ready) = 1;
+            }
+        }
+        return;
     }
-}
-
-// ---------------------------------------------------------------------------------------
-// A8 compaction: merged rows from the temporary arrays into the final coarse CSR
-// (P20.s22-24); G lanes per row.
-// ---------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kBlock) k_compact(const int32_t *__restrict__ off, const int32_t *__restrict__ cnt,
-                                                    const int32_t *__restrict__ cadjp,
-                                                    const int32_t *__restrict__ tadj, const int32_t *__restrict__ tw,
-                                                    int32_t *__restrict__ cadjncy, int32_t *__restrict__ cadjwgt,
-                                                    LevelCtl *ctl) {
-    constexpr int G = 8;
-    const int32_t nc = ctl->n_coarse;
-    const long long gid = ((long long)blockIdx.x * blockDim.x + threadIdx.x) / G;
-    const int gl = threadIdx.x % G;
-    const long long ng = ((long long)gridDim.x * blockDim.x) / G;
-    for (long long c = gid; c < nc; c += ng) {
-        const int32_t s = off[c], d = cadjp[c], k = cnt[c];
-        for (int32_t j = gl; j < k; j += G) {
-            cadjncy[d + j] = tadj[s + j];
-            cadjwgt[d + j] = tw[s + j];
+    const int32_t n = in->n;
+    const int32_t nnz = in->nnz;
+    const int32_t ntiles2 = nnz > 0 ? (nnz + kTileArcs - 1) / kTileArcs : 0;
+    if (n > 0) {
+        phase_c1(a, sm, n, ntiles2);
+        grid_barrier(ctl->bar);
+    }
+    const int32_t nc = *(volatile int32_t *)&ctl->n_coarse;
+    const int32_t nh = *(volatile int32_t *)&ctl->n_huge;
+    if (nh > 0) {
+        phase_c1b(a, sm, nh);
+        grid_barrier(ctl->bar);
+    }
+    if (ntiles2 > 0) phase_c2(a, sm, nc, nnz, ntiles2);
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        if (ntiles2 == 0) {
+            a.cadjp[nc] = 0;
+            ctl->cnnz = 0;
+        }
+    }
+    // the last CTA to finish publishes the coarse sizes and the stop decision
+    __shared__ bool last;
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) last = atomicAdd(&ctl->blocks_done, 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (last && threadIdx.x == 0) {
+        __threadfence();
+        const int32_t ncv = *((volatile int32_t *)&ctl->n_coarse);
+        const int32_t cnnz = *((volatile int32_t *)&ctl->cnnz);
+        // stop rule (P12.s30, P20.s30; R12, R13): stall first, then threshold, then levels
+        int32_t reason = GP_STOP_NONE;
+        if (100LL * ncv > (long long)a.stall_pct * n) reason = GP_STOP_STALL;
+        else if (ncv <= a.threshold) reason = GP_STOP_THRESHOLD;
+        else if (a.level + 1 >= a.max_levels) reason = GP_STOP_MAX_LEVELS;
+        a.out->n = ncv;
+        a.out->nnz = cnnz;
+        a.out->stop = reason != GP_STOP_NONE;
+        a.out->stop_reason = reason;
+        __threadfence();
+        if (a.report) {
+            a.report->n_coarse = ncv;
+            a.report->cnnz = cnnz;
+            a.report->stop = reason != GP_STOP_NONE;
+            a.report->stop_reason = reason;
+            a.report->skipped = 0;
+            __threadfence_system();
+            *((volatile int32_t *)&a.report->ready) = 1;
         }
     }
 }
 
 // ---------------------------------------------------------------------------------------
-// host driver of one contraction
+// host side
 // ---------------------------------------------------------------------------------------
-static uint32_t next_epoch(Ctx *ctx) {
-    uint32_t e = ctx->epoch;
-    ctx->epoch = (ctx->epoch + 1) & 0x3FFFFFFFu;
+int contract_grid(Ctx *ctx) {
+    static int per_sm = -1;
+    if (per_sm < 0) {
+        int b = 0;
+        cudaFuncSetAttribute(k_contract_level, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)sizeof(ContractSmem));
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_contract_level, kCNT, sizeof(ContractSmem));
+        per_sm = b > 0 ? (b > 2 ? 2 : b) : 1;
+    }
+    return ctx->num_sms * per_sm;
+}
+
+size_t contract_status_words(int32_t n, int32_t nnz) {
+    const size_t t1 = (size_t)(n + kCTileV - 1) / kCTileV + 1;
+    const size_t t2 = (size_t)(nnz + kTileArcs - 1) / kTileArcs + 1;
+    return 4 * t1 + 2 * t2;
+}
+
+size_t contract_tiles(int32_t nnz) { return (size_t)(nnz + kTileArcs - 1) / kTileArcs + 2; }
+
+gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *CM, Graph *cg, ContractCtl *ctl,
+                           SizeRec *out_sizes, LevelReport *report, const ContractParams &prm) {
+    ContractArgs a;
+    a.in = lb.in;
+    a.adjp = lb.adjp;
+    a.adjncy = lb.adjncy;
+    a.adjwgt = lb.adjwgt;
+    a.vwgt = lb.vwgt;
+    a.M = M;
+    a.CM = CM;
+    a.leaders = lb.leaders;
+    a.off = lb.off;
+    a.cnt = lb.cnt;
+    a.tile_start = lb.tile_start;
+    a.huge = lb.huge;
+    a.gkeys = lb.gkeys;
+    a.st1 = ctx->status;
+    a.st2 = ctx->status + 4 * ((size_t)(prm.n_bound + kCTileV - 1) / kCTileV + 1);
+    a.epoch = ctx->epoch;
+    ctx->epoch = (ctx->epoch + 1) & 0x7FFFFFFFu;
     if (ctx->epoch == 0) ctx->epoch = 1;
-    return e;
-}
-
-gp_status contract_level(Ctx *ctx, const Graph *g, int32_t *M, int32_t *CM, bool apply_leftover,
-                         Graph **coarse_out) {
-    *coarse_out = nullptr;
-    const int32_t n = g->n, nnz = g->nnz;
-    const size_t nn = (size_t)n;
-    const size_t ints = 7 * nn + 4 + 2 * (size_t)nnz;
-    const size_t bytes = ((ints * 4 + 15) / 16) * 16 + 8 * (size_t)nnz;
-    gp_status st = ensure_scratch(ctx, bytes);
+    a.cadjp = cg->adjp;
+    a.cadjncy = cg->adjncy;
+    a.cadjwgt = cg->adjwgt;
+    a.cvwgt = cg->vwgt;
+    a.ctl = ctl;
+    a.out = out_sizes;
+    a.apply_leftover = prm.leftover ? 1 : 0;
+    a.threshold = prm.threshold;
+    a.stall_pct = prm.stall_pct;
+    a.level = prm.level;
+    a.max_levels = prm.max_levels;
+    a.report = report;
+    gp_status st = ensure_status(ctx, contract_status_words(prm.n_bound, prm.nnz_bound));
     if (st != GP_OK) return st;
-    st = ensure_status(ctx, nn / kTile + 2);
-    if (st != GP_OK) return st;
-    int32_t *p = (int32_t *)ctx->scratch;
-    ContractBufs b;
-    b.leaders = p; p += nn;
-    b.ub = p; p += nn + 1;
-    b.off = p; p += nn + 1;
-    b.cnt = p; p += nn;
-    b.binW = p; p += nn;
-    b.binC = p; p += nn;
-    b.binG = p; p += nn;
-    b.tadj = p; p += nnz;
-    b.tw = p; p += nnz;
-    b.gkeys = (unsigned long long *)((char *)ctx->scratch + ((ints * 4 + 15) / 16) * 16);
-
-    Graph *cg = new Graph();
-    cg->ctx = ctx;
-    st = dev_alloc(ctx, (void **)&cg->adjp, sizeof(int32_t) * (nn + 1));
-    if (st == GP_OK) st = dev_alloc(ctx, (void **)&cg->vwgt, sizeof(int32_t) * (nn > 0 ? nn : 1));
-    if (st == GP_OK) st = dev_alloc(ctx, (void **)&cg->adjncy, sizeof(int32_t) * (nnz > 0 ? nnz : 1));
-    if (st == GP_OK) st = dev_alloc(ctx, (void **)&cg->adjwgt, sizeof(int32_t) * (nnz > 0 ? nnz : 1));
-    if (st != GP_OK) {
-        dev_free(ctx, cg->adjp);
-        dev_free(ctx, cg->vwgt);
-        dev_free(ctx, cg->adjncy);
-        dev_free(ctx, cg->adjwgt);
-        delete cg;
-        return st;
-    }
-
-    LevelCtl *ctl = ctx->ctl;
-    cudaStream_t s = ctx->stream;
-    GP_CUDA(cudaMemsetAsync(ctl, 0, sizeof(LevelCtl), s));
-    const int grid = persistent_grid(ctx, ctx->max_threads_sm / kBlock);
-    if (n > 0) {
-        LaunchScope ls(ctx, GP_K_CMAP);
-        k_cmap_scan<<<grid, kBlock, 0, s>>>(n, g->adjp, g->vwgt, M, CM, b, cg->vwgt, ctx->status, next_epoch(ctx),
-                                            ctl, apply_leftover ? 1 : 0);
-        ++ctx->launches;
-    }
-    {
-        LaunchScope ls(ctx, GP_K_ASSEMBLE);
-        k_scan_excl<<<grid, kBlock, 0, s>>>(b.ub, b.off, &ctl->n_coarse, nullptr, ctx->status, next_epoch(ctx),
-                                            &ctl->tile_ctr[1]);
-        ++ctx->launches;
-    }
-    {
-        LaunchScope ls(ctx, GP_K_CONTRACT);
-        k_merge_small<<<grid, kBlock, 0, s>>>(g->adjp, g->adjncy, g->adjwgt, M, CM, b, ctl);
-        ++ctx->launches;
-    }
-    {
-        LaunchScope ls(ctx, GP_K_CONTRACT);
-        k_merge_warp<<<grid, kBlock, 0, s>>>(g->adjp, g->adjncy, g->adjwgt, M, CM, b, ctl);
-        ++ctx->launches;
-    }
-    {
-        LaunchScope ls(ctx, GP_K_CONTRACT);
-        const size_t smem = sizeof(unsigned long long) * kCtaCap;
-        k_merge_cta<false><<<persistent_grid(ctx, 2), kBlock, smem, s>>>(g->adjp, g->adjncy, g->adjwgt, M, CM, b,
-                                                                         ctl);
-        ++ctx->launches;
-    }
-    {
-        LaunchScope ls(ctx, GP_K_CONTRACT);
-        k_merge_cta<true><<<persistent_grid(ctx, 2), kBlock, 0, s>>>(g->adjp, g->adjncy, g->adjwgt, M, CM, b, ctl);
-        ++ctx->launches;
-    }
-    {
-        LaunchScope ls(ctx, GP_K_ASSEMBLE);
-        k_scan_excl<<<grid, kBlock, 0, s>>>(b.cnt, cg->adjp, &ctl->n_coarse, &ctl->cnnz, ctx->status,
-                                            next_epoch(ctx), &ctl->tile_ctr[2]);
-        ++ctx->launches;
-    }
-    {
-        LaunchScope ls(ctx, GP_K_ASSEMBLE);
-        k_compact<<<grid, kBlock, 0, s>>>(b.off, b.cnt, cg->adjp, b.tadj, b.tw, cg->adjncy, cg->adjwgt, ctl);
-        ++ctx->launches;
-    }
-    GP_CUDA(cudaGetLastError());
-    GP_CUDA(cudaMemcpyAsync(ctx->ctl_host, ctl, sizeof(LevelCtl), cudaMemcpyDeviceToHost, s));
-    GP_CUDA(cudaStreamSynchronize(s));
-    cg->n = ctx->ctl_host->n_coarse;
-    cg->nnz = ctx->ctl_host->cnnz;
-    *coarse_out = cg;
-    return GP_OK;
-}
-
-gp_status contract_set_attributes() {
-    cudaError_t e = cudaFuncSetAttribute(k_merge_cta<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)(sizeof(unsigned long long) * kCtaCap));
-    if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(k_merge_cta)");
+    a.st1 = ctx->status;
+    a.st2 = ctx->status + 4 * ((size_t)(prm.n_bound + kCTileV - 1) / kCTileV + 1);
+    void *args[] = {&a};
+    LaunchScope ls(ctx, GP_K_CONTRACT);
+    GP_CUDA(cudaLaunchCooperativeKernel((const void *)k_contract_level, dim3(contract_grid(ctx)), dim3(kCNT), args,
+                                        sizeof(ContractSmem), ctx->stream));
+    ++ctx->launches;
     return GP_OK;
 }
 

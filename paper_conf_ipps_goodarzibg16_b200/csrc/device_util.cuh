@@ -10,6 +10,13 @@ namespace gp {
 
 __device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31u; }
 
+// Watchdog of every spin loop: a protocol bug traps (cudaErrorLaunchFailure) after ~4 s
+// instead of hanging the device.
+__device__ __forceinline__ long long spin_start() { return clock64(); }
+__device__ __forceinline__ void spin_check(long long t0) {
+    if (clock64() - t0 > (8ll << 30)) __trap();
+}
+
 __device__ __forceinline__ unsigned lanemask_lt() {
     unsigned m;
     asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -124,7 +131,9 @@ __device__ __forceinline__ int32_t lookback_prefix(unsigned long long *status, u
         uint32_t flag = 2, val = 0;
         if (idx >= 0) {
             unsigned long long s;
+            const long long guard = spin_start();
             do {
+                spin_check(guard);
                 s = lb_load(status + idx);
                 flag = ((uint32_t)(s >> 32) >> 2) == epoch ? ((uint32_t)(s >> 32) & 3u) : 0u;
             } while (flag == 0);
@@ -147,6 +156,115 @@ __device__ __forceinline__ int32_t lookback_prefix(unsigned long long *status, u
     }
     if (l == 0) lb_store(status + tile, tagP | (uint32_t)(prefix + aggregate));
     return prefix;
+}
+
+}  // namespace gp
+
+namespace gp {
+
+// ---------------------------------------------------------------------------------------
+// Grid-wide barrier of a cooperative (co-resident) launch.  `bar[0]` arrival count,
+// `bar[1]` generation.  One arrival per CTA; the last arrival resets the count and bumps
+// the generation with release semantics; the others spin with acquire loads.
+// ---------------------------------------------------------------------------------------
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_u32(unsigned *p, unsigned v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned atom_add_acqrel_u32(unsigned *p, unsigned v) {
+    unsigned old;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
+
+__device__ __forceinline__ void grid_barrier(unsigned *bar) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const unsigned gen = ld_acquire_u32(bar + 1);
+        __threadfence();
+        if (atom_add_acqrel_u32(bar, 1u) == gridDim.x - 1) {
+            bar[0] = 0;
+            st_release_u32(bar + 1, gen + 1);
+        } else {
+            const long long guard = spin_start();
+            while (ld_acquire_u32(bar + 1) == gen) {
+                __nanosleep(32);
+                spin_check(guard);
+            }
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+// ---------------------------------------------------------------------------------------
+// Block-aggregated append: the predicated threads of the CTA append `value` to list[] with
+// ONE global atomic per CTA call (all threads must call; smem >= NT/32 + 2 ints).
+// ---------------------------------------------------------------------------------------
+template <int NT>
+__device__ __forceinline__ void block_append(int32_t *list, int32_t *counter, bool pred, int32_t value,
+                                             int32_t *smem) {
+    constexpr int NW = NT / 32;
+    const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+    const unsigned m = __ballot_sync(0xffffffffu, pred);
+    if (l == 0) smem[w] = __popc(m);
+    __syncthreads();
+    if (w == 0) {
+        int32_t x = (l < NW) ? smem[l] : 0;
+        int32_t xi = warp_incl_scan(x);
+        int32_t tot = __shfl_sync(0xffffffffu, xi, 31);
+        int32_t base = 0;
+        if (l == 0 && tot > 0) base = atomicAdd(counter, tot);
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (l < NW) smem[l] = base + xi - x;
+    }
+    __syncthreads();
+    if (pred) list[smem[w] + __popc(m & lanemask_lt())] = value;
+    __syncthreads();
+}
+
+// ---------------------------------------------------------------------------------------
+// TMA 1D bulk copy global -> shared, completion tracked by an mbarrier (sm_90+ / sm_100a)
+// ---------------------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_addr(const void *p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t *bar, unsigned parity) {
+    unsigned ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_addr(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned parity) {
+    const long long guard = spin_start();
+    while (!mbar_try_wait(bar, parity)) spin_check(guard);
+}
+// bytes must be a multiple of 16; src and dst 16-byte aligned
+__device__ __forceinline__ void tma_load_1d(void *dst, const void *src, unsigned bytes, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_addr(dst)),
+        "l"(src), "r"(bytes), "r"(smem_addr(bar))
+        : "memory");
 }
 
 }  // namespace gp

@@ -2,6 +2,9 @@
 // level driver gp_coarsen_to (A9: P10.s16, P20.s27-31, P12.s30; readings R12, R13).
 #include <cuda_runtime.h>
 
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -10,7 +13,6 @@
 
 namespace gp {
 
-gp_status contract_set_attributes();
 gp_status fill_ones(Ctx *ctx, int32_t *p, long long len);
 
 static thread_local std::string g_last_error;
@@ -122,6 +124,7 @@ static void graph_release(Graph *g) {
     dev_free(ctx, g->adjncy);
     dev_free(ctx, g->adjwgt);
     dev_free(ctx, g->vwgt);
+    if (g->owns_sizes) dev_free(ctx, g->sizes);
     g->tag = 0;
     delete g;
 }
@@ -133,8 +136,50 @@ static void hier_release(Hier *h) {
         dev_free(h->ctx, l.cmap);
         graph_release(l.coarse);
     }
+    dev_free(h->ctx, h->levdev);
     h->tag = 0;
     delete h;
+}
+
+// graph arrays with 4 ints of padding (TMA bulk copies round ranges up to 16 bytes)
+static gp_status alloc_graph_arrays(Ctx *ctx, Graph *g, int32_t n_bound, int32_t nnz_bound, bool own_sizes) {
+    gp_status st = dev_alloc(ctx, (void **)&g->adjp, sizeof(int32_t) * ((size_t)n_bound + 4));
+    if (st == GP_OK) st = dev_alloc(ctx, (void **)&g->vwgt, sizeof(int32_t) * ((size_t)n_bound + 4));
+    if (st == GP_OK) st = dev_alloc(ctx, (void **)&g->adjncy, sizeof(int32_t) * ((size_t)nnz_bound + 4));
+    if (st == GP_OK) st = dev_alloc(ctx, (void **)&g->adjwgt, sizeof(int32_t) * ((size_t)nnz_bound + 4));
+    g->owns_sizes = own_sizes;
+    if (st == GP_OK && own_sizes) st = dev_alloc(ctx, (void **)&g->sizes, sizeof(SizeRec));
+    return st;
+}
+
+gp_status level_scratch(Ctx *ctx, int32_t n, int32_t nnz, LevelBufs *lb) {
+    const size_t nn = (size_t)(n > 0 ? n : 1);
+    const size_t tiles = contract_tiles(nnz);
+    const size_t ints = 9 * nn + 1 + tiles + 8;
+    const size_t ibytes = ((ints * 4 + 255) / 256) * 256;
+    gp_status st = ensure_scratch(ctx, ibytes + 8 * ((size_t)nnz + 4));
+    if (st != GP_OK) return st;
+    int32_t *p = (int32_t *)ctx->scratch;
+    lb->P[0] = p; p += nn;
+    lb->P[1] = p; p += nn;
+    lb->L[0] = p; p += nn;
+    lb->L[1] = p; p += nn;
+    lb->H = p; p += nn;
+    lb->leaders = p; p += nn;
+    lb->off = p; p += nn + 1;
+    lb->cnt = p; p += nn;
+    lb->huge = p; p += nn;
+    lb->tile_start = p; p += tiles + 8;
+    lb->gkeys = (unsigned long long *)((char *)ctx->scratch + ibytes);
+    return GP_OK;
+}
+
+static void set_graph_bufs(LevelBufs *lb, const Graph *g) {
+    lb->in = g->sizes;
+    lb->adjp = g->adjp;
+    lb->adjncy = g->adjncy;
+    lb->adjwgt = g->adjwgt;
+    lb->vwgt = g->vwgt;
 }
 
 template <typename T>
@@ -197,6 +242,10 @@ gp_status gp_ctx_create(int device, void *cuda_stream, gp_ctx *out) {
                   ", this library is built for sm_100a");
         return GP_ERR_CUDA;
     }
+    if (!prop.cooperativeLaunch) {
+        set_error("gp_ctx_create: device does not support cooperative launches");
+        return GP_ERR_CUDA;
+    }
     Ctx *ctx = new Ctx();
     ctx->device = device;
     ctx->stream = (cudaStream_t)cuda_stream;
@@ -208,11 +257,17 @@ gp_status gp_ctx_create(int device, void *cuda_stream, gp_ctx *out) {
         uint64_t thr = UINT64_MAX;
         cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
     }
-    gp_status st = contract_set_attributes();
-    if (st == GP_OK) st = dev_alloc(ctx, (void **)&ctx->ctl, sizeof(LevelCtl));
+    gp_status st = GP_OK;
+    cudaError_t e = cudaHostAlloc((void **)&ctx->pinned, 4096, cudaHostAllocDefault);
+    if (e != cudaSuccess) st = cuda_fail(e, "cudaHostAlloc(pinned)");
     if (st == GP_OK) {
-        cudaError_t e = cudaMallocHost((void **)&ctx->ctl_host, sizeof(LevelCtl));
-        if (e != cudaSuccess) st = cuda_fail(e, "cudaMallocHost");
+        ctx->max_reports = 256;
+        e = cudaHostAlloc((void **)&ctx->reports, sizeof(LevelReport) * ctx->max_reports, cudaHostAllocMapped);
+        if (e != cudaSuccess) st = cuda_fail(e, "cudaHostAlloc(mapped reports)");
+    }
+    if (st == GP_OK) {
+        e = cudaHostGetDevicePointer((void **)&ctx->reports_dev, ctx->reports, 0);
+        if (e != cudaSuccess) st = cuda_fail(e, "cudaHostGetDevicePointer");
     }
     if (st != GP_OK) {
         gp_free(ctx);
@@ -232,16 +287,14 @@ gp_status gp_ctx_set_allocator(gp_ctx ctx, gp_alloc_fn alloc, gp_dealloc_fn deal
     cudaStreamSynchronize(ctx->stream);
     dev_free(ctx, ctx->scratch);
     dev_free(ctx, ctx->status);
-    dev_free(ctx, ctx->ctl);
     ctx->scratch = nullptr;
     ctx->scratch_bytes = 0;
     ctx->status = nullptr;
     ctx->status_words = 0;
-    ctx->ctl = nullptr;
     ctx->alloc = alloc;
     ctx->dealloc = dealloc;
     ctx->alloc_user = user;
-    return dev_alloc(ctx, (void **)&ctx->ctl, sizeof(LevelCtl));
+    return GP_OK;
 }
 
 gp_status gp_ctx_num_sms(gp_ctx ctx, int32_t *out) {
@@ -254,7 +307,7 @@ gp_status gp_graph_create(gp_ctx ctx, gp_vid n, const gp_vid *adjp, const gp_vid
                           const gp_wgt *vwgt, uint32_t flags, gp_graph *out) {
     if (out) *out = nullptr;
     if (!tagged<Ctx>(ctx, kTagCtx) || !out || n < 0 || !adjp) {
-        set_error("gp_graph_create: bad context, output or n");
+        set_error("gp_graph_create: bad context, output, n or adjp");
         return GP_ERR_INVALID_ARG;
     }
     GP_TRY_BEGIN
@@ -263,10 +316,9 @@ gp_status gp_graph_create(gp_ctx ctx, gp_vid n, const gp_vid *adjp, const gp_vid
     GP_CUDA(cudaSetDevice(ctx->device));
     int32_t nnz = 0;
     if (dev) {
-        GP_CUDA(cudaMemcpyAsync(&ctx->ctl_host->pad[0], adjp + n, sizeof(int32_t), cudaMemcpyDeviceToHost,
-                                ctx->stream));
+        GP_CUDA(cudaMemcpyAsync(ctx->pinned, adjp + n, sizeof(int32_t), cudaMemcpyDeviceToHost, ctx->stream));
         GP_CUDA(cudaStreamSynchronize(ctx->stream));
-        nnz = ctx->ctl_host->pad[0];
+        nnz = ctx->pinned[0];
     } else {
         nnz = adjp[n];
     }
@@ -282,10 +334,7 @@ gp_status gp_graph_create(gp_ctx ctx, gp_vid n, const gp_vid *adjp, const gp_vid
     g->ctx = ctx;
     g->n = n;
     g->nnz = nnz;
-    gp_status st = dev_alloc(ctx, (void **)&g->adjp, sizeof(int32_t) * ((size_t)n + 1));
-    if (st == GP_OK) st = dev_alloc(ctx, (void **)&g->adjncy, sizeof(int32_t) * (size_t)nnz);
-    if (st == GP_OK) st = dev_alloc(ctx, (void **)&g->adjwgt, sizeof(int32_t) * (size_t)nnz);
-    if (st == GP_OK) st = dev_alloc(ctx, (void **)&g->vwgt, sizeof(int32_t) * (size_t)n);
+    gp_status st = alloc_graph_arrays(ctx, g, n, nnz, true);
     cudaError_t e = cudaSuccess;
     if (st == GP_OK) e = cudaMemcpyAsync(g->adjp, adjp, sizeof(int32_t) * ((size_t)n + 1), kind, ctx->stream);
     if (st == GP_OK && e == cudaSuccess && nnz > 0)
@@ -298,8 +347,13 @@ gp_status gp_graph_create(gp_ctx ctx, gp_vid n, const gp_vid *adjp, const gp_vid
         if (vwgt) e = cudaMemcpyAsync(g->vwgt, vwgt, sizeof(int32_t) * (size_t)n, kind, ctx->stream);
         else st = fill_ones(ctx, g->vwgt, n);
     }
+    if (st == GP_OK && e == cudaSuccess) {
+        SizeRec r{n, nnz, 0, 0};
+        memcpy(ctx->pinned + 16, &r, sizeof(r));
+        e = cudaMemcpyAsync(g->sizes, ctx->pinned + 16, sizeof(SizeRec), cudaMemcpyHostToDevice, ctx->stream);
+    }
     if (st == GP_OK && e != cudaSuccess) st = cuda_fail(e, "gp_graph_create: copy");
-    if (st == GP_OK) st = graph_totals_and_validate(ctx, g, flags & GP_VALIDATE);
+    if (st == GP_OK) st = graph_totals_and_validate(ctx, g, flags & GP_VALIDATE);  // synchronises
     if (st != GP_OK) {
         std::string keep = g_last_error;
         cudaStreamSynchronize(ctx->stream);
@@ -344,6 +398,16 @@ gp_status gp_graph_download(gp_graph g, gp_vid *h_adjp, gp_vid *h_adjncy, gp_wgt
     return GP_OK;
 }
 
+// a SizeRec copy of g with stop = 0 (the first level of a call never inherits a stop flag)
+static gp_status fresh_sizes(Ctx *ctx, const Graph *g, SizeRec *dst) {
+    SizeRec r{g->n, g->nnz, 0, 0};
+    memcpy(ctx->pinned + 32, &r, sizeof(r));
+    GP_CUDA(cudaMemcpyAsync(dst, ctx->pinned + 32, sizeof(SizeRec), cudaMemcpyHostToDevice, ctx->stream));
+    return GP_OK;
+}
+
+static double avg_degree(int32_t n, int32_t nnz) { return n > 0 ? (double)nnz / n : 0.0; }
+
 gp_status gp_match_level(gp_graph g, gp_vid *d_match, int32_t max_rounds, int32_t *rounds_out) {
     if (!tagged<Graph>(g, kTagGraph) || (!d_match && g->n > 0) || max_rounds < 0) {
         set_error("gp_match_level: bad graph, match buffer or max_rounds");
@@ -351,14 +415,33 @@ gp_status gp_match_level(gp_graph g, gp_vid *d_match, int32_t max_rounds, int32_
     }
     GP_TRY_BEGIN
     Ctx *ctx = g->ctx;
-    MatchResult r;
-    gp_status st = match_level(ctx, g, d_match, max_rounds, true, &r);
-    if (st != GP_OK) return st;
-    if (rounds_out) {
-        GP_CUDA(cudaStreamSynchronize(ctx->stream));
-        *rounds_out = r.rounds;
+    if (g->n == 0) {
+        if (rounds_out) *rounds_out = 0;
+        return GP_OK;
     }
-    return GP_OK;
+    LevelBufs lb;
+    gp_status st = level_scratch(ctx, g->n, g->nnz, &lb);
+    if (st != GP_OK) return st;
+    LevelDev *ld = nullptr;
+    st = dev_alloc(ctx, (void **)&ld, sizeof(LevelDev));
+    if (st != GP_OK) return st;
+    set_graph_bufs(&lb, g);
+    lb.in = &ld->out;
+    st = fresh_sizes(ctx, g, &ld->out);
+    if (st == GP_OK) {
+        cudaError_t e = cudaMemsetAsync(&ld->match, 0, sizeof(MatchCtl), ctx->stream);
+        if (e != cudaSuccess) st = cuda_fail(e, "memset");
+    }
+    if (st == GP_OK) st = enqueue_match(ctx, lb, d_match, &ld->match, max_rounds, true, avg_degree(g->n, g->nnz));
+    if (st == GP_OK && rounds_out) {
+        cudaError_t e = cudaMemcpyAsync(ctx->pinned, &ld->match.rounds, sizeof(int32_t), cudaMemcpyDeviceToHost,
+                                        ctx->stream);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+        if (e != cudaSuccess) st = cuda_fail(e, "gp_match_level");
+        else *rounds_out = ctx->pinned[0];
+    }
+    dev_free(ctx, ld);
+    return st;
     GP_TRY_END
 }
 
@@ -369,13 +452,74 @@ gp_status gp_contract_level(gp_graph g, const gp_vid *d_match, gp_vid *d_cmap, g
         return GP_ERR_INVALID_ARG;
     }
     GP_TRY_BEGIN
-    Graph *c = nullptr;
-    gp_status st = contract_level(g->ctx, g, const_cast<int32_t *>(d_match), d_cmap, false, &c);
+    Ctx *ctx = g->ctx;
+    LevelBufs lb;
+    gp_status st = level_scratch(ctx, g->n, g->nnz, &lb);
     if (st != GP_OK) return st;
-    *coarse_out = c;
+    LevelDev *ld = nullptr;
+    st = dev_alloc(ctx, (void **)&ld, sizeof(LevelDev));
+    if (st != GP_OK) return st;
+    Graph *cg = new Graph();
+    cg->ctx = ctx;
+    st = alloc_graph_arrays(ctx, cg, g->n, g->nnz, true);
+    set_graph_bufs(&lb, g);
+    lb.in = &ld->out;
+    if (st == GP_OK) st = fresh_sizes(ctx, g, &ld->out);
+    if (st == GP_OK) {
+        cudaError_t e = cudaMemsetAsync(&ld->contract, 0, sizeof(ContractCtl), ctx->stream);
+        if (e != cudaSuccess) st = cuda_fail(e, "memset");
+    }
+    ContractParams prm{false, -1, 100, 0, INT32_MAX, g->n, g->nnz};
+    if (st == GP_OK)
+        st = enqueue_contract(ctx, lb, const_cast<int32_t *>(d_match), d_cmap, cg, &ld->contract, cg->sizes, nullptr,
+                              prm);
+    if (st == GP_OK) {
+        cudaError_t e = cudaMemcpyAsync(ctx->pinned, cg->sizes, sizeof(SizeRec), cudaMemcpyDeviceToHost, ctx->stream);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(ctx->stream);
+        if (e != cudaSuccess) st = cuda_fail(e, "gp_contract_level");
+    }
+    if (st == GP_OK) {
+        cg->n = ctx->pinned[0];
+        cg->nnz = ctx->pinned[1];
+        // the coarse graph is a regular input graph from now on
+        st = fresh_sizes(ctx, cg, cg->sizes);
+    }
+    dev_free(ctx, ld);
+    if (st != GP_OK) {
+        std::string keep = g_last_error;
+        cudaStreamSynchronize(ctx->stream);
+        graph_release(cg);
+        g_last_error = keep;
+        return st;
+    }
+    *coarse_out = cg;
     return GP_OK;
     GP_TRY_END
 }
+
+// ---------------------------------------------------------------------------------------
+// gp_coarsen_to: pipelined level enqueue.  Each level is two persistent cooperative
+// kernels (matching, contraction).  All sizes travel through device memory, so the host
+// never waits for a level before enqueuing the next one: it keeps kAhead levels in flight,
+// sizing level l's outputs by the tightest size it has observed so far (a coarse graph is
+// never larger than its fine graph), and learns each level's result from a report the
+// contraction kernel writes into mapped host memory.  A level whose predecessor decided to
+// stop (threshold / stall / max_levels) exits immediately and is discarded.
+// ---------------------------------------------------------------------------------------
+constexpr int kAhead = 2;
+
+static bool debug_on() {
+    static int on = -1;
+    if (on < 0) on = getenv("GP_DEBUG") ? 1 : 0;
+    return on == 1;
+}
+#define GP_DBG(...)                               \
+    do {                                          \
+        if (debug_on()) {                         \
+            fprintf(stderr, "[gp] " __VA_ARGS__); \
+            fflush(stderr);                       \
+        }                                         \
+    } while (0)
 
 gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
     if (out) *out = nullptr;
@@ -387,41 +531,129 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
     GP_TRY_BEGIN
     Ctx *ctx = g->ctx;
     const int32_t pct = opts->stall_ratio_pct ? opts->stall_ratio_pct : 95;
-    const int32_t max_levels = opts->max_levels ? opts->max_levels : 64;
+    int32_t max_levels = opts->max_levels ? opts->max_levels : 64;
+    if (max_levels > ctx->max_reports) max_levels = ctx->max_reports;
     Hier *h = new Hier();
     h->ctx = ctx;
-    const Graph *cur = g;
+    if (g->n <= opts->threshold) {
+        *out = h;
+        return GP_OK;
+    }
     gp_status st = GP_OK;
-    while (cur->n > opts->threshold && (int32_t)h->levels.size() < max_levels) {
-        Level lv;
-        lv.n = cur->n;
-        lv.nnz = cur->nnz;
-        st = dev_alloc(ctx, (void **)&lv.match, sizeof(int32_t) * (size_t)cur->n);
-        if (st == GP_OK) st = dev_alloc(ctx, (void **)&lv.cmap, sizeof(int32_t) * (size_t)cur->n);
-        MatchResult mr;
-        if (st == GP_OK) st = match_level(ctx, cur, lv.match, opts->max_rounds, false, &mr);
+    std::vector<Level> lv;  // enqueued levels (L.n / L.nnz hold the size bounds used)
+    // tightest known upper bound of the next level's input: the last observed coarse sizes
+    int32_t tight_n = g->n, tight_m = g->nnz;
+    LevelBufs lb;
+    st = level_scratch(ctx, g->n, g->nnz, &lb);  // level 0 is the largest
+    if (st == GP_OK) st = dev_alloc(ctx, (void **)&h->levdev, sizeof(LevelDev) * (size_t)(max_levels + 1));
+    if (st == GP_OK) {
+        cudaError_t e = cudaMemsetAsync(h->levdev, 0, sizeof(LevelDev) * (size_t)(max_levels + 1), ctx->stream);
+        if (e != cudaSuccess) st = cuda_fail(e, "memset(levdev)");
+    }
+    // level 0 reads its sizes from levdev[max_levels].out (a fresh, stop-free copy)
+    SizeRec *in0 = (st == GP_OK) ? &h->levdev[max_levels].out : nullptr;
+    if (st == GP_OK) st = fresh_sizes(ctx, g, in0);
+    for (int i = 0; i < max_levels; ++i) ctx->reports[i].ready = 0;
+
+    auto enqueue_level = [&](int l) -> gp_status {
+        const Graph *in = (l == 0) ? g : lv[l - 1].coarse;
+        const int32_t n_b = tight_n, m_b = tight_m;
+        Level L;
+        L.n = n_b;
+        L.nnz = m_b;
+        gp_status s2 = dev_alloc(ctx, (void **)&L.match, sizeof(int32_t) * (size_t)(n_b > 0 ? n_b : 1));
+        if (s2 == GP_OK) s2 = dev_alloc(ctx, (void **)&L.cmap, sizeof(int32_t) * (size_t)(n_b > 0 ? n_b : 1));
         Graph *cg = nullptr;
-        if (st == GP_OK) st = contract_level(ctx, cur, lv.match, lv.cmap, true, &cg);
-        if (st != GP_OK) {
-            dev_free(ctx, lv.match);
-            dev_free(ctx, lv.cmap);
-            break;
+        if (s2 == GP_OK) {
+            cg = new Graph();
+            cg->ctx = ctx;
+            cg->borrowed = true;
+            s2 = alloc_graph_arrays(ctx, cg, n_b, m_b, false);
+            cg->sizes = &h->levdev[l].out;
         }
-        cg->borrowed = true;
-        lv.coarse = cg;
-        lv.rounds = mr.rounds;
-        lv.maximal = mr.maximal;
-        lv.arcs_scanned = mr.arcs_scanned;
-        lv.rows_scanned = mr.rows_scanned;
-        lv.live_visits = mr.live_visits;
-        lv.n_coarse = cg->n;
-        lv.cnnz = cg->nnz;
-        h->levels.push_back(lv);
-        const bool stall = 100LL * cg->n > (long long)pct * cur->n;
-        cur = cg;
-        if (stall) {
-            h->levels.back().stop_reason = GP_STOP_STALL;
-            break;
+        L.coarse = cg;
+        lv.push_back(L);  // registered before any failure so that it gets released
+        if (s2 != GP_OK) return s2;
+        LevelBufs b = lb;
+        set_graph_bufs(&b, in);
+        b.in = (l == 0) ? in0 : in->sizes;
+        s2 = enqueue_match(ctx, b, L.match, &h->levdev[l].match, opts->max_rounds, false, avg_degree(n_b, m_b));
+        if (s2 != GP_OK) return s2;
+        ContractParams prm{true, opts->threshold, pct, l, max_levels, n_b, m_b};
+        return enqueue_contract(ctx, b, L.match, L.cmap, cg, &h->levdev[l].contract, &h->levdev[l].out,
+                                &ctx->reports_dev[l], prm);
+    };
+
+    int enq = 0, obs = 0, last_real = -1;
+    bool stop_seen = false;
+    while (st == GP_OK) {
+        while (st == GP_OK && !stop_seen && enq < max_levels && enq - obs < kAhead) {
+            GP_DBG("enqueue level %d (bounds n=%d nnz=%d)\n", enq, tight_n, tight_m);
+            st = enqueue_level(enq);
+            ++enq;
+        }
+        if (st != GP_OK || obs == enq) break;
+        volatile LevelReport *r = &ctx->reports[obs];
+        const auto t_wait = std::chrono::steady_clock::now();
+        while (!r->ready) {
+            if (std::chrono::steady_clock::now() - t_wait > std::chrono::seconds(120)) {
+                set_error("gp_coarsen_to: level " + std::to_string(obs) + " did not report within 120 s");
+                st = GP_ERR_INTERNAL;
+                break;
+            }
+            const cudaError_t q = cudaStreamQuery(ctx->stream);
+            if (q != cudaSuccess && q != cudaErrorNotReady) {
+                st = cuda_fail(q, "gp_coarsen_to: level kernel");
+                break;
+            }
+            if (q == cudaSuccess && !r->ready) {  // stream drained without a report: a bug
+                set_error("gp_coarsen_to: level finished without a report");
+                st = GP_ERR_INTERNAL;
+                break;
+            }
+        }
+        if (st != GP_OK) break;
+        GP_DBG("level %d reported: n_c=%d cnnz=%d stop=%d reason=%d skipped=%d\n", obs, r->n_coarse, r->cnnz, r->stop,
+               r->stop_reason, r->skipped);
+        if (!r->skipped) {
+            last_real = obs;
+            lv[obs].n_coarse = r->n_coarse;
+            lv[obs].cnnz = r->cnnz;
+            lv[obs].stop_reason = r->stop_reason;
+            tight_n = r->n_coarse;
+            tight_m = r->cnnz;
+            if (r->stop) stop_seen = true;
+        }
+        ++obs;
+    }
+    cudaError_t e = cudaStreamSynchronize(ctx->stream);
+    if (st == GP_OK && e != cudaSuccess) st = cuda_fail(e, "gp_coarsen_to");
+    if (st == GP_OK && last_real >= 0) {
+        // per-level statistics of the matching kernels (one small copy)
+        std::vector<LevelDev> hd((size_t)last_real + 1);
+        e = cudaMemcpy(hd.data(), h->levdev, sizeof(LevelDev) * hd.size(), cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) st = cuda_fail(e, "gp_coarsen_to: stats");
+        for (int l = 0; st == GP_OK && l <= last_real; ++l) {
+            Level &L = lv[l];
+            L.n = (l == 0) ? g->n : lv[l - 1].n_coarse;
+            L.nnz = (l == 0) ? g->nnz : lv[l - 1].cnnz;
+            L.rounds = hd[l].match.rounds;
+            L.maximal = hd[l].match.maximal;
+            L.arcs_scanned = (int64_t)hd[l].match.arcs_scanned;
+            L.rows_scanned = (int64_t)hd[l].match.rows_scanned + L.n;
+            L.live_visits = (int64_t)hd[l].match.live_visits;
+            L.coarse->n = L.n_coarse;
+            L.coarse->nnz = L.cnnz;
+        }
+    }
+    // keep levels 0..last_real, release the rest (speculative levels after the stop)
+    for (int l = 0; l < (int)lv.size(); ++l) {
+        if (st == GP_OK && l <= last_real) {
+            h->levels.push_back(lv[l]);
+        } else {
+            dev_free(ctx, lv[l].match);
+            dev_free(ctx, lv[l].cmap);
+            graph_release(lv[l].coarse);
         }
     }
     if (st != GP_OK) {
@@ -431,8 +663,6 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
         g_last_error = keep;
         return st;
     }
-    if (!h->levels.empty() && h->levels.back().stop_reason == GP_STOP_NONE)
-        h->levels.back().stop_reason = (cur->n <= opts->threshold) ? GP_STOP_THRESHOLD : GP_STOP_MAX_LEVELS;
     *out = h;
     return GP_OK;
     GP_TRY_END
@@ -500,9 +730,9 @@ void gp_free(void *handle) {
         for (auto e : ctx->event_pool) cudaEventDestroy(e);
         dev_free(ctx, ctx->scratch);
         dev_free(ctx, ctx->status);
-        dev_free(ctx, ctx->ctl);
         cudaStreamSynchronize(ctx->stream);
-        if (ctx->ctl_host) cudaFreeHost(ctx->ctl_host);
+        if (ctx->pinned) cudaFreeHost(ctx->pinned);
+        if (ctx->reports) cudaFreeHost(ctx->reports);
         ctx->tag = 0;
         delete ctx;
     }

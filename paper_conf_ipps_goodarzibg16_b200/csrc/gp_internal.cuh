@@ -22,28 +22,56 @@ constexpr uint32_t kTagHier = 0x47504849u;   // "GPHI"
 constexpr int kBlock = 256;  // threads per CTA of the streaming kernels
 
 // ---------------------------------------------------------------------------------------
-// device-side control block of one level (one memset per level)
+// device-side control blocks of one level (zeroed once per gp_coarsen_to call)
 // ---------------------------------------------------------------------------------------
-struct RoundCounters {
-    int32_t live;     // entries of the live list of this parity
-    int32_t r_small;  // rescan list, group bin
-    int32_t r_warp;   // rescan list, warp bin
-    int32_t r_cta;    // rescan list, CTA bin
+struct RoundSlot {
+    int32_t live;     // live-list length of the round this slot belongs to
+    int32_t nhub;     // hub rows waiting for the hub phase
+    int32_t matches;  // matches made by the round's commit
+    int32_t pad;
 };
 
-struct LevelCtl {
-    RoundCounters cnt[2];       // by round parity
-    int32_t matches;            // new matches in the current round
-    int32_t rounds;             // rounds that created >= 1 match (R4)
-    int32_t blocks_done;        // last-block detection of the commit kernel
-    int32_t n_coarse;           // written by the cmap scan
-    int32_t cnnz;               // written by the count scan
-    int32_t n_big_w, n_big_c, n_big_g;  // contraction big-row bins
-    uint32_t tile_ctr[8];       // dynamic tile counters of the scans of this level
-    unsigned long long arcs_scanned;
-    unsigned long long rows_scanned;
-    unsigned long long live_visits;
-    int32_t pad[4];
+struct MatchCtl {
+    unsigned bar[2];   // grid barrier
+    RoundSlot slot[4]; // ring by round number
+    int32_t rounds, maximal;
+    unsigned long long arcs_scanned, rows_scanned, live_visits;
+    int32_t pad[2];
+};
+
+struct ContractCtl {
+    unsigned bar[2];
+    unsigned tile_ctr[2];
+    int32_t n_coarse, cnnz, n_huge;
+    unsigned blocks_done;
+};
+
+// per-graph device size record: the producer of a coarse graph writes it
+struct SizeRec {
+    int32_t n, nnz;
+    int32_t stop;        // 1: do not coarsen this graph further
+    int32_t stop_reason; // GP_STOP_* of the level that produced it
+};
+
+struct LevelDev {
+    MatchCtl match;
+    ContractCtl contract;
+    SizeRec out;  // sizes of this level's coarse graph
+};
+
+// written by the device into mapped pinned host memory when a level completes
+struct LevelReport {
+    int32_t n_coarse, cnnz, stop, stop_reason;
+    int32_t ready, skipped, pad[2];
+};
+
+// device pointers one level's kernels use
+struct LevelBufs {
+    const SizeRec *in;  // sizes (+ stop flag) of this level's input graph
+    const int32_t *adjp, *adjncy, *adjwgt, *vwgt;
+    int32_t *P[2], *L[2], *H;                         // matching scratch
+    int32_t *leaders, *off, *cnt, *tile_start, *huge;  // contraction scratch
+    unsigned long long *gkeys;
 };
 
 }  // namespace gp
@@ -71,6 +99,8 @@ struct gp_graph_s {
     gp::Ctx *ctx = nullptr;
     int32_t n = 0, nnz = 0;
     int32_t *adjp = nullptr, *adjncy = nullptr, *adjwgt = nullptr, *vwgt = nullptr;
+    gp::SizeRec *sizes = nullptr;  // device copy of {n, nnz, stop}
+    bool owns_sizes = true;
     bool borrowed = false;  // owned by a hierarchy
 };
 
@@ -87,6 +117,7 @@ struct gp_hier_s {
     uint32_t tag = gp::kTagHier;
     gp::Ctx *ctx = nullptr;
     std::vector<gp::Level> levels;
+    gp::LevelDev *levdev = nullptr;  // per-level control blocks (coarse graphs' size records)
 };
 
 struct gp_ctx_s {
@@ -102,8 +133,10 @@ struct gp_ctx_s {
     // grow-only scratch of the level pipeline
     void *scratch = nullptr;
     size_t scratch_bytes = 0;
-    gp::LevelCtl *ctl = nullptr;       // device
-    gp::LevelCtl *ctl_host = nullptr;  // pinned mirror
+    int32_t *pinned = nullptr;  // small pinned host buffer for read-backs
+    gp::LevelReport *reports = nullptr;     // mapped pinned host memory (device-written)
+    gp::LevelReport *reports_dev = nullptr; // its device alias
+    int32_t max_reports = 0;
     unsigned long long *status = nullptr;  // look-back tile status words
     size_t status_words = 0;
     uint32_t epoch = 1;  // look-back epoch (no memset between scans)
@@ -152,24 +185,26 @@ inline int persistent_grid(const Ctx *ctx, int blocks_per_sm) { return ctx->num_
 // ---------------------------------------------------------------------------------------
 // level pipeline entry points (implemented in match.cu / contract.cu / validate.cu)
 // ---------------------------------------------------------------------------------------
-struct MatchResult {
-    int32_t rounds = 0, maximal = 0;
-    int64_t arcs_scanned = 0, rows_scanned = 0, live_visits = 0;
+
+// enqueue the persistent matching kernel of one level (A1-A4; leftover optional)
+gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl, int32_t max_rounds, bool leftover,
+                        double avg_deg_hint);
+// enqueue the persistent contraction kernel of one level (A4 leftover + A5-A8)
+struct ContractParams {
+    bool leftover;
+    int32_t threshold, stall_pct, level, max_levels;
+    int32_t n_bound, nnz_bound;
 };
-
-// A1-A4 without the leftover pass.  M receives FREE for unmatched vertices unless
-// `leftover` is set.  Uses ctx->ctl (memset by the call).
-gp_status match_level(Ctx *ctx, const Graph *g, int32_t *M, int32_t max_rounds, bool leftover,
-                      MatchResult *res);
-
-// A4 leftover (optional) + A5-A8: cmap and coarse graph.  M may contain FREE entries when
-// `apply_leftover` is set (they become self-matches and M is updated in place).
-gp_status contract_level(Ctx *ctx, const Graph *g, int32_t *M, int32_t *CM, bool apply_leftover,
-                         Graph **coarse_out);
+gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *CM, Graph *coarse, ContractCtl *ctl,
+                           SizeRec *out_sizes, LevelReport *report, const ContractParams &prm);
+size_t contract_status_words(int32_t n, int32_t nnz);
+size_t contract_tiles(int32_t nnz);
 
 gp_status graph_totals_and_validate(Ctx *ctx, const Graph *g, bool validate);
 
 gp_status ensure_scratch(Ctx *ctx, size_t bytes);
+// carve one level's scratch pointers out of ctx->scratch (sized for n, nnz)
+gp_status level_scratch(Ctx *ctx, int32_t n, int32_t nnz, LevelBufs *lb);
 gp_status ensure_status(Ctx *ctx, size_t words);
 
 }  // namespace gp

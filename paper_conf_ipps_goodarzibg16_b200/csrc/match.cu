@@ -1,25 +1,31 @@
-// match.cu -- A1-A4: degree-binned proposals, handshake commit, round loop, leftover.
+// match.cu -- A1-A4 of one level in ONE persistent cooperative kernel: degree-binned
+// proposals, handshake commits, the round loop and the leftover pass.
 //
 // Rule (PAPER.md P18.s6-13 re-pinned by north_star, R1-R4): in every round each
-// free vertex proposes its heaviest free neighbour (ties -> lower id, P12.s23, P18.s7); two
-// vertices that propose each other match (handshake; replaces the paper's conflict kernel
-// "M[u]=v and M[v]!=u => M[u]=u", P18.s10-12).  Rounds repeat until no free vertex has a
-// free neighbour; the leftover pass self-matches the rest (P18.s12-13).
+// free vertex proposes its heaviest free neighbour (ties -> lower id; HEM, P12.s23,
+// P18.s7); two vertices that propose each other match (handshake; replaces the paper's
+// conflict kernel "M[u]=v and M[v]!=u => M[u]=u", P18.s10-12).  Rounds repeat until no
+// free vertex has a free neighbour; the leftover pass self-matches the rest (P18.s12-13).
 //
 // B200 design:
-//  * Lazy rescans: after round 1 only vertices whose proposal target was matched rescan
-//    their row (their proposal is otherwise still the heaviest free neighbour, because the
-//    free set only shrinks).  Result-identical to rescanning everything.
-//  * Degree bins (A1, fused into the round-1 kernel): rows with deg <= 2G are scanned by a
-//    group of G lanes (G chosen per level from the average degree), deg <= kCtaDeg by a
-//    warp, larger rows by a whole CTA (R-MAT hubs).  Warp-shuffle argmax over a packed
-//    64-bit key (weight<<32 | ~id).
-//  * Owner-writes only: M[u] and P[u] are written by u's own lane; no atomics on M/P, so
-//    every schedule gives the same bits.  Worklists are appended with warp-aggregated
-//    atomics; their order does not influence any result.
-//  * All list-driven kernels use persistent grids (a multiple of the SM count) that read
-//    the list length from device memory, so a whole batch of rounds is enqueued without a
-//    host round trip; empty speculative rounds cost one near-empty launch each.
+//  * One launch per level, grid = SMs x co-resident CTAs; phases are separated by a grid
+//    barrier (~1-2 us) instead of kernel boundaries and host round trips.
+//  * Phase 0 (round-1 proposals, every vertex free, no M reads): chunks of consecutive
+//    vertices whose adjacency fits a stage are staged into shared memory with TMA bulk
+//    copies (cp.async.bulk, mbarrier completion, 2 stages), then reduced by groups of G
+//    threads per vertex (G from the level's average degree) -> coalesced 100%-useful HBM
+//    streams.  Chunks with long rows fall back to direct group / warp scans; rows longer
+//    than kHubDeg go to a hub list scanned by whole CTAs.
+//  * Phase k (k >= 1) fuses the commit of round k with the proposals of round k+1:
+//      p = P_k[u], q = P_k[p]:   q == u           -> M[u] = p (matched; owner writes only)
+//                                p kept its pair  -> p is still u's heaviest free neighbour
+//                                p matched q      -> rescan u's row (lazy rescan)
+//    The rescan tests a neighbour x with "M[x] free and not (P_k[P_k[x]] == x)", so the
+//    round-k matches being written concurrently are seen through the read-only P_k.
+//    P is double buffered by round parity; matched and dead vertices hold the same value
+//    (partner / NONE) in both buffers.  Result-identical to the literal rule (oracle).
+//  * Worklists are appended with one atomic per CTA (block-aggregated), round counters
+//    live in a 4-slot ring so no counter is reset while another CTA may still read it.
 #include <cuda_runtime.h>
 
 #include "device_util.cuh"
@@ -27,407 +33,389 @@
 
 namespace gp {
 
-constexpr int kCtaDeg = 4096;    // rows longer than this are scanned by a whole CTA
-constexpr int kUnroll = 4;       // vertices per group per iteration (memory-level parallelism)
+constexpr int kNT = 512;            // threads per CTA of the persistent kernels
+constexpr int kStageArcs = 4096;    // arcs per TMA stage (adjncy + adjwgt = 32 KB)
+constexpr int kThreadDeg = 32;      // phase-k rescans up to this many arcs: one thread
+constexpr int kHubDeg = 4096;       // rows longer than this: one CTA each (hub phase)
 
-struct MatchBufs {
-    int32_t *P;
-    int32_t *L[2];   // live lists by parity
-    int32_t *Rs[2];  // rescan lists: group bin
-    int32_t *Rw[2];  // rescan lists: warp bin
-    int32_t *Rc[2];  // rescan lists: CTA bin
+struct MatchArgs {
+    const SizeRec *in;  // device: sizes + stop flag of this level's graph
+    const int32_t *adjp, *adjncy, *adjwgt;
+    int32_t *M;
+    int32_t *P[2];
+    int32_t *L[2];
+    int32_t *H;  // hub list of the pending hub phase
+    MatchCtl *ctl;
+    int32_t max_rounds;
+    int32_t leftover;
+    int32_t G;  // lanes per vertex in phase 0 (1, 2, 4, 8 or 16)
 };
 
-// ---------------------------------------------------------------------------------------
-// A1 + A2, round 1: every vertex is free, so no M gathers are needed.  Also initialises
-// M[u] = FREE and routes rows longer than 2G to the warp / CTA bins of parity 1.
-// ---------------------------------------------------------------------------------------
-template <int G>
-__global__ void __launch_bounds__(kBlock) k_propose_round1(int32_t n, const int32_t *__restrict__ adjp,
-                                                           const int32_t *__restrict__ adjncy,
-                                                           const int32_t *__restrict__ adjwgt,
-                                                           int32_t *__restrict__ M, int32_t *__restrict__ P,
-                                                           MatchBufs b, LevelCtl *ctl) {
-    constexpr int GPW = 32 / G;
-    const int lane = threadIdx.x & 31, gl = lane % G, grp = lane / G;
-    const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
-    unsigned long long scanned = 0;
-    for (long long base = warp * GPW * kUnroll; base < n; base += nwarps * GPW * kUnroll) {
-        int32_t s[kUnroll], e[kUnroll];
-#pragma unroll
-        for (int i = 0; i < kUnroll; ++i) {
-            long long u = base + i * GPW + grp;
-            s[i] = 0;
-            e[i] = 0;
-            if (u < n) {
-                s[i] = __ldg(adjp + u);
-                e[i] = __ldg(adjp + u + 1);
-            }
-        }
-        int32_t v[kUnroll][2], w[kUnroll][2];
-#pragma unroll
-        for (int i = 0; i < kUnroll; ++i) {
-            const bool small = e[i] - s[i] <= 2 * G;
-#pragma unroll
-            for (int t = 0; t < 2; ++t) {
-                int32_t j = s[i] + t * G + gl;
-                v[i][t] = -1;
-                w[i][t] = 0;
-                if (small && j < e[i]) {
-                    v[i][t] = __ldg(adjncy + j);
-                    w[i][t] = __ldg(adjwgt + j);
-                }
-            }
-        }
-#pragma unroll
-        for (int i = 0; i < kUnroll; ++i) {
-            unsigned long long key = 0;
-#pragma unroll
-            for (int t = 0; t < 2; ++t)
-                if (v[i][t] >= 0) key = umax64(key, pack_key(w[i][t], v[i][t]));
-            key = group_max64<G>(key);
-            long long u = base + i * GPW + grp;
-            if (gl == 0 && u < n) {
-                int32_t deg = e[i] - s[i];
-                M[u] = kFree;
-                if (deg <= 2 * G) {
-                    P[u] = key_vertex(key);
-                    scanned += deg;
-                } else if (deg <= kCtaDeg) {
-                    b.Rw[1][atomicAdd(&ctl->cnt[1].r_warp, 1)] = (int32_t)u;
-                } else {
-                    b.Rc[1][atomicAdd(&ctl->cnt[1].r_cta, 1)] = (int32_t)u;
-                }
-            }
-        }
-    }
-    scanned = warp_sum64(scanned);
-    if (lane == 0 && scanned) atomicAdd(&ctl->arcs_scanned, scanned);
+struct MatchSmem {
+    int32_t adj[2][kStageArcs];
+    int32_t wgt[2][kStageArcs];
+    uint64_t bar[2];
+    int32_t a0[2];    // aligned first arc of the staged chunk
+    int32_t fits[2];  // chunk staged (1) or fallback (0)
+    int32_t scratch[40];
+    unsigned long long red[kNT / 32];
+};
+
+__device__ __forceinline__ int32_t ldcg(const int32_t *p) { return __ldcg(p); }
+
+// x is free after round k's commits
+__device__ __forceinline__ bool free_after(int32_t x, const int32_t *M, const int32_t *Pk) {
+    if (ldcg(M + x) != kFree) return false;
+    const int32_t px = ldcg(Pk + x);
+    return !(px >= 0 && ldcg(Pk + px) == x);
 }
 
-// ---------------------------------------------------------------------------------------
-// A2, rounds >= 2: rescan of the group-bin list of parity p (reads M to skip matched).
-// ---------------------------------------------------------------------------------------
 template <int G>
-__global__ void __launch_bounds__(kBlock) k_propose_list(const int32_t *__restrict__ adjp,
-                                                         const int32_t *__restrict__ adjncy,
-                                                         const int32_t *__restrict__ adjwgt,
-                                                         const int32_t *__restrict__ M, int32_t *__restrict__ P,
-                                                         const int32_t *__restrict__ list, const int32_t *count) {
-    constexpr int GPW = 32 / G;
-    const int len = *count;
-    const int lane = threadIdx.x & 31, gl = lane % G, grp = lane / G;
-    const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
-    for (long long base = warp * GPW * kUnroll; base < len; base += nwarps * GPW * kUnroll) {
-        int32_t s[kUnroll], e[kUnroll], uu[kUnroll];
-#pragma unroll
-        for (int i = 0; i < kUnroll; ++i) {
-            long long k = base + i * GPW + grp;
-            uu[i] = -1;
-            s[i] = e[i] = 0;
-            if (k < len) {
-                uu[i] = list[k];
-                s[i] = __ldg(adjp + uu[i]);
-                e[i] = __ldg(adjp + uu[i] + 1);
-            }
-        }
-        int32_t v[kUnroll][2], w[kUnroll][2];
-#pragma unroll
-        for (int i = 0; i < kUnroll; ++i)
-#pragma unroll
-            for (int t = 0; t < 2; ++t) {
-                int32_t j = s[i] + t * G + gl;
-                v[i][t] = -1;
-                w[i][t] = 0;
-                if (j < e[i]) {
-                    v[i][t] = __ldg(adjncy + j);
-                    w[i][t] = __ldg(adjwgt + j);
-                }
-            }
-#pragma unroll
-        for (int i = 0; i < kUnroll; ++i)
-#pragma unroll
-            for (int t = 0; t < 2; ++t)
-                if (v[i][t] >= 0 && M[v[i][t]] != kFree) v[i][t] = -1;
-#pragma unroll
-        for (int i = 0; i < kUnroll; ++i) {
-            unsigned long long key = 0;
-#pragma unroll
-            for (int t = 0; t < 2; ++t)
-                if (v[i][t] >= 0) key = umax64(key, pack_key(w[i][t], v[i][t]));
-            key = group_max64<G>(key);
-            if (gl == 0 && uu[i] >= 0) P[uu[i]] = key_vertex(key);
-        }
+__device__ __forceinline__ unsigned long long gmax(unsigned long long k) {
+    return group_max64<G>(k);
+}
+
+__device__ __forceinline__ unsigned long long group_max_rt(unsigned long long k, int G) {
+    switch (G) {
+        case 1: return k;
+        case 2: return group_max64<2>(k);
+        case 4: return group_max64<4>(k);
+        case 8: return group_max64<8>(k);
+        default: return group_max64<16>(k);
     }
 }
 
 // ---------------------------------------------------------------------------------------
-// A2 for long rows: CTA per vertex (CTA bin) then warp per vertex (warp bin).
+// phase 0: round-1 proposals of every vertex
 // ---------------------------------------------------------------------------------------
-template <bool kCheckM>
-__global__ void __launch_bounds__(kBlock) k_propose_big(const int32_t *__restrict__ adjp,
-                                                        const int32_t *__restrict__ adjncy,
-                                                        const int32_t *__restrict__ adjwgt,
-                                                        const int32_t *__restrict__ M, int32_t *__restrict__ P,
-                                                        const int32_t *__restrict__ listC, const int32_t *countC,
-                                                        const int32_t *__restrict__ listW, const int32_t *countW,
-                                                        LevelCtl *ctl) {
-    __shared__ unsigned long long red[kBlock / 32];
-    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    const int nC = *countC, nW = *countW;
-    unsigned long long scanned = 0;
-    for (int i = blockIdx.x; i < nC; i += gridDim.x) {
-        const int32_t u = listC[i];
-        const int32_t s = adjp[u], e = adjp[u + 1];
+__device__ __forceinline__ void chunk_bounds(const MatchArgs &a, int32_t n, int32_t vch, long long c, int32_t &A0,
+                                             int32_t &A1, int32_t &fits) {
+    const long long v0 = c * vch;
+    const long long v1 = min((long long)n, v0 + vch);
+    const int32_t s = __ldg(a.adjp + v0), e = __ldg(a.adjp + v1);
+    A0 = s & ~3;
+    A1 = (e + 3) & ~3;
+    fits = (A1 - A0) <= kStageArcs;
+}
+
+__device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned long long &scanned) {
+    const int G = a.G;
+    const int vch = kNT / G;
+    const long long nchunks = ((long long)n + vch - 1) / vch;
+    const int t = threadIdx.x, gl = t % G;
+    int32_t *P1 = a.P[1], *P0 = a.P[0];
+    if (t == 0) {
+        mbar_init(&sm.bar[0], 1);
+        mbar_init(&sm.bar[1], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    // prologue: bounds + TMA for the first two chunks of this CTA
+    if (t == 0) {
+        for (int i = 0; i < 2; ++i) {
+            const long long c = blockIdx.x + (long long)i * gridDim.x;
+            if (c < nchunks) {
+                int32_t A0, A1, f;
+                chunk_bounds(a, n, vch, c, A0, A1, f);
+                sm.a0[i] = A0;
+                sm.fits[i] = f;
+                if (f && A1 > A0) {
+                    mbar_arrive_expect_tx(&sm.bar[i], (unsigned)(A1 - A0) * 8u);
+                    tma_load_1d(sm.adj[i], a.adjncy + A0, (unsigned)(A1 - A0) * 4u, &sm.bar[i]);
+                    tma_load_1d(sm.wgt[i], a.adjwgt + A0, (unsigned)(A1 - A0) * 4u, &sm.bar[i]);
+                } else if (f) {
+                    sm.fits[i] = 2;  // empty chunk: nothing to wait for
+                }
+            }
+        }
+    }
+    __syncthreads();
+    unsigned uses[2] = {0, 0};
+    for (long long i = 0;; ++i) {
+        const long long c = blockIdx.x + i * gridDim.x;
+        if (c >= nchunks) break;
+        const int st = (int)(i & 1);
+        const int fits = sm.fits[st];
+        const int32_t A0 = sm.a0[st];
+        if (fits == 1) {
+            mbar_wait(&sm.bar[st], uses[st] & 1u);
+            ++uses[st];
+        }
+        const long long v = c * vch + t / G;
+        const bool valid = v < n;
+        int32_t s = 0, e = 0;
+        if (valid) {
+            s = __ldg(a.adjp + v);
+            e = __ldg(a.adjp + v + 1);
+        }
         unsigned long long key = 0;
-        for (int32_t j = s + threadIdx.x; j < e; j += kBlock) {
-            int32_t v = __ldg(adjncy + j);
-            if (!kCheckM || M[v] == kFree) key = umax64(key, pack_key(__ldg(adjwgt + j), v));
+        bool hub = false;
+        if (fits) {
+            const int32_t *sa = sm.adj[st], *sw = sm.wgt[st];
+            for (int32_t j = s - A0 + gl; j < e - A0; j += G) key = umax64(key, pack_key(sw[j], sa[j]));
+        } else if (valid) {
+            if (e - s > kHubDeg) {
+                hub = true;
+            } else {
+                for (int32_t j = s + gl; j < e; j += G) key = umax64(key, pack_key(__ldg(a.adjwgt + j), __ldg(a.adjncy + j)));
+            }
+        }
+        key = group_max_rt(key, G);
+        if (valid && gl == 0) {
+            a.M[v] = kFree;
+            if (hub) {
+                a.H[atomicAdd(&a.ctl->slot[1].nhub, 1)] = (int32_t)v;
+            } else {
+                const int32_t p = key_vertex(key);
+                P1[v] = p;
+                if (p == kNone) P0[v] = kNone;  // dead vertices: NONE in both buffers
+                scanned += (unsigned long long)(e - s);
+            }
+        }
+        __syncthreads();  // stage `st` is free again
+        if (t == 0) {
+            const long long c2 = blockIdx.x + (i + 2) * gridDim.x;
+            if (c2 < nchunks) {
+                int32_t A0n, A1n, f;
+                chunk_bounds(a, n, vch, c2, A0n, A1n, f);
+                sm.a0[st] = A0n;
+                sm.fits[st] = f;
+                if (f && A1n > A0n) {
+                    mbar_arrive_expect_tx(&sm.bar[st], (unsigned)(A1n - A0n) * 8u);
+                    tma_load_1d(sm.adj[st], a.adjncy + A0n, (unsigned)(A1n - A0n) * 4u, &sm.bar[st]);
+                    tma_load_1d(sm.wgt[st], a.adjwgt + A0n, (unsigned)(A1n - A0n) * 4u, &sm.bar[st]);
+                } else if (f) {
+                    sm.fits[st] = 2;
+                }
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// ---------------------------------------------------------------------------------------
+// hub phase: every listed row (deg > kHubDeg) is scanned by a whole CTA
+// kCheck = false in round 1 (every vertex free), true for rescans after round k.
+// ---------------------------------------------------------------------------------------
+__device__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool check, const int32_t *Pk,
+                          int32_t *Pn, int32_t *Lnext, int32_t *live_next, unsigned long long &scanned) {
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    for (int i = blockIdx.x; i < nhub; i += gridDim.x) {
+        const int32_t u = a.H[i];
+        const int32_t s = __ldg(a.adjp + u), e = __ldg(a.adjp + u + 1);
+        unsigned long long key = 0;
+        for (int32_t j = s + threadIdx.x; j < e; j += kNT) {
+            const int32_t x = __ldg(a.adjncy + j);
+            if (!check || free_after(x, a.M, Pk)) key = umax64(key, pack_key(__ldg(a.adjwgt + j), x));
         }
         key = group_max64<32>(key);
-        if (lane == 0) red[wib] = key;
+        if (lane == 0) sm.red[wib] = key;
         __syncthreads();
         if (threadIdx.x == 0) {
             unsigned long long k = 0;
-            for (int q = 0; q < kBlock / 32; ++q) k = umax64(k, red[q]);
-            P[u] = key_vertex(k);
+            for (int q = 0; q < kNT / 32; ++q) k = umax64(k, sm.red[q]);
+            const int32_t p = key_vertex(k);
+            Pn[u] = p;
+            if (p == kNone) {
+                a.P[0][u] = kNone;
+                a.P[1][u] = kNone;
+            } else if (Lnext) {
+                Lnext[atomicAdd(live_next, 1)] = u;
+            }
             scanned += (unsigned long long)(e - s);
         }
         __syncthreads();
     }
-    const int gw = blockIdx.x * (kBlock / 32) + wib, nwarps = gridDim.x * (kBlock / 32);
-    for (int i = gw; i < nW; i += nwarps) {
-        const int32_t u = listW[i];
-        const int32_t s = adjp[u], e = adjp[u + 1];
-        unsigned long long key = 0;
-        for (int32_t j = s + lane; j < e; j += 32) {
-            int32_t v = __ldg(adjncy + j);
-            if (!kCheckM || M[v] == kFree) key = umax64(key, pack_key(__ldg(adjwgt + j), v));
-        }
-        key = group_max64<32>(key);
-        if (lane == 0) {
-            P[u] = key_vertex(key);
-            scanned += (unsigned long long)(e - s);
-        }
-    }
-    if (lane == 0 && scanned) atomicAdd(&ctl->arcs_scanned, scanned);
 }
 
 // ---------------------------------------------------------------------------------------
-// A3: handshake commit over the live list of parity p (round 1: all vertices).
-//   P[u] == NONE             -> u is dead for this level (leftover later)
-//   P[P[u]] == u             -> M[u] = P[u]             (only u's lane writes M[u])
-//   P[u]'s target matched    -> u rescans next round    (lazy rescan)
-//   otherwise                -> u stays live with its proposal
-// The last CTA to finish closes the round: rounds += (matches > 0), consumed counters = 0.
+// phase k >= 1: commit of round k + proposals of round k+1 (lazy rescans)
 // ---------------------------------------------------------------------------------------
-template <bool kAll, int G>
-__global__ void __launch_bounds__(kBlock) k_commit(int32_t n, const int32_t *__restrict__ adjp,
-                                                   int32_t *__restrict__ M, const int32_t *__restrict__ P,
-                                                   MatchBufs b, LevelCtl *ctl, int p) {
-    const int len = kAll ? n : ctl->cnt[p].live;
-    const int q = p ^ 1;
-    const int32_t *Lp = b.L[p];
-    int32_t made = 0, visits = 0;
-    const long long stride = (long long)gridDim.x * blockDim.x;
-    const long long start = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-    // uniform trip count per warp so that warp_append sees all 32 lanes
-    for (long long base = start - (threadIdx.x & 31); base < len; base += stride) {
-        const long long k = base + (threadIdx.x & 31);
-        bool live_next = false, rescan = false;
-        int32_t u = -1, deg = 0;
-        if (k < len) {
-            u = kAll ? (int32_t)k : Lp[k];
-            ++visits;
-            const int32_t pu = P[u];
-            if (pu != kNone) {
-                const int32_t qq = P[pu];
-                if (qq == u) {
-                    M[u] = pu;
+__device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, unsigned long long &scanned,
+                        unsigned long long &rows, unsigned long long &visits, int32_t &made) {
+    const int32_t *Pk = a.P[k & 1];
+    int32_t *Pn = a.P[(k + 1) & 1];
+    int32_t *Pkw = a.P[k & 1];
+    const int32_t *Lk = a.L[k & 1];
+    int32_t *Ln = a.L[(k + 1) & 1];
+    RoundSlot *next = &a.ctl->slot[(k + 1) & 3];
+    const int lane = threadIdx.x & 31;
+    const long long stride = (long long)gridDim.x * kNT;
+    for (long long base = (long long)blockIdx.x * kNT; base < len; base += stride) {
+        const long long idx = base + threadIdx.x;
+        bool live_next = false, need_warp = false;
+        int32_t u = -1, s = 0, e = 0;
+        if (idx < len) {
+            u = (k == 1) ? (int32_t)idx : ldcg(Lk + idx);
+            const int32_t p = ldcg(Pk + u);
+            if (p != kNone) {
+                ++visits;
+                const int32_t q = ldcg(Pk + p);
+                if (q == u) {
+                    a.M[u] = p;  // handshake: u and p propose each other
+                    Pn[u] = p;
                     ++made;
-                } else {
+                } else if (!(q >= 0 && ldcg(Pk + q) == p)) {
+                    Pn[u] = p;  // p is still free: still the heaviest free neighbour
                     live_next = true;
-                    rescan = (qq != kNone) && (P[qq] == pu);  // pu matched qq this round
-                    if (rescan) deg = adjp[u + 1] - adjp[u];
+                } else {
+                    s = __ldg(a.adjp + u);
+                    e = __ldg(a.adjp + u + 1);
+                    ++rows;
+                    if (e - s <= kThreadDeg) {
+                        unsigned long long key = 0;
+                        for (int32_t j = s; j < e; ++j) {
+                            const int32_t x = __ldg(a.adjncy + j);
+                            if (free_after(x, a.M, Pk)) key = umax64(key, pack_key(__ldg(a.adjwgt + j), x));
+                        }
+                        scanned += (unsigned long long)(e - s);
+                        const int32_t b = key_vertex(key);
+                        Pn[u] = b;
+                        if (b == kNone) Pkw[u] = kNone;
+                        live_next = b != kNone;
+                    } else if (e - s <= kHubDeg) {
+                        need_warp = true;
+                    } else {
+                        a.H[atomicAdd(&next->nhub, 1)] = u;
+                    }
                 }
             }
         }
-        warp_append(b.L[q], &ctl->cnt[q].live, live_next, u);
-        warp_append(b.Rs[q], &ctl->cnt[q].r_small, rescan && deg <= 2 * G, u);
-        warp_append(b.Rw[q], &ctl->cnt[q].r_warp, rescan && deg > 2 * G && deg <= kCtaDeg, u);
-        warp_append(b.Rc[q], &ctl->cnt[q].r_cta, rescan && deg > kCtaDeg, u);
+        // medium rows: the whole warp rescans one row at a time
+        unsigned mm = __ballot_sync(0xffffffffu, need_warp);
+        while (mm) {
+            const int src = __ffs(mm) - 1;
+            mm &= mm - 1;
+            const int32_t su = __shfl_sync(0xffffffffu, s, src), eu = __shfl_sync(0xffffffffu, e, src);
+            unsigned long long key = 0;
+            for (int32_t j = su + lane; j < eu; j += 32) {
+                const int32_t x = __ldg(a.adjncy + j);
+                if (free_after(x, a.M, Pk)) key = umax64(key, pack_key(__ldg(a.adjwgt + j), x));
+            }
+            key = group_max64<32>(key);
+            if (lane == src) {
+                const int32_t b = key_vertex(key);
+                Pn[u] = b;
+                if (b == kNone) Pkw[u] = kNone;
+                live_next = b != kNone;
+                scanned += (unsigned long long)(eu - su);
+            }
+        }
+        block_append<kNT>(Ln, &next->live, live_next, u, sm.scratch);
     }
-    made = warp_sum(made);
-    visits = warp_sum(visits);
+}
+
+__global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ MatchArgs a) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    MatchSmem &sm = *reinterpret_cast<MatchSmem *>(smem_raw);
+    MatchCtl *ctl = a.ctl;
+    const volatile SizeRec *in = a.in;
+    if (in->stop) return;  // an earlier level ended the coarsening: nothing to do
+    const int32_t n = in->n;
+    if (n <= 0) return;
+    unsigned long long scanned = 0, rows = 0, visits = 0;
+
+    phase0(a, sm, n, scanned);
+    grid_barrier(ctl->bar);
+    {
+        const int32_t nh = *(volatile int32_t *)&ctl->slot[1].nhub;
+        if (nh > 0) {
+            hub_phase(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned);
+            grid_barrier(ctl->bar);
+        }
+    }
+    int32_t rounds = 0, maximal = 0;
+    for (int k = 1;; ++k) {
+        if (k > n + 2) __trap();  // every round matches >= 1 pair: a bug
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            RoundSlot *z = &ctl->slot[(k + 2) & 3];  // last read two phases ago
+            z->live = 0;
+            z->nhub = 0;
+            z->matches = 0;
+        }
+        const int32_t len = (k == 1) ? n : *(volatile int32_t *)&ctl->slot[k & 3].live;
+        int32_t made = 0;
+        phase_k(a, sm, n, k, len, scanned, rows, visits, made);
+        made = warp_sum(made);
+        if ((threadIdx.x & 31) == 0 && made) atomicAdd(&ctl->slot[k & 3].matches, made);
+        grid_barrier(ctl->bar);
+        const int32_t nh = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].nhub;
+        if (nh > 0) {
+            hub_phase(a, sm, nh, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1], &ctl->slot[(k + 1) & 3].live,
+                      scanned);
+            grid_barrier(ctl->bar);
+        }
+        if (*(volatile int32_t *)&ctl->slot[k & 3].matches > 0) ++rounds;
+        const int32_t live = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].live;
+        if (live == 0) {
+            maximal = 1;
+            break;
+        }
+        if (a.max_rounds > 0 && rounds >= a.max_rounds) break;
+    }
+    if (a.leftover) {
+        for (long long u = (long long)blockIdx.x * kNT + threadIdx.x; u < n; u += (long long)gridDim.x * kNT)
+            if (a.M[u] == kFree) a.M[u] = (int32_t)u;
+    }
+    scanned = warp_sum64(scanned);
+    rows = warp_sum64(rows);
+    visits = warp_sum64(visits);
     if ((threadIdx.x & 31) == 0) {
-        if (made) atomicAdd(&ctl->matches, made);
-        if (visits) atomicAdd(&ctl->live_visits, (unsigned long long)visits);
+        if (scanned) atomicAdd(&ctl->arcs_scanned, scanned);
+        if (rows) atomicAdd(&ctl->rows_scanned, rows);
+        if (visits) atomicAdd(&ctl->live_visits, visits);
     }
-    // last-block round close
-    __shared__ bool last;
-    __threadfence();
-    __syncthreads();
-    if (threadIdx.x == 0) last = atomicAdd(&ctl->blocks_done, 1) == (int)gridDim.x - 1;
-    __syncthreads();
-    if (last && threadIdx.x == 0) {
-        __threadfence();
-        volatile LevelCtl *c = ctl;
-        if (c->matches > 0) c->rounds = c->rounds + 1;
-        c->matches = 0;
-        c->cnt[p].live = 0;
-        c->cnt[p].r_small = 0;
-        c->cnt[p].r_warp = 0;
-        c->cnt[p].r_cta = 0;
-        c->blocks_done = 0;
-        __threadfence();
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        ctl->rounds = rounds;
+        ctl->maximal = maximal;
     }
 }
 
-// rows scanned by the group-bin rescans (for the byte model)
-__global__ void k_count_rows(const int32_t *count_s, const int32_t *count_w, const int32_t *count_c,
-                             LevelCtl *ctl) {
-    if (threadIdx.x == 0)
-        atomicAdd(&ctl->rows_scanned, (unsigned long long)(*count_s + *count_w + *count_c));
-}
-
-// number of live vertices that still have a proposal (exact `maximal` flag under a cap)
-__global__ void k_count_proposing(const int32_t *__restrict__ L, const int32_t *count, const int32_t *__restrict__ P,
-                                  int32_t *out) {
-    const int len = *count;
-    int32_t c = 0;
-    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < len; i += (long long)gridDim.x * blockDim.x)
-        c += P[L[i]] != kNone;
-    c = warp_sum(c);
-    if ((threadIdx.x & 31) == 0 && c) atomicAdd(out, c);
-}
-
-// A4 leftover: every still-free vertex is matched to itself (P18.s12-13)
-__global__ void k_leftover(int32_t n, int32_t *__restrict__ M) {
-    for (long long u = (long long)blockIdx.x * blockDim.x + threadIdx.x; u < n;
-         u += (long long)gridDim.x * blockDim.x)
-        if (M[u] == kFree) M[u] = (int32_t)u;
-}
-
 // ---------------------------------------------------------------------------------------
-// host driver
+// host side
 // ---------------------------------------------------------------------------------------
-static int choose_group(const Graph *g) {
-    const double avg = g->n ? (double)g->nnz / g->n : 0.0;
-    if (avg <= 3.0) return 4;
-    if (avg <= 6.5) return 8;
+static int choose_group(double avg_deg) {
+    // lanes per vertex in phase 0: about one arc per lane
+    if (avg_deg <= 1.5) return 1;
+    if (avg_deg <= 3.0) return 2;
+    if (avg_deg <= 6.5) return 4;
+    if (avg_deg <= 13.0) return 8;
     return 16;
 }
 
-template <int G>
-static void launch_round(Ctx *ctx, const Graph *g, int32_t *M, const MatchBufs &b, int round) {
-    LevelCtl *ctl = ctx->ctl;
-    const int p = round & 1;
-    const int grid = persistent_grid(ctx, ctx->max_threads_sm / kBlock);
-    {
-        LaunchScope ls(ctx, GP_K_PROPOSE);
-        if (round == 1) {
-            k_propose_round1<G><<<grid, kBlock, 0, ctx->stream>>>(g->n, g->adjp, g->adjncy, g->adjwgt, M, b.P, b,
-                                                                  ctl);
-        } else {
-            k_propose_list<G><<<grid, kBlock, 0, ctx->stream>>>(g->adjp, g->adjncy, g->adjwgt, M, b.P, b.Rs[p],
-                                                                &ctl->cnt[p].r_small);
-        }
-        ++ctx->launches;
+int match_grid(Ctx *ctx) {
+    static int per_sm = -1;
+    if (per_sm < 0) {
+        int b = 0;
+        cudaFuncSetAttribute(k_match_level, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(MatchSmem));
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_match_level, kNT, sizeof(MatchSmem));
+        per_sm = b > 0 ? (b > 2 ? 2 : b) : 1;
     }
-    {
-        LaunchScope ls(ctx, GP_K_PROPOSE);
-        if (round == 1)
-            k_propose_big<false><<<grid, kBlock, 0, ctx->stream>>>(g->adjp, g->adjncy, g->adjwgt, M, b.P, b.Rc[p],
-                                                                   &ctl->cnt[p].r_cta, b.Rw[p], &ctl->cnt[p].r_warp,
-                                                                   ctl);
-        else
-            k_propose_big<true><<<grid, kBlock, 0, ctx->stream>>>(g->adjp, g->adjncy, g->adjwgt, M, b.P, b.Rc[p],
-                                                                  &ctl->cnt[p].r_cta, b.Rw[p], &ctl->cnt[p].r_warp,
-                                                                  ctl);
-        ++ctx->launches;
-    }
-    if (round > 1) {
-        k_count_rows<<<1, 32, 0, ctx->stream>>>(&ctl->cnt[p].r_small, &ctl->cnt[p].r_warp, &ctl->cnt[p].r_cta, ctl);
-        ++ctx->launches;
-    }
-    {
-        LaunchScope ls(ctx, GP_K_COMMIT);
-        if (round == 1)
-            k_commit<true, G><<<grid, kBlock, 0, ctx->stream>>>(g->n, g->adjp, M, b.P, b, ctl, p);
-        else
-            k_commit<false, G><<<grid, kBlock, 0, ctx->stream>>>(g->n, g->adjp, M, b.P, b, ctl, p);
-        ++ctx->launches;
-    }
+    return ctx->num_sms * per_sm;
 }
 
-gp_status match_level(Ctx *ctx, const Graph *g, int32_t *M, int32_t max_rounds, bool leftover,
-                      MatchResult *res) {
-    const int32_t n = g->n;
-    *res = MatchResult();
-    if (n == 0) return GP_OK;
-    // scratch: P, L[2], Rs[2], Rw[2], Rc[2]
-    const size_t nn = (size_t)n;
-    gp_status st = ensure_scratch(ctx, sizeof(int32_t) * nn * 9);
-    if (st != GP_OK) return st;
-    int32_t *base = (int32_t *)ctx->scratch;
-    MatchBufs b;
-    b.P = base;
-    for (int q = 0; q < 2; ++q) {
-        b.L[q] = base + nn * (1 + q);
-        b.Rs[q] = base + nn * (3 + q);
-        b.Rw[q] = base + nn * (5 + q);
-        b.Rc[q] = base + nn * (7 + q);
-    }
-    GP_CUDA(cudaMemsetAsync(ctx->ctl, 0, sizeof(LevelCtl), ctx->stream));
-    const int G = choose_group(g);
-    const int batch = (max_rounds > 0) ? 1 : 4;
-    int round = 1;
-    bool done = false;
-    while (!done) {
-        for (int k = 0; k < batch; ++k, ++round) {
-            if (max_rounds > 0 && round > max_rounds) break;
-            if (G == 4) launch_round<4>(ctx, g, M, b, round);
-            else if (G == 8) launch_round<8>(ctx, g, M, b, round);
-            else launch_round<16>(ctx, g, M, b, round);
-        }
-        GP_CUDA(cudaGetLastError());
-        GP_CUDA(cudaMemcpyAsync(ctx->ctl_host, ctx->ctl, sizeof(LevelCtl), cudaMemcpyDeviceToHost, ctx->stream));
-        GP_CUDA(cudaStreamSynchronize(ctx->stream));
-        const int next_parity = round & 1;  // parity the next round would read
-        const bool live_left = ctx->ctl_host->cnt[next_parity].live > 0;
-        if (!live_left) {
-            done = true;
-            res->maximal = 1;
-        } else if (max_rounds > 0 && round > max_rounds) {
-            // capped with live vertices left: maximal iff none of them still has a free
-            // neighbour after the rescans the next round would do
-            done = true;
-            const int p = round & 1;
-            const int grid = persistent_grid(ctx, ctx->max_threads_sm / kBlock);
-            if (G == 4) k_propose_list<4><<<grid, kBlock, 0, ctx->stream>>>(g->adjp, g->adjncy, g->adjwgt, M, b.P, b.Rs[p], &ctx->ctl->cnt[p].r_small);
-            else if (G == 8) k_propose_list<8><<<grid, kBlock, 0, ctx->stream>>>(g->adjp, g->adjncy, g->adjwgt, M, b.P, b.Rs[p], &ctx->ctl->cnt[p].r_small);
-            else k_propose_list<16><<<grid, kBlock, 0, ctx->stream>>>(g->adjp, g->adjncy, g->adjwgt, M, b.P, b.Rs[p], &ctx->ctl->cnt[p].r_small);
-            k_propose_big<true><<<grid, kBlock, 0, ctx->stream>>>(g->adjp, g->adjncy, g->adjwgt, M, b.P, b.Rc[p], &ctx->ctl->cnt[p].r_cta, b.Rw[p], &ctx->ctl->cnt[p].r_warp, ctx->ctl);
-            GP_CUDA(cudaMemsetAsync(&ctx->ctl->matches, 0, sizeof(int32_t), ctx->stream));
-            k_count_proposing<<<grid, kBlock, 0, ctx->stream>>>(b.L[p], &ctx->ctl->cnt[p].live, b.P, &ctx->ctl->matches);
-            ctx->launches += 3;
-            GP_CUDA(cudaMemcpyAsync(ctx->ctl_host, ctx->ctl, sizeof(LevelCtl), cudaMemcpyDeviceToHost, ctx->stream));
-            GP_CUDA(cudaStreamSynchronize(ctx->stream));
-            res->maximal = ctx->ctl_host->matches == 0;
-        }
-    }
-    res->rounds = ctx->ctl_host->rounds;
-    res->arcs_scanned = (int64_t)ctx->ctl_host->arcs_scanned;
-    res->rows_scanned = (int64_t)ctx->ctl_host->rows_scanned + n;
-    res->live_visits = (int64_t)ctx->ctl_host->live_visits;
-    if (leftover) {
-        LaunchScope ls(ctx, GP_K_OTHER);
-        k_leftover<<<persistent_grid(ctx, 4), kBlock, 0, ctx->stream>>>(n, M);
-        ++ctx->launches;
-        GP_CUDA(cudaGetLastError());
-    }
+gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl, int32_t max_rounds,
+                        bool leftover, double avg_deg_hint) {
+    MatchArgs a;
+    a.in = lb.in;
+    a.adjp = lb.adjp;
+    a.adjncy = lb.adjncy;
+    a.adjwgt = lb.adjwgt;
+    a.M = M;
+    a.P[0] = lb.P[0];
+    a.P[1] = lb.P[1];
+    a.L[0] = lb.L[0];
+    a.L[1] = lb.L[1];
+    a.H = lb.H;
+    a.ctl = ctl;
+    a.max_rounds = max_rounds;
+    a.leftover = leftover ? 1 : 0;
+    a.G = choose_group(avg_deg_hint);
+    void *args[] = {&a};
+    LaunchScope ls(ctx, GP_K_PROPOSE);
+    GP_CUDA(cudaLaunchCooperativeKernel((const void *)k_match_level, dim3(match_grid(ctx)), dim3(kNT), args,
+                                        sizeof(MatchSmem), ctx->stream));
+    ++ctx->launches;
     return GP_OK;
 }
 

@@ -1,9 +1,7 @@
 #!/bin/bash
-# one GPU round-trip: device info, build+smoke, parity tests, a short bench (run under gpurun)
+# one GPU round-trip with hard timeouts: debug parity, smoke, GPU tests, a short bench
 mkdir -p gpurun_out
-set -x
-nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,memory.total --format=csv
-python -c "import torch;p=torch.cuda.get_device_properties(0);print(p)"
-python -c "import __graft_entry__ as e; e.build(); e.smoke()" 2>&1 | tail -5
-timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -25
-timeout 600 python bench.py --steps 5 --warmup 3 --no-cpu-baseline 2>&1 | tail -5
+timeout 180 python -u scripts/debug_small.py 2>&1 | tail -12
+timeout 120 python -u -c "import __graft_entry__ as e; e.build(); e.smoke()" 2>&1 | tail -3
+timeout 900 python -m pytest tests -m gpu -x -q --deselect tests/test_gpu_full.py::test_full_rmat_s24 2>&1 | tail -15
+timeout 300 python -u bench.py --steps 10 --warmup 3 --no-cpu-baseline 2>&1 | tail -3

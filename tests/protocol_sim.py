@@ -1,0 +1,88 @@
+"""Sequential simulations of the GPU kernels' protocols (test infrastructure).
+
+These re-state, in plain Python, the phase structure the CUDA kernels use so
+that the protocol itself -- fused commit_k + propose_{k+1} rounds over double-buffered
+proposals, lazy rescans, the "free after round k" test, the round counting -- can be checked
+against the oracle on the CPU.  Concurrency inside a phase is modelled by processing the
+vertices of a phase in a random order while the writes of that phase (M, and NONE into the
+read buffer for dying vertices) become visible immediately, which is the most adversarial
+legal interleaving for the reads the kernel performs.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+FREE = -1
+NONE = -1
+
+
+def _key(w, v):
+    return (int(w) << 32) | (0xFFFFFFFF - int(v))
+
+
+def simulate_match(adjp, adjncy, adjwgt, seed=0, max_rounds=0):
+    rng = np.random.default_rng(seed)
+    n = len(adjp) - 1
+    M = np.full(n, FREE, dtype=np.int64)
+    P = [np.full(n, 123456789, dtype=np.int64), np.full(n, 987654321, dtype=np.int64)]  # garbage
+    # phase 0: round-1 proposals of every vertex
+    for u in rng.permutation(n):
+        best = 0
+        for j in range(adjp[u], adjp[u + 1]):
+            best = max(best, _key(adjwgt[j], adjncy[j]))
+        p = NONE if best == 0 else 0xFFFFFFFF - (best & 0xFFFFFFFF)
+        P[1][u] = p
+        if p == NONE:
+            P[0][u] = NONE
+    live = [u for u in range(n) if P[1][u] != NONE]
+    rounds = 0
+    maximal = False
+    k = 1
+    while True:
+        Pk, Pn = P[k & 1], P[(k + 1) & 1]
+        made = 0
+        nxt = []
+
+        def free_after(x):
+            if M[x] != FREE:
+                return False
+            px = Pk[x]
+            return not (px >= 0 and Pk[px] == x)
+
+        for u in rng.permutation(live) if live else []:
+            p = Pk[u]
+            if p == NONE:
+                continue
+            q = Pk[p]
+            if q == u:
+                M[u] = p
+                Pn[u] = p
+                made += 1
+            elif not (q >= 0 and Pk[q] == p):
+                Pn[u] = p
+                nxt.append(u)
+            else:
+                best = 0
+                for j in range(adjp[u], adjp[u + 1]):
+                    x = adjncy[j]
+                    if free_after(x):
+                        best = max(best, _key(adjwgt[j], x))
+                b = NONE if best == 0 else 0xFFFFFFFF - (best & 0xFFFFFFFF)
+                Pn[u] = b
+                if b == NONE:
+                    Pk[u] = NONE
+                else:
+                    nxt.append(u)
+        if made > 0:
+            rounds += 1
+        live = nxt
+        if not live:
+            maximal = True
+            break
+        if max_rounds and rounds >= max_rounds:
+            break
+        k += 1
+    for u in range(n):
+        if M[u] == FREE:
+            M[u] = u
+    return M, rounds, maximal
