@@ -247,6 +247,14 @@ def run_ours(args, rank, world, local_rank):
     # end-to-end through the C ABI with host buffers
     host = {k: g[k].cpu().pin_memory() for k in ("adjp", "adjncy", "adjwgt", "vwgt")}
     h2d = sum(t.numel() * 4 for t in host.values())
+    # pinned result buffers sized from the warm-up hierarchy (what a partitioner keeps:
+    # every level's CM for projection, and the coarsest graph)
+    cm_bufs = [torch.empty(l["n"], dtype=torch.int32).pin_memory() for l in levels]
+    last_l = levels[-1]
+    last_bufs = {"adjp": torch.empty(last_l["n_coarse"] + 1, dtype=torch.int32).pin_memory(),
+                 "adjncy": torch.empty(last_l["cnnz"], dtype=torch.int32).pin_memory(),
+                 "adjwgt": torch.empty(last_l["cnnz"], dtype=torch.int32).pin_memory(),
+                 "vwgt": torch.empty(last_l["n_coarse"], dtype=torch.int32).pin_memory()}
     e2e_ms = []
     d2h = 0
     for it in range(max(2, min(args.steps, 5)) + 1):
@@ -258,9 +266,9 @@ def run_ours(args, rank, world, local_rank):
         hh = gh.coarsen_to(threshold)
         nb = 0
         for i in range(len(hh)):
-            _, c = hh.download_level(i)
+            _, c = hh.download_level(i, cmap=cm_bufs[i], want_match=False)
             nb += c.numel() * 4
-        last = hh.level(len(hh) - 1).coarse.download()
+        last = hh.level(len(hh) - 1).coarse.download(out=last_bufs)
         nb += sum(last[k].numel() * 4 for k in ("adjp", "adjncy", "adjwgt", "vwgt"))
         b.record(stream)
         torch.cuda.synchronize()

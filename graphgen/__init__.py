@@ -322,6 +322,11 @@ def from_edge_list(n: int, edges, vwgt=None) -> Dict[str, object]:
 # --------------------------------------------------------------------------------------
 # the five BASELINE.json configs (full size) and reduced-size versions for tests
 # --------------------------------------------------------------------------------------
+# Weight ranges keep sum(adjwgt) <= INT32_MAX at full size (reading R14): C4 has ~5.2e8 arcs
+# (mean weight 2.5 -> ~1.3e9), C5 ~1.7e8 arcs (mean 5.5 -> ~9.2e8).  C2/C3 use [1,100].
+C4_WMAX = 4
+C5_WMAX = 10
+
 CONFIGS = {
     "C1": dict(desc="64x64 2D grid graph (4,096 vertices, unit weights), coarsen to <=100", threshold=100),
     "C2": dict(desc="random geometric graph rgg n=2^20, avg degree ~13", threshold=100),
@@ -340,7 +345,7 @@ def make_config(name: str, device: str = "cpu", reduce: int = 0) -> Dict[str, ob
     if name == "C3":
         return delaunay_like(2048 >> (reduce // 2), device=device)
     if name == "C4":
-        return rmat(24 - reduce, 16, device=device)
+        return rmat(24 - reduce, 16, wmax=C4_WMAX, device=device)
     if name == "C5":
-        return road_like(8192 >> (reduce // 2), device=device)
+        return road_like(8192 >> (reduce // 2), wmax=C5_WMAX, device=device)
     raise KeyError(name)

@@ -13,6 +13,16 @@ __device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31u; }
 // Watchdog of every spin loop: a protocol bug traps (cudaErrorLaunchFailure) after ~4 s
 // instead of hanging the device.
 __device__ __forceinline__ long long spin_start() { return clock64(); }
+
+__device__ __forceinline__ unsigned long long globaltimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+// block 0 / thread 0 records a phase timestamp (slot i < kTrace)
+__device__ __forceinline__ void trace_mark(unsigned long long *trace, int i) {
+    if (blockIdx.x == 0 && threadIdx.x == 0 && i < kTrace) trace[i] = globaltimer();
+}
 __device__ __forceinline__ void spin_check(long long t0) {
     if (clock64() - t0 > (8ll << 30)) __trap();
 }
@@ -132,8 +142,11 @@ __device__ __forceinline__ int32_t lookback_prefix(unsigned long long *status, u
         if (idx >= 0) {
             unsigned long long s;
             const long long guard = spin_start();
+            unsigned backoff = 0;
             do {
                 spin_check(guard);
+                if (backoff) __nanosleep(backoff);
+                backoff = backoff ? min(backoff * 2, 512u) : 32u;
                 s = lb_load(status + idx);
                 flag = ((uint32_t)(s >> 32) >> 2) == epoch ? ((uint32_t)(s >> 32) & 3u) : 0u;
             } while (flag == 0);

@@ -31,7 +31,10 @@ struct RoundSlot {
     int32_t pad;
 };
 
+constexpr int kTrace = 48;  // phase timestamps per kernel (debug tracing)
+
 struct MatchCtl {
+    unsigned long long trace[kTrace];  // %globaltimer at phase boundaries (block 0; debug)
     unsigned bar[2];   // grid barrier
     RoundSlot slot[4]; // ring by round number
     int32_t rounds, maximal;
@@ -40,6 +43,7 @@ struct MatchCtl {
 };
 
 struct ContractCtl {
+    unsigned long long trace[kTrace];
     unsigned bar[2];
     unsigned tile_ctr[2];
     int32_t n_coarse, cnnz, n_huge;
@@ -70,7 +74,8 @@ struct LevelBufs {
     const SizeRec *in;  // sizes (+ stop flag) of this level's input graph
     const int32_t *adjp, *adjncy, *adjwgt, *vwgt;
     int32_t *P[2], *L[2], *H;                         // matching scratch
-    int32_t *leaders, *off, *cnt, *tile_start, *huge;  // contraction scratch
+    int32_t *leaders, *off, *cnt, *tile_start, *huge, *rlen;  // contraction scratch
+    int4 *seg;
     unsigned long long *gkeys;
 };
 

@@ -35,6 +35,8 @@ namespace gp {
 
 constexpr int kNT = 512;            // threads per CTA of the persistent kernels
 constexpr int kStageArcs = 4096;    // arcs per TMA stage (adjncy + adjwgt = 32 KB)
+constexpr int kStages = 3;          // TMA pipeline depth of phase 0
+constexpr int kMaxVch = 1024;       // vertices per phase-0 chunk (adjp slice staged too)
 constexpr int kThreadDeg = 32;      // phase-k rescans up to this many arcs: one thread
 constexpr int kHubDeg = 4096;       // rows longer than this: one CTA each (hub phase)
 
@@ -48,15 +50,17 @@ struct MatchArgs {
     MatchCtl *ctl;
     int32_t max_rounds;
     int32_t leftover;
-    int32_t G;  // lanes per vertex in phase 0 (1, 2, 4, 8 or 16)
+    int32_t G;    // lanes per vertex in phase 0 (1, 2, 4, 8 or 16)
+    int32_t vch;  // vertices per phase-0 chunk (about 80 % of a stage at the average degree)
 };
 
 struct MatchSmem {
-    int32_t adj[2][kStageArcs];
-    int32_t wgt[2][kStageArcs];
-    uint64_t bar[2];
-    int32_t a0[2];    // aligned first arc of the staged chunk
-    int32_t fits[2];  // chunk staged (1) or fallback (0)
+    int32_t adj[kStages][kStageArcs];
+    int32_t wgt[kStages][kStageArcs];
+    int32_t ap[kStages][kMaxVch + 8];  // adjp[v0 .. v0+vch] of the staged chunk
+    uint64_t bar[kStages];
+    int32_t a0[kStages];    // aligned first arc of the staged chunk
+    int32_t fits[kStages];  // 1 staged, 2 empty, 0 fallback
     int32_t scratch[40];
     unsigned long long red[kNT / 32];
 };
@@ -88,108 +92,117 @@ __device__ __forceinline__ unsigned long long group_max_rt(unsigned long long k,
 // ---------------------------------------------------------------------------------------
 // phase 0: round-1 proposals of every vertex
 // ---------------------------------------------------------------------------------------
-__device__ __forceinline__ void chunk_bounds(const MatchArgs &a, int32_t n, int32_t vch, long long c, int32_t &A0,
-                                             int32_t &A1, int32_t &fits) {
-    const long long v0 = c * vch;
-    const long long v1 = min((long long)n, v0 + vch);
-    const int32_t s = __ldg(a.adjp + v0), e = __ldg(a.adjp + v1);
-    A0 = s & ~3;
-    A1 = (e + 3) & ~3;
-    fits = (A1 - A0) <= kStageArcs;
+// thread 0: stage chunk c (bounds A0/A1 already loaded) into stage st with TMA bulk copies
+// of its adjp slice and arc range, or mark it as fallback (too many arcs) / empty
+__device__ __forceinline__ void stage_chunk(const MatchArgs &a, MatchSmem &sm, int32_t n, long long c, int32_t s,
+                                            int32_t e, int st) {
+    const int32_t A0 = s & ~3, A1 = (e + 3) & ~3;
+    sm.a0[st] = A0;
+    const bool fits = (A1 - A0) <= kStageArcs;
+    const long long nv = min((long long)a.vch, (long long)n - c * a.vch);   // vertices in the chunk
+    const unsigned apb = (unsigned)((nv + 1 + 3) & ~3ll) * 4u;  // adjp slice (<= adjp[n+3]), 16-byte multiple
+    if (fits) {
+        sm.fits[st] = 1;
+        mbar_arrive_expect_tx(&sm.bar[st], apb + (unsigned)(A1 - A0) * 8u);
+        tma_load_1d(sm.ap[st], a.adjp + c * a.vch, apb, &sm.bar[st]);
+        if (A1 > A0) {
+            tma_load_1d(sm.adj[st], a.adjncy + A0, (unsigned)(A1 - A0) * 4u, &sm.bar[st]);
+            tma_load_1d(sm.wgt[st], a.adjwgt + A0, (unsigned)(A1 - A0) * 4u, &sm.bar[st]);
+        }
+    } else {
+        sm.fits[st] = 0;
+    }
+}
+
+__device__ __forceinline__ void load_bounds(const MatchArgs &a, int32_t n, long long nchunks, long long c, int32_t &s,
+                                            int32_t &e) {
+    s = e = 0;
+    if (c < nchunks) {
+        s = __ldg(a.adjp + c * a.vch);
+        e = __ldg(a.adjp + min((long long)n, (c + 1) * a.vch));
+    }
 }
 
 __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned long long &scanned) {
     const int G = a.G;
-    const int vch = kNT / G;
-    const long long nchunks = ((long long)n + vch - 1) / vch;
-    const int t = threadIdx.x, gl = t % G;
+    const int ngroups = kNT / G;
+    const long long nchunks = ((long long)n + a.vch - 1) / a.vch;
+    const int t = threadIdx.x, gl = t % G, grp = t / G;
     int32_t *P1 = a.P[1], *P0 = a.P[0];
+    int32_t nb_s = 0, nb_e = 0;  // thread 0: prefetched bounds of the next chunk to stage
     if (t == 0) {
-        mbar_init(&sm.bar[0], 1);
-        mbar_init(&sm.bar[1], 1);
+        for (int q = 0; q < kStages; ++q) mbar_init(&sm.bar[q], 1);
         fence_mbar_init();
-    }
-    __syncthreads();
-    // prologue: bounds + TMA for the first two chunks of this CTA
-    if (t == 0) {
-        for (int i = 0; i < 2; ++i) {
-            const long long c = blockIdx.x + (long long)i * gridDim.x;
+        for (int q = 0; q < kStages; ++q) {
+            const long long c = blockIdx.x + (long long)q * gridDim.x;
             if (c < nchunks) {
-                int32_t A0, A1, f;
-                chunk_bounds(a, n, vch, c, A0, A1, f);
-                sm.a0[i] = A0;
-                sm.fits[i] = f;
-                if (f && A1 > A0) {
-                    mbar_arrive_expect_tx(&sm.bar[i], (unsigned)(A1 - A0) * 8u);
-                    tma_load_1d(sm.adj[i], a.adjncy + A0, (unsigned)(A1 - A0) * 4u, &sm.bar[i]);
-                    tma_load_1d(sm.wgt[i], a.adjwgt + A0, (unsigned)(A1 - A0) * 4u, &sm.bar[i]);
-                } else if (f) {
-                    sm.fits[i] = 2;  // empty chunk: nothing to wait for
-                }
+                int32_t cs, ce;
+                load_bounds(a, n, nchunks, c, cs, ce);
+                stage_chunk(a, sm, n, c, cs, ce, q);
             }
         }
+        load_bounds(a, n, nchunks, blockIdx.x + (long long)kStages * gridDim.x, nb_s, nb_e);
     }
     __syncthreads();
-    unsigned uses[2] = {0, 0};
+    unsigned uses[kStages] = {};
     for (long long i = 0;; ++i) {
         const long long c = blockIdx.x + i * gridDim.x;
         if (c >= nchunks) break;
-        const int st = (int)(i & 1);
-        const int fits = sm.fits[st];
+        const int st = (int)(i % kStages);
+        const bool fits = sm.fits[st] != 0;
         const int32_t A0 = sm.a0[st];
-        if (fits == 1) {
+        if (fits) {
             mbar_wait(&sm.bar[st], uses[st] & 1u);
             ++uses[st];
         }
-        const long long v = c * vch + t / G;
-        const bool valid = v < n;
-        int32_t s = 0, e = 0;
-        if (valid) {
-            s = __ldg(a.adjp + v);
-            e = __ldg(a.adjp + v + 1);
-        }
-        unsigned long long key = 0;
-        bool hub = false;
-        if (fits) {
-            const int32_t *sa = sm.adj[st], *sw = sm.wgt[st];
-            for (int32_t j = s - A0 + gl; j < e - A0; j += G) key = umax64(key, pack_key(sw[j], sa[j]));
-        } else if (valid) {
-            if (e - s > kHubDeg) {
-                hub = true;
-            } else {
-                for (int32_t j = s + gl; j < e; j += G) key = umax64(key, pack_key(__ldg(a.adjwgt + j), __ldg(a.adjncy + j)));
+        const long long vbeg = c * a.vch, vend = min((long long)n, vbeg + a.vch);
+        const int32_t *sp = sm.ap[st];
+        // a uniform trip count per warp keeps the group shuffles converged
+        for (long long vb = vbeg; vb < vend; vb += ngroups) {
+            const long long v = vb + grp;
+            const bool valid = v < vend;
+            int32_t s = 0, e = 0;
+            if (valid) {
+                if (fits) {
+                    s = sp[v - vbeg];
+                    e = sp[v - vbeg + 1];
+                } else {
+                    s = __ldg(a.adjp + v);
+                    e = __ldg(a.adjp + v + 1);
+                }
             }
-        }
-        key = group_max_rt(key, G);
-        if (valid && gl == 0) {
-            a.M[v] = kFree;
-            if (hub) {
-                a.H[atomicAdd(&a.ctl->slot[1].nhub, 1)] = (int32_t)v;
-            } else {
-                const int32_t p = key_vertex(key);
-                P1[v] = p;
-                if (p == kNone) P0[v] = kNone;  // dead vertices: NONE in both buffers
-                scanned += (unsigned long long)(e - s);
+            unsigned long long key = 0;
+            bool hub = false;
+            if (fits) {
+                const int32_t *sa = sm.adj[st], *sw = sm.wgt[st];
+                for (int32_t j = s - A0 + gl; j < e - A0; j += G) key = umax64(key, pack_key(sw[j], sa[j]));
+            } else if (valid) {
+                if (e - s > kHubDeg) {
+                    hub = true;
+                } else {
+                    for (int32_t j = s + gl; j < e; j += G)
+                        key = umax64(key, pack_key(__ldg(a.adjwgt + j), __ldg(a.adjncy + j)));
+                }
+            }
+            key = group_max_rt(key, G);
+            if (valid && gl == 0) {
+                a.M[v] = kFree;
+                if (hub) {
+                    a.H[atomicAdd(&a.ctl->slot[1].nhub, 1)] = (int32_t)v;
+                } else {
+                    const int32_t p = key_vertex(key);
+                    P1[v] = p;
+                    if (p == kNone) P0[v] = kNone;  // dead vertices: NONE in both buffers
+                    scanned += (unsigned long long)(e - s);
+                }
             }
         }
         __syncthreads();  // stage `st` is free again
         if (t == 0) {
-            const long long c2 = blockIdx.x + (i + 2) * gridDim.x;
-            if (c2 < nchunks) {
-                int32_t A0n, A1n, f;
-                chunk_bounds(a, n, vch, c2, A0n, A1n, f);
-                sm.a0[st] = A0n;
-                sm.fits[st] = f;
-                if (f && A1n > A0n) {
-                    mbar_arrive_expect_tx(&sm.bar[st], (unsigned)(A1n - A0n) * 8u);
-                    tma_load_1d(sm.adj[st], a.adjncy + A0n, (unsigned)(A1n - A0n) * 4u, &sm.bar[st]);
-                    tma_load_1d(sm.wgt[st], a.adjwgt + A0n, (unsigned)(A1n - A0n) * 4u, &sm.bar[st]);
-                } else if (f) {
-                    sm.fits[st] = 2;
-                }
-            }
+            const long long c2 = blockIdx.x + (i + kStages) * gridDim.x;
+            if (c2 < nchunks) stage_chunk(a, sm, n, c2, nb_s, nb_e, st);
+            load_bounds(a, n, nchunks, c2 + gridDim.x, nb_s, nb_e);  // in flight during the next chunk
         }
-        __syncthreads();
     }
 }
 
@@ -263,10 +276,23 @@ __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int
                     e = __ldg(a.adjp + u + 1);
                     ++rows;
                     if (e - s <= kThreadDeg) {
+                        // batches of 8 arcs: every dependent load level is issued for the
+                        // whole batch at once (arc -> M[x] -> P_k[x] -> P_k[P_k[x]])
                         unsigned long long key = 0;
-                        for (int32_t j = s; j < e; ++j) {
-                            const int32_t x = __ldg(a.adjncy + j);
-                            if (free_after(x, a.M, Pk)) key = umax64(key, pack_key(__ldg(a.adjwgt + j), x));
+                        for (int32_t j0 = s; j0 < e; j0 += 8) {
+                            int32_t x[8], m[8], px[8], pp[8];
+#pragma unroll
+                            for (int b = 0; b < 8; ++b) x[b] = (j0 + b < e) ? __ldg(a.adjncy + j0 + b) : -1;
+#pragma unroll
+                            for (int b = 0; b < 8; ++b) m[b] = (x[b] >= 0) ? ldcg(a.M + x[b]) : 0;
+#pragma unroll
+                            for (int b = 0; b < 8; ++b) px[b] = (x[b] >= 0 && m[b] == kFree) ? ldcg(Pk + x[b]) : -1;
+#pragma unroll
+                            for (int b = 0; b < 8; ++b) pp[b] = (px[b] >= 0) ? ldcg(Pk + px[b]) : -1;
+#pragma unroll
+                            for (int b = 0; b < 8; ++b)
+                                if (x[b] >= 0 && m[b] == kFree && pp[b] != x[b])
+                                    key = umax64(key, pack_key(__ldg(a.adjwgt + j0 + b), x[b]));
                         }
                         scanned += (unsigned long long)(e - s);
                         const int32_t b = key_vertex(key);
@@ -314,9 +340,12 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
     const int32_t n = in->n;
     if (n <= 0) return;
     unsigned long long scanned = 0, rows = 0, visits = 0;
-
+    int tr = 0;
+    trace_mark(ctl->trace, tr++);
     phase0(a, sm, n, scanned);
+    trace_mark(ctl->trace, tr++);
     grid_barrier(ctl->bar);
+    trace_mark(ctl->trace, tr++);
     {
         const int32_t nh = *(volatile int32_t *)&ctl->slot[1].nhub;
         if (nh > 0) {
@@ -338,7 +367,9 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
         phase_k(a, sm, n, k, len, scanned, rows, visits, made);
         made = warp_sum(made);
         if ((threadIdx.x & 31) == 0 && made) atomicAdd(&ctl->slot[k & 3].matches, made);
+        trace_mark(ctl->trace, tr++);
         grid_barrier(ctl->bar);
+        trace_mark(ctl->trace, tr++);
         const int32_t nh = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].nhub;
         if (nh > 0) {
             hub_phase(a, sm, nh, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1], &ctl->slot[(k + 1) & 3].live,
@@ -353,6 +384,7 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
         }
         if (a.max_rounds > 0 && rounds >= a.max_rounds) break;
     }
+    trace_mark(ctl->trace, tr++);
     if (a.leftover) {
         for (long long u = (long long)blockIdx.x * kNT + threadIdx.x; u < n; u += (long long)gridDim.x * kNT)
             if (a.M[u] == kFree) a.M[u] = (int32_t)u;
@@ -411,6 +443,12 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     a.max_rounds = max_rounds;
     a.leftover = leftover ? 1 : 0;
     a.G = choose_group(avg_deg_hint);
+    {
+        const double d = avg_deg_hint > 0.5 ? avg_deg_hint : 0.5;
+        int v = (int)(0.8 * kStageArcs / d);
+        v = (v / 32) * 32;
+        a.vch = v < 32 ? 32 : (v > kMaxVch ? kMaxVch : v);
+    }
     void *args[] = {&a};
     LaunchScope ls(ctx, GP_K_PROPOSE);
     GP_CUDA(cudaLaunchCooperativeKernel((const void *)k_match_level, dim3(match_grid(ctx)), dim3(kNT), args,

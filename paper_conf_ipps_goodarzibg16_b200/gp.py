@@ -200,11 +200,13 @@ class Graph:
     def nnz(self) -> int:
         return self.view()[1]
 
-    def download(self) -> Dict[str, torch.Tensor]:
-        """Copy the CSR arrays to host int32 tensors (gp_graph_download)."""
+    def download(self, out: Optional[Dict[str, torch.Tensor]] = None) -> Dict[str, torch.Tensor]:
+        """Copy the CSR arrays to host int32 tensors (gp_graph_download); `out` may supply
+        preallocated (e.g. pinned) host tensors of at least the right sizes."""
         n, nnz = self.view()
-        out = {k: torch.empty(sz, dtype=torch.int32) for k, sz in
-               (("adjp", n + 1), ("adjncy", nnz), ("adjwgt", nnz), ("vwgt", n))}
+        if out is None:
+            out = {k: torch.empty(sz, dtype=torch.int32) for k, sz in
+                   (("adjp", n + 1), ("adjncy", nnz), ("adjwgt", nnz), ("vwgt", n))}
         _check(_lib.gp_graph_download(self.handle, out["adjp"].data_ptr(), out["adjncy"].data_ptr(),
                                       out["adjwgt"].data_ptr(), out["vwgt"].data_ptr()), "gp_graph_download")
         out["n"], out["nnz"] = n, nnz
@@ -278,12 +280,15 @@ class Hierarchy:
     def levels(self) -> List[LevelInfo]:
         return [self.level(i) for i in range(len(self))]
 
-    def download_level(self, i: int):
-        """(match, cmap) of level i as host int32 tensors."""
+    def download_level(self, i: int, match: Optional[torch.Tensor] = None, cmap: Optional[torch.Tensor] = None,
+                       want_match: bool = True):
+        """(match, cmap) of level i as host int32 tensors (optionally preallocated/pinned);
+        want_match=False skips the match copy and returns (None, cmap)."""
         info = self.level(i)
-        m = torch.empty(info.n, dtype=torch.int32)
-        c = torch.empty(info.n, dtype=torch.int32)
-        _check(_lib.gp_hier_download_level(self.handle, i, m.data_ptr(), c.data_ptr()), "gp_hier_download_level")
+        m = None if not want_match else (match if match is not None else torch.empty(info.n, dtype=torch.int32))
+        c = cmap if cmap is not None else torch.empty(info.n, dtype=torch.int32)
+        _check(_lib.gp_hier_download_level(self.handle, i, m.data_ptr() if m is not None else None, c.data_ptr()),
+               "gp_hier_download_level")
         return m, c
 
 
