@@ -8,19 +8,25 @@
 // final arrays (P20.s22-26).
 //
 // B200 design:
-//  C1  one decoupled look-back pass over u in [0,n): leftover self-match, leader flags,
-//      exclusive scan (= the paper's inclusive scan minus one), leader list, the partner's
-//      CM (written by its leader: no second pass), cvwgt, and the exclusive prefix `off`
-//      of the merged-row upper bounds ub = deg(u) + deg(partner) (P20.s6-8).  Coarse rows
-//      are cut into tiles of kTileArcs upper-bound entries; C1 also records each tile's
-//      first row.
-//  C1b (only if some ub > kTileArcs, e.g. R-MAT hubs) such rows are merged by a whole CTA
-//      in global scratch.
-//  C2  one pass over the tiles in order: every row of the tile is merged into the tile's
-//      shared-memory slots (ub <= 16: one thread, registers + bitonic network; longer: one
-//      warp, shared-memory bitonic sort), counted, the tile total gets its global prefix
-//      by decoupled look-back, and the rows are written straight into the final compact
-//      cadjp/cadjncy/cadjwgt (no temporary arrays, no second scan, no copy kernel).
+//  * Work units are WARP tiles: a warp never waits for its CTA, so an SM keeps 32
+//    independent dependent-load chains in flight (a CTA-tile design kept ~4 and was
+//    latency-bound; measured).  No CTA ever waits on another one except at grid barriers.
+//  * Prefixes are "chunked reduce-then-scan": phase A accumulates each tile's aggregate
+//    into the sum of the contiguous chunk of tiles one CTA owns in phase B (integer
+//    atomics: order-free, deterministic); phase B block-scans its chunk once.
+//  C1a warp tiles of 256 vertices: leftover self-match (P18.s12-13), leader flags u<=M[u]
+//      (P18.s18), #leaders and the sum of merged-row upper bounds ub = deg(u)+deg(v)
+//      (P20.s5-8).                                                               | barrier
+//  C1b CM (= the paper's inclusive scan minus one, P18.s20-24; the leader also writes its
+//      partner's CM, P18.s26), cvwgt (P12.s27), the ub prefix `off`, each coarse row's two
+//      fine segments, and C2's warp-tile starts (256 upper-bound entries each). | barrier
+//  C1h (only if some ub > 256): one CTA per such row merges it in shared memory (ub <=
+//      4096) or global scratch and leaves it compacted.                          | barrier
+//  C2a warp tiles: every row is merged (ub <= 16: one thread, registers + bitonic network;
+//      <= 64: the warp, registers + shuffles; <= 256: the warp, shared-memory bitonic sort)
+//      and the tile is written compacted to scratch at its own ub offset, with each row's
+//      tile-local offset and the tile total.                                     | barrier
+//  C2b cadjp and a coalesced copy of every tile into the final compact CSR.
 //  Rows come out sorted by coarse id (R10) with repeated coarse neighbours summed (R8) and
 //  the collapsed edge dropped (R9).
 #include <cuda_runtime.h>
@@ -30,26 +36,27 @@
 
 namespace gp {
 
-constexpr int kCNT = 256;              // threads per CTA (4 co-resident CTAs per SM)
-constexpr int kCItems = 8;             // vertices per thread per C1 tile
-constexpr int kCTileV = kCNT * kCItems;  // 2048 vertices per C1 tile
-constexpr int kTileArcs = 2048;        // C2 tile budget (upper-bound entries); rows with a
-                                       // larger bound are merged by C1b
-constexpr int kTileBuf = 2 * kTileArcs;  // a row starting inside the budget ends within 2x
-constexpr int kNet = 16;               // one-thread merge capacity
-constexpr int kWarpNet = 64;           // one-warp register merge capacity
+constexpr int kCNT = 256;        // threads per CTA (4 co-resident CTAs per SM)
+constexpr int kCW = kCNT / 32;   // warps per CTA
+constexpr int kCItems = 8;       // vertices per lane of a C1 warp tile
+constexpr int kVW = 32 * kCItems;  // 256 vertices per C1 warp tile
+constexpr int kWB = 256;         // C2 warp-tile budget (upper-bound entries)
+constexpr int kCtaRow = 4096;    // C1h: rows up to this bound are merged in shared memory
+constexpr int kNet = 16;         // one-thread merge capacity
+constexpr int kWarpNet = 64;     // one-warp register merge capacity
+constexpr int kBuf = 4096;       // shared u64 buffer (warp regions of 2*kWB / C1h rows / C2b)
 constexpr unsigned long long kMaxKey = ~0ull;
 
 struct ContractArgs {
     const SizeRec *in;  // device: sizes + stop flag of this level's graph
     const int32_t *adjp, *adjncy, *adjwgt, *vwgt;
     int32_t *M, *CM;
-    int32_t *leaders, *off, *cnt, *tile_start, *huge, *rlen;
+    int32_t *off, *cnt, *tile_start, *huge, *lofs;
+    int32_t *tagg1;             // C1 warp-tile aggregates {#leaders, sum ub}
+    int32_t *ttot;              // C2 warp-tile totals
     int4 *seg;                  // per coarse row: {start, deg} of the leader and of the partner
-    unsigned long long *gkeys;  // C1b scratch (nnz entries)
-    unsigned long long *st1;    // C1 look-back status (4 words per tile)
-    unsigned long long *st2;    // C2 look-back status (2 words per tile)
-    uint32_t epoch;
+    unsigned long long *gkeys;  // C1h scratch at off[c] (nnz entries)
+    unsigned long long *tout;   // C2a output scratch at each tile's ub offset (nnz entries)
     int32_t *cadjp, *cadjncy, *cadjwgt, *cvwgt;  // coarse graph (upper-bound sized)
     ContractCtl *ctl;
     SizeRec *out;  // device: sizes + stop decision of the coarse graph
@@ -59,97 +66,13 @@ struct ContractArgs {
 };
 
 struct ContractSmem {
-    unsigned long long buf[kTileBuf];
+    unsigned long long buf[kBuf];
     int32_t scan[40];
-    int32_t tile, prefix, len;
-    unsigned long long prefix2;
-    int32_t wlen[kCNT / 32];
+    int32_t red[2][kCW];
+    int32_t wlen[kCW];
     int32_t lead[kCNT], has[kCNT];
-    int32_t hub_c, hub_o;
+    int32_t len, last;
 };
-
-// ---------------------------------------------------------------------------------------
-// look-back over V values per tile (V in {1,2}); words per tile: V aggregate + V inclusive;
-// a word is valid when its high half equals (epoch | 2^31).
-// ---------------------------------------------------------------------------------------
-template <int V>
-__device__ __forceinline__ void lookback(unsigned long long *st, uint32_t epoch, int tile, const int32_t (&agg)[V],
-                                         int32_t (&prefix)[V]) {
-    // Wide window: lane l inspects the K predecessors pred-l*K .. pred-l*K-K+1, so one step
-    // covers 32*K tiles.  With hundreds of CTAs finishing a wave of tiles at once, the
-    // nearest inclusive prefix is often a whole wave back; a 32-tile window would need
-    // ~wave/32 dependent steps.
-    constexpr int K = 8;
-    const int l = threadIdx.x & 31;
-    const unsigned long long tag = ((unsigned long long)(epoch | 0x80000000u)) << 32;
-    unsigned long long *me = st + (size_t)tile * 2 * V;
-#pragma unroll
-    for (int i = 0; i < V; ++i) prefix[i] = 0;
-    if (tile == 0) {
-        if (l == 0)
-#pragma unroll
-            for (int i = 0; i < V; ++i) lb_store(me + V + i, tag | (uint32_t)agg[i]);
-        return;
-    }
-    if (l == 0)
-#pragma unroll
-        for (int i = 0; i < V; ++i) lb_store(me + i, tag | (uint32_t)agg[i]);
-    int pred = tile - 1;
-    while (true) {
-        // my K entries, nearest first; stop at the first inclusive one
-        int32_t part[V];
-#pragma unroll
-        for (int i = 0; i < V; ++i) part[i] = 0;
-        bool found = false;
-        for (int k = 0; k < K && !found; ++k) {
-            const int idx = pred - l * K - k;
-            if (idx < 0) {
-                found = true;  // before tile 0: an inclusive prefix of 0
-                break;
-            }
-            const unsigned long long *w = st + (size_t)idx * 2 * V;
-            const long long guard = spin_start();
-            unsigned backoff = 0;
-            while (true) {
-                spin_check(guard);
-                bool inc = true, ag = true;
-                unsigned long long wi[V], wa[V];
-#pragma unroll
-                for (int i = 0; i < V; ++i) {
-                    wi[i] = lb_load(w + V + i);
-                    inc &= (wi[i] & 0xFFFFFFFF00000000ull) == tag;
-                }
-                if (inc) {
-#pragma unroll
-                    for (int i = 0; i < V; ++i) part[i] += (int32_t)(uint32_t)wi[i];
-                    found = true;
-                    break;
-                }
-#pragma unroll
-                for (int i = 0; i < V; ++i) {
-                    wa[i] = lb_load(w + i);
-                    ag &= (wa[i] & 0xFFFFFFFF00000000ull) == tag;
-                }
-                if (ag) {
-#pragma unroll
-                    for (int i = 0; i < V; ++i) part[i] += (int32_t)(uint32_t)wa[i];
-                    break;
-                }
-                if (backoff) __nanosleep(backoff);
-                backoff = backoff ? min(backoff * 2, 256u) : 32u;
-            }
-        }
-        const unsigned incl = __ballot_sync(0xffffffffu, found);
-        const int first = incl ? __ffs(incl) - 1 : 32;
-#pragma unroll
-        for (int i = 0; i < V; ++i) prefix[i] += warp_sum(l <= first ? part[i] : 0);
-        if (incl) break;
-        pred -= 32 * K;
-    }
-    if (l == 0)
-#pragma unroll
-        for (int i = 0; i < V; ++i) lb_store(me + V + i, tag | (uint32_t)(prefix[i] + agg[i]));
-}
 
 // ---------------------------------------------------------------------------------------
 // merge helpers
@@ -162,6 +85,87 @@ __device__ __forceinline__ void cswap(unsigned long long &a, unsigned long long 
     const unsigned long long lo = a < b ? a : b, hi = a < b ? b : a;
     a = lo;
     b = hi;
+}
+
+// Batcher odd-even merge sort network for 16 inputs (63 comparators; generated and checked
+// against sorted() offline).
+// sort (cx, w) pairs by cx only: equal coarse ids are summed afterwards, so their order is
+// irrelevant; a comparator is one 32-bit compare and four selects
+__device__ __forceinline__ void cx_sort16(uint32_t (&cx)[16], int32_t (&w)[16]) {
+#define GP_CE(i, j)                                                      \
+    {                                                                    \
+        const bool sw = cx[i] > cx[j];                                   \
+        const uint32_t c0 = sw ? cx[j] : cx[i], c1 = sw ? cx[i] : cx[j]; \
+        const int32_t w0 = sw ? w[j] : w[i], w1 = sw ? w[i] : w[j];      \
+        cx[i] = c0;                                                      \
+        cx[j] = c1;                                                      \
+        w[i] = w0;                                                       \
+        w[j] = w1;                                                       \
+    }
+    GP_CE(0, 1)
+    GP_CE(2, 3)
+    GP_CE(0, 2)
+    GP_CE(1, 3)
+    GP_CE(1, 2)
+    GP_CE(4, 5)
+    GP_CE(6, 7)
+    GP_CE(4, 6)
+    GP_CE(5, 7)
+    GP_CE(5, 6)
+    GP_CE(0, 4)
+    GP_CE(2, 6)
+    GP_CE(2, 4)
+    GP_CE(1, 5)
+    GP_CE(3, 7)
+    GP_CE(3, 5)
+    GP_CE(1, 2)
+    GP_CE(3, 4)
+    GP_CE(5, 6)
+    GP_CE(8, 9)
+    GP_CE(10, 11)
+    GP_CE(8, 10)
+    GP_CE(9, 11)
+    GP_CE(9, 10)
+    GP_CE(12, 13)
+    GP_CE(14, 15)
+    GP_CE(12, 14)
+    GP_CE(13, 15)
+    GP_CE(13, 14)
+    GP_CE(8, 12)
+    GP_CE(10, 14)
+    GP_CE(10, 12)
+    GP_CE(9, 13)
+    GP_CE(11, 15)
+    GP_CE(11, 13)
+    GP_CE(9, 10)
+    GP_CE(11, 12)
+    GP_CE(13, 14)
+    GP_CE(0, 8)
+    GP_CE(4, 12)
+    GP_CE(4, 8)
+    GP_CE(2, 10)
+    GP_CE(6, 14)
+    GP_CE(6, 10)
+    GP_CE(2, 4)
+    GP_CE(6, 8)
+    GP_CE(10, 12)
+    GP_CE(1, 9)
+    GP_CE(5, 13)
+    GP_CE(5, 9)
+    GP_CE(3, 11)
+    GP_CE(7, 15)
+    GP_CE(7, 11)
+    GP_CE(3, 5)
+    GP_CE(7, 9)
+    GP_CE(11, 13)
+    GP_CE(1, 2)
+    GP_CE(3, 4)
+    GP_CE(5, 6)
+    GP_CE(7, 8)
+    GP_CE(9, 10)
+    GP_CE(11, 12)
+    GP_CE(13, 14)
+#undef GP_CE
 }
 
 // ascending bitonic network on N registers (flip formulation: all comparators ascending)
@@ -360,87 +364,175 @@ __device__ __forceinline__ int32_t warp_runmerge64(const unsigned long long (&v)
 }
 
 // ---------------------------------------------------------------------------------------
-// C1: leftover + cmap + cvwgt + ub prefix + tile starts
+// block-wide helpers (all threads call)
 // ---------------------------------------------------------------------------------------
-// Tiles are assigned statically (tile = blockIdx + i*gridDim): every CTA of a cooperative
-// launch is resident, and a tile only waits on lower tiles, which their CTAs reach first.
-__device__ void phase_c1(const ContractArgs &a, ContractSmem &sm, int32_t n, int32_t ntiles2) {
-    const int ntiles = (n + kCTileV - 1) / kCTileV;
-    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        const long long base = (long long)tile * kCTileV + (long long)threadIdx.x * kCItems;
-        int32_t m[kCItems];
-        int32_t d[kCItems];
+__device__ __forceinline__ void block_sum2(ContractSmem &sm, int32_t &x, int32_t &y) {
+    const int l = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int32_t a = warp_sum(x), b = warp_sum(y);
+    if (l == 0) {
+        sm.red[0][w] = a;
+        sm.red[1][w] = b;
+    }
+    __syncthreads();
+    a = 0;
+    b = 0;
+#pragma unroll
+    for (int q = 0; q < kCW; ++q) {
+        a += sm.red[0][q];
+        b += sm.red[1][q];
+    }
+    __syncthreads();
+    x = a;
+    y = b;
+}
+
+// exclusive scan of vals[k*stride + comp] for k in [0, cnt) into out[k] (shared), plus base;
+// returns the sum of the list
+__device__ __forceinline__ int32_t block_scan_list(ContractSmem &sm, const int32_t *vals, int stride, int comp,
+                                                   int cnt, int32_t base, int32_t *out) {
+    const int per = (cnt + kCNT - 1) / kCNT;
+    const int lo = min(cnt, (int)threadIdx.x * per), hi = min(cnt, lo + per);
+    int32_t s = 0;
+    for (int k = lo; k < hi; ++k) s += __ldcg(vals + (size_t)k * stride + comp);
+    int32_t tot;
+    int32_t run = base + block_excl_scan<kCNT>(s, sm.scan, tot);
+    for (int k = lo; k < hi; ++k) {
+        out[k] = run;
+        run += __ldcg(vals + (size_t)k * stride + comp);
+    }
+    __syncthreads();
+    return tot;
+}
+
+__device__ __forceinline__ int32_t warp_excl(int32_t v, int32_t &total) {
+    const int32_t inc = warp_incl_scan(v);
+    total = __shfl_sync(0xffffffffu, inc, 31);
+    return inc - v;
+}
+
+// ---------------------------------------------------------------------------------------
+// C1a: leftover + leader flags + warp-tile aggregates (+ chunk sums of C1b's owners)
+// ---------------------------------------------------------------------------------------
+__device__ void phase_c1a(const ContractArgs &a, int32_t n, int nt1, int T1) {
+    const int lane = threadIdx.x & 31;
+    const int gw = blockIdx.x * kCW + (threadIdx.x >> 5), nw = gridDim.x * kCW;
+    for (int wt = gw; wt < nt1; wt += nw) {
+        const long long base = (long long)wt * kVW;
         int32_t cnt = 0, ubs = 0;
 #pragma unroll
         for (int i = 0; i < kCItems; ++i) {
-            const long long u = base + i;
-            m[i] = -2;
-            d[i] = 0;
+            const long long u = base + i * 32 + lane;  // coalesced
             if (u < n) {
-                m[i] = a.M[u];
-                if (m[i] == kFree && a.apply_leftover) {
-                    m[i] = (int32_t)u;  // leftover: matched to itself (P18.s12-13)
-                    a.M[u] = (int32_t)u;
+                int32_t m = a.M[u];
+                if (m == kFree && a.apply_leftover) {
+                    m = (int32_t)u;  // leftover: matched to itself (P18.s12-13)
+                    a.M[u] = m;
                 }
-                if (u <= m[i]) {  // leader flag (P18.s18, R7)
+                if (u <= m) {  // leader flag (P18.s18, R7)
                     ++cnt;
-                    d[i] = __ldg(a.adjp + u + 1) - __ldg(a.adjp + u);
-                    if (m[i] != u) d[i] += __ldg(a.adjp + m[i] + 1) - __ldg(a.adjp + m[i]);  // P20.s6-8
-                    ubs += d[i];
+                    ubs += __ldg(a.adjp + u + 1) - __ldg(a.adjp + u);
+                    if (m != u) ubs += __ldg(a.adjp + m + 1) - __ldg(a.adjp + m);  // P20.s6-8
                 }
             }
         }
-        int32_t tc, tu;
-        const int32_t ec = block_excl_scan<kCNT>(cnt, sm.scan, tc);
-        const int32_t eu = block_excl_scan<kCNT>(ubs, sm.scan, tu);
-        if (threadIdx.x < 32) {
-            const int32_t agg[2] = {tc, tu};
-            int32_t pre[2];
-            lookback<2>(a.st1, a.epoch, tile, agg, pre);
-            if (threadIdx.x == 0) {
-                sm.prefix = pre[0];
-                sm.prefix2 = (unsigned long long)(uint32_t)pre[1];
-            }
+        cnt = warp_sum(cnt);
+        ubs = warp_sum(ubs);
+        if (lane == 0) {
+            a.tagg1[2 * wt] = cnt;
+            a.tagg1[2 * wt + 1] = ubs;
+            atomicAdd(&a.ctl->chunk1[2 * (wt / T1)], cnt);
+            atomicAdd(&a.ctl->chunk1[2 * (wt / T1) + 1], ubs);
         }
-        __syncthreads();
-        int32_t c = sm.prefix + ec;
-        int32_t o = (int32_t)sm.prefix2 + eu;
-        if (tile == 0 && threadIdx.x == 0) a.tile_start[0] = 0;
-        if (tile == ntiles - 1 && threadIdx.x == 0) {
-            const int32_t nc = sm.prefix + tc;
-            a.ctl->n_coarse = nc;
-            a.off[nc] = (int32_t)sm.prefix2 + tu;  // = nnz
-            a.tile_start[ntiles2] = nc;
-        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------
+// C1b: CM, cvwgt, off, seg, C2 warp-tile starts, huge rows
+// ---------------------------------------------------------------------------------------
+__device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, int nt1, int T1, int32_t ntiles2) {
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int t_lo = blockIdx.x * T1, t_hi = min(nt1, t_lo + T1);
+    if (t_lo >= t_hi) return;
+    int32_t pc = 0, pu = 0;
+    for (int b = threadIdx.x; b < (int)blockIdx.x; b += kCNT) {
+        pc += __ldcg(a.ctl->chunk1 + 2 * b);
+        pu += __ldcg(a.ctl->chunk1 + 2 * b + 1);
+    }
+    block_sum2(sm, pc, pu);
+    int32_t *tpc = reinterpret_cast<int32_t *>(sm.buf);  // segments of <= kBuf tiles per value
+    int32_t *tpu = tpc + kBuf;
+    for (int s_lo = t_lo; s_lo < t_hi; s_lo += kBuf) {
+    const int s_hi = min(t_hi, s_lo + kBuf);
+    pc += block_scan_list(sm, a.tagg1 + 2 * s_lo, 2, 0, s_hi - s_lo, pc, tpc);
+    pu += block_scan_list(sm, a.tagg1 + 2 * s_lo, 2, 1, s_hi - s_lo, pu, tpu);
+    for (int t = s_lo + wib; t < s_hi; t += kCW) {
+        // lane owns the contiguous vertices base + lane*8 .. +7 (scan order)
+        const long long base = (long long)t * kVW + (long long)lane * kCItems;
+        int32_t m[kCItems], d[kCItems];
+        int32_t cnt = 0, ubs = 0;
+        // counts: M first, then the degrees of leader and partner (loads hoisted per level)
+#pragma unroll
+        for (int i = 0; i < kCItems; ++i) m[i] = (base + i < n) ? __ldcg(a.M + base + i) : -2;
 #pragma unroll
         for (int i = 0; i < kCItems; ++i) {
             const long long u = base + i;
+            const bool lead = u < n && u <= m[i];
+            const bool pair = u < n && u < m[i];
+            const int32_t v = pair ? m[i] : 0;
+            const int32_t a0 = lead ? __ldg(a.adjp + u) : 0, a1 = lead ? __ldg(a.adjp + u + 1) : 0;
+            const int32_t b0 = pair ? __ldg(a.adjp + v) : 0, b1 = pair ? __ldg(a.adjp + v + 1) : 0;
+            d[i] = (a1 - a0) + (b1 - b0);  // P20.s6-8
+            cnt += lead;
+            ubs += d[i];
+        }
+        int32_t tc, tu;
+        int32_t c = tpc[t - s_lo] + warp_excl(cnt, tc);
+        int32_t o = tpu[t - s_lo] + warp_excl(ubs, tu);
+        if (t == 0 && lane == 0) a.tile_start[0] = 0;
+        if (t == nt1 - 1 && lane == 0) {
+            const int32_t nc = tpc[t - s_lo] + tc;
+            a.ctl->n_coarse = nc;
+            a.off[nc] = tpu[t - s_lo] + tu;  // = nnz
+            a.tile_start[ntiles2] = nc;
+        }
+        // stores in two halves; each half gathers everything it needs before any store
+#pragma unroll
+        for (int h = 0; h < kCItems; h += kCItems / 2) {
+            int32_t su[kCItems / 2], ep[kCItems / 2], sv[kCItems / 2], vw[kCItems / 2];
+#pragma unroll
+            for (int q = 0; q < kCItems / 2; ++q) {
+                const int i = h + q;
+                const long long u = base + i;
+                const bool lead = u < n && u <= m[i];
+                const bool pair = u < n && u < m[i];
+                su[q] = lead ? __ldg(a.adjp + u) : 0;
+                ep[q] = lead ? __ldg(a.adjp + u + 1) : 0;
+                sv[q] = pair ? __ldg(a.adjp + m[i]) : 0;
+                vw[q] = (lead ? __ldg(a.vwgt + u) : 0) + (pair ? __ldg(a.vwgt + m[i]) : 0);  // P12.s27
+            }
+#pragma unroll
+        for (int q = 0; q < kCItems / 2; ++q) {
+            const int i = h + q;
+            const long long u = base + i;
             if (u < n && u <= m[i]) {
                 const int32_t v = m[i];
-                a.CM[u] = c;                      // exclusive scan = inclusive - 1 (P18.s20-24)
-                a.leaders[c] = (int32_t)u;
-                int32_t vw = __ldg(a.vwgt + u);
-                if (v != u) {
-                    a.CM[v] = c;                  // partner copies its leader's id (P18.s26)
-                    vw += __ldg(a.vwgt + v);      // w(c) = w(u) + w(v) (P12.s27)
-                }
-                a.cvwgt[c] = vw;
+                const int32_t dl = ep[q] - su[q];
+                a.CM[u] = c;              // exclusive scan = inclusive - 1 (P18.s20-24)
+                if (v != u) a.CM[v] = c;  // partner copies its leader's id (P18.s26)
+                a.cvwgt[c] = vw[q];
                 a.off[c] = o;
-                {
-                    const int32_t su = __ldg(a.adjp + u);
-                    const int32_t du = __ldg(a.adjp + u + 1) - su;
-                    a.seg[c] = make_int4(su, du, v != u ? __ldg(a.adjp + v) : 0, d[i] - du);
-                }
-                // tile t starts at the first row with off >= t*kTileArcs: row c+1 for every t
-                // with off[c] < t*kTileArcs <= off[c+1]
-                for (int32_t t = o / kTileArcs + 1; t <= (o + d[i]) / kTileArcs && t < ntiles2; ++t)
-                    a.tile_start[t] = c + 1;
-                if (d[i] > kTileArcs) a.huge[atomicAdd(&a.ctl->n_huge, 1)] = c;
+                a.seg[c] = make_int4(su[q], dl, sv[q], d[i] - dl);
+                // warp tile t2 starts at the first row with off >= t2*kWB: row c+1 for
+                // every t2 with off[c] < t2*kWB <= off[c+1]
+                for (int32_t t2 = o / kWB + 1; t2 <= (o + d[i]) / kWB && t2 < ntiles2; ++t2) a.tile_start[t2] = c + 1;
+                if (d[i] > kWB) a.huge[atomicAdd(&a.ctl->n_huge, 1)] = c;
                 ++c;
                 o += d[i];
             }
         }
-        __syncthreads();
+        }
+    }
+    __syncthreads();  // the prefix arrays are rewritten by the next segment
     }
 }
 
@@ -454,17 +546,22 @@ __device__ __forceinline__ void gather_row(const ContractArgs &a, int32_t c, int
     for (int side = 0; side < 2; ++side) {
         const int32_t s = side ? sg.z : sg.x, e = s + (side ? sg.w : sg.y);
         for (int32_t j = s + tid; j < e; j += nthr) {
-            const int32_t cx = __ldcg(a.CM + __ldg(a.adjncy + j));
-            if (cx != c) dst[claim()] = ckey(cx, __ldg(a.adjwgt + j));  // drop the collapsed edge (R9)
+            const int32_t cx = __ldcg(a.CM + __ldcs(a.adjncy + j));
+            if (cx != c) dst[claim()] = ckey(cx, __ldcs(a.adjwgt + j));  // drop the collapsed edge (R9)
         }
     }
 }
 
-// C1b: rows whose upper bound exceeds a tile: one CTA per row in global scratch
-__device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
+// ---------------------------------------------------------------------------------------
+// C1h: rows with ub > kWB, one CTA each; result compacted at gkeys[off[c]], count cnt[c]
+// ---------------------------------------------------------------------------------------
+__device__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
     for (int i = blockIdx.x; i < nh; i += gridDim.x) {
         const int32_t c = a.huge[i];
-        unsigned long long *keys = a.gkeys + __ldcg(a.off + c);
+        const int32_t o0 = __ldcg(a.off + c);
+        const int32_t ub = __ldcg(a.off + c + 1) - o0;
+        unsigned long long *dst = a.gkeys + o0;
+        unsigned long long *keys = (ub <= kCtaRow) ? sm.buf : dst;
         if (threadIdx.x == 0) sm.len = 0;
         __syncthreads();
         gather_row(a, c, threadIdx.x, kCNT, keys, [&]() { return atomicAdd(&sm.len, 1); });
@@ -475,100 +572,146 @@ __device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
             keys, len, threadIdx.x, kCNT, sm.lead, sm.has,
             [&](int32_t v, int32_t &tot) { return block_excl_scan<kCNT>(v, sm.scan, tot); },
             []() { __syncthreads(); });
-        if (threadIdx.x == 0) {
-            a.cnt[c] = cnt;
-            a.rlen[c] = len;
+        // compact the run heads into dst (in place when keys == dst: a chunk's writes land
+        // below its reads, and every read of a chunk precedes its writes)
+        int32_t wr = 0;
+        for (int32_t b0 = 0; b0 < len; b0 += kCNT) {
+            const int32_t j = b0 + threadIdx.x;
+            const unsigned long long kv = j < len ? keys[j] : 0ull;
+            const bool h = j < len && is_head(keys, j);
+            int32_t tot;
+            const int32_t ex = block_excl_scan<kCNT>(h ? 1 : 0, sm.scan, tot);
+            if (h) dst[wr + ex] = kv;
+            wr += tot;
+            __syncthreads();
         }
+        if (threadIdx.x == 0) a.cnt[c] = cnt;
         __syncthreads();
     }
 }
 
 // ---------------------------------------------------------------------------------------
-// C2: tiled merge + assembly
+// C2a: warp tiles: merge every row, write the tile compacted to tout at its ub offset
 // ---------------------------------------------------------------------------------------
-__device__ void phase_c2(const ContractArgs &a, ContractSmem &sm, int32_t nc, int32_t nnz, int32_t ntiles2) {
+__device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntiles2, int T2) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    for (int tile = blockIdx.x; tile < ntiles2; tile += gridDim.x) {
-        const int32_t r0 = __ldcg(a.tile_start + tile), r1 = __ldcg(a.tile_start + tile + 1);
-        const int32_t tbase = tile * kTileArcs;
-        const bool single = (r1 - r0) <= kCNT;  // one row per thread: keep pass-1 state in registers
-        int32_t k_cnt = 0, k_slot = 0, k_ub = 0, k_ex = 0;
-        // ---- pass 1: merge every row of the tile into its shared-memory slot, count ----
-        int32_t total = 0;
-        for (int32_t g0 = r0; g0 < r1; g0 += kCNT) {
-            const int32_t c = g0 + threadIdx.x;
-            int32_t ub = 0, slot = 0, cntc = 0;
-            bool warp_row = false;
+    const int gw = blockIdx.x * kCW + wib, nw = gridDim.x * kCW;
+    unsigned long long *wb = sm.buf + wib * 2 * kWB;  // this warp's slots (2*kWB entries)
+    for (int wt = gw; wt < ntiles2; wt += nw) {
+        int32_t r0 = 0, r1 = 0;
+        if (lane < 2) {
+            const int32_t x = __ldcg(a.tile_start + wt + lane);
+            r0 = x;
+        }
+        r1 = __shfl_sync(0xffffffffu, r0, 1);
+        r0 = __shfl_sync(0xffffffffu, r0, 0);
+        const int32_t tbase = wt * kWB;
+        unsigned long long *out = a.tout + (r0 < r1 ? __ldcg(a.off + r0) : 0);
+        int32_t run = 0;
+        for (int32_t g0 = r0; g0 < r1; g0 += 32) {
+            const int32_t c = g0 + lane;
+            int32_t ub = 0, slot = 0x7fffffff, cntc = 0;
+            int4 sg = make_int4(0, 0, 0, 0);
             if (c < r1) {
                 const int32_t o0 = __ldcg(a.off + c);
                 slot = o0 - tbase;
                 ub = __ldcg(a.off + c + 1) - o0;
-                if (ub > kTileArcs) {
-                    cntc = __ldcg(a.cnt + c);  // merged by C1b
-                } else if (ub > kNet) {
-                    warp_row = true;
-                } else if (ub > 0) {
-                    const int4 sg = __ldcg(a.seg + c);
-                    const int32_t su = sg.x, du = sg.y, sv = sg.z;
-                    unsigned long long k[kNet];
-#pragma unroll
-                    for (int i = 0; i < kNet; ++i) {
-                        k[i] = kMaxKey;
-                        if (i < ub) {
-                            const int32_t j = (i < du) ? su + i : sv + (i - du);
-                            const int32_t cx = __ldcg(a.CM + __ldg(a.adjncy + j));
-                            if (cx != c) k[i] = ckey(cx, __ldg(a.adjwgt + j));
-                        }
-                    }
-                    reg_sort<kNet>(k);
-                    int32_t prev = -1, acc = 0;
-#pragma unroll
-                    for (int i = 0; i < kNet; ++i) {
-                        if (k[i] != kMaxKey) {
-                            const int32_t cx = (int32_t)(k[i] >> 32), w = (int32_t)(uint32_t)k[i];
-                            if (cx == prev) {
-                                acc += w;  // repeated coarse neighbour: weights summed (R8, P12.s28)
-                            } else {
-                                if (prev >= 0) sm.buf[slot + cntc++] = ckey(prev, acc);
-                                prev = cx;
-                                acc = w;
-                            }
-                        }
-                    }
-                    if (prev >= 0) sm.buf[slot + cntc++] = ckey(prev, acc);
-                }
+                if (ub <= kWarpNet) sg = __ldcg(a.seg + c);
+                if (ub > kWB) cntc = __ldcg(a.cnt + c);  // merged by C1h
             }
-            // rows of 17..64 entries: one warp each, registers + shuffles
-            unsigned m64 = __ballot_sync(0xffffffffu, warp_row && ub <= kWarpNet);
+            // ---- stage the arcs of every row with ub <= 64 into its slot, coalesced: lane
+            // e of a step owns flat index idx; its row is the last lane with slot <= idx ----
+            {
+                const int32_t lo = __shfl_sync(0xffffffffu, slot, 0);
+                int32_t hi = (c < r1 && ub <= kWarpNet) ? slot + ub : 0;  // staged rows only
+#pragma unroll
+                for (int off = 16; off > 0; off >>= 1) hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, off));
+                constexpr int kB = 8;  // steps per batch: all loads of a batch are in flight together
+                for (int32_t b0 = lo; b0 < hi; b0 += 32 * kB) {
+                    int32_t jj[kB], rc[kB], x[kB], w[kB], cx[kB];
+#pragma unroll
+                    for (int k = 0; k < kB; ++k) {
+                        const int32_t idx = b0 + k * 32 + lane;
+                        int r = 0;
+#pragma unroll
+                        for (int step = 16; step > 0; step >>= 1) {
+                            const int32_t sl = __shfl_sync(0xffffffffu, slot, r + step);
+                            if (sl <= idx) r += step;
+                        }
+                        const int32_t rs = __shfl_sync(0xffffffffu, slot, r);
+                        const int32_t rub = __shfl_sync(0xffffffffu, ub, r);
+                        const int32_t rsu = __shfl_sync(0xffffffffu, sg.x, r);
+                        const int32_t rdu = __shfl_sync(0xffffffffu, sg.y, r);
+                        const int32_t rsv = __shfl_sync(0xffffffffu, sg.z, r);
+                        const int32_t p = idx - rs;
+                        rc[k] = g0 + r;
+                        jj[k] = (idx < hi && p < rub && rub <= kWarpNet) ? ((p < rdu) ? rsu + p : rsv + (p - rdu)) : -1;
+                    }
+#pragma unroll
+                    for (int k = 0; k < kB; ++k) {
+                        x[k] = jj[k] >= 0 ? __ldcs(a.adjncy + jj[k]) : 0;
+                        w[k] = jj[k] >= 0 ? __ldcs(a.adjwgt + jj[k]) : 0;
+                    }
+#pragma unroll
+                    for (int k = 0; k < kB; ++k) cx[k] = jj[k] >= 0 ? __ldcg(a.CM + x[k]) : 0;
+#pragma unroll
+                    for (int k = 0; k < kB; ++k)
+                        if (jj[k] >= 0)  // collapsed edge dropped (R9)
+                            wb[b0 + k * 32 + lane] = (cx[k] != rc[k]) ? ckey(cx[k], w[k]) : kMaxKey;
+                }
+                __syncwarp();
+            }
+            if (c < r1 && ub > 0 && ub <= kNet) {
+                uint32_t kc[kNet];
+                int32_t kw[kNet];
+#pragma unroll
+                for (int i = 0; i < kNet; ++i) {
+                    const unsigned long long kv = (i < ub) ? wb[slot + i] : kMaxKey;
+                    kc[i] = (uint32_t)(kv >> 32);
+                    kw[i] = (int32_t)(uint32_t)kv;
+                }
+                cx_sort16(kc, kw);
+                uint32_t prev = 0xFFFFFFFFu;
+                int32_t acc = 0;
+#pragma unroll
+                for (int i = 0; i < kNet; ++i) {
+                    if (kc[i] == prev) {
+                        acc += kw[i];  // repeated coarse neighbour: weights summed (R8, P12.s28)
+                    } else {
+                        if (prev != 0xFFFFFFFFu) wb[slot + cntc++] = ckey((int32_t)prev, acc);
+                        prev = kc[i];
+                        acc = kw[i];
+                    }
+                }
+                if (prev != 0xFFFFFFFFu) wb[slot + cntc++] = ckey((int32_t)prev, acc);
+            }
+            // rows of 17..64 entries: the warp, registers + shuffles, keys from the slot
+            unsigned m64 = __ballot_sync(0xffffffffu, c < r1 && ub > kNet && ub <= kWarpNet);
             while (m64) {
                 const int src = __ffs(m64) - 1;
                 m64 &= m64 - 1;
-                const int32_t cw = __shfl_sync(0xffffffffu, c, src);
                 const int32_t sl = __shfl_sync(0xffffffffu, slot, src);
-                const int4 sg = __ldcg(a.seg + cw);
+                const int32_t rub = __shfl_sync(0xffffffffu, ub, src);
                 unsigned long long v[2];
 #pragma unroll
                 for (int r = 0; r < 2; ++r) {
                     const int32_t e = r * 32 + lane;
-                    v[r] = kMaxKey;
-                    if (e < sg.y + sg.w) {
-                        const int32_t j = (e < sg.y) ? sg.x + e : sg.z + (e - sg.y);
-                        const int32_t cx = __ldcg(a.CM + __ldg(a.adjncy + j));
-                        if (cx != cw) v[r] = ckey(cx, __ldg(a.adjwgt + j));  // collapsed edge dropped (R9)
-                    }
+                    v[r] = (e < rub) ? wb[sl + e] : kMaxKey;
                 }
+                __syncwarp();
                 warp_sort64(v);
-                const int32_t cc = warp_runmerge64(v, sm.buf + sl);  // compacted in the slot
+                const int32_t cc = warp_runmerge64(v, wb + sl);  // compacted in the slot
+                __syncwarp();
                 if (lane == src) cntc = cc;
             }
-            // rows of 65..kTileArcs entries: one warp each, shared-memory sort in their slot
-            unsigned mm = __ballot_sync(0xffffffffu, warp_row && ub > kWarpNet);
+            // rows of 65..kWB entries: the warp, shared-memory sort in the slot, compacted
+            unsigned mm = __ballot_sync(0xffffffffu, c < r1 && ub > kWarpNet && ub <= kWB);
             while (mm) {
                 const int src = __ffs(mm) - 1;
                 mm &= mm - 1;
                 const int32_t cw = __shfl_sync(0xffffffffu, c, src);
                 const int32_t sl = __shfl_sync(0xffffffffu, slot, src);
-                unsigned long long *keys = sm.buf + sl;
+                unsigned long long *keys = wb + sl;
                 if (lane == 0) sm.wlen[wib] = 0;
                 __syncwarp();
                 gather_row(a, cw, lane, 32, keys, [&]() { return atomicAdd(&sm.wlen[wib], 1); });
@@ -577,127 +720,103 @@ __device__ void phase_c2(const ContractArgs &a, ContractSmem &sm, int32_t nc, in
                 coop_sort(keys, len, lane, 32, []() { __syncwarp(); });
                 const int32_t cc = coop_runsum(
                     keys, len, lane, 32, sm.lead + wib * 32, sm.has + wib * 32,
-                    [&](int32_t v, int32_t &tot) {
-                        const int32_t inc = warp_incl_scan(v);
-                        tot = __shfl_sync(0xffffffffu, inc, 31);
-                        return inc - v;
-                    },
-                    []() { __syncwarp(); });
-                if (lane == src) {
-                    cntc = cc;
-                    a.rlen[cw] = len;
-                }
-            }
-            int32_t part;
-            const int32_t ex = block_excl_scan<kCNT>(cntc, sm.scan, part);
-            if (single) {
-                k_cnt = cntc;
-                k_slot = slot;
-                k_ub = ub;
-                k_ex = ex;
-            } else if (c < r1) {
-                a.cnt[c] = cntc;
-            }
-            total += part;
-        }
-        // ---- tile prefix by decoupled look-back ----
-        if (threadIdx.x < 32) {
-            const int32_t agg[1] = {total};
-            int32_t pre[1];
-            lookback<1>(a.st2, a.epoch, tile, agg, pre);
-            if (threadIdx.x == 0) sm.prefix = pre[0];
-        }
-        __syncthreads();
-        int32_t pos0 = sm.prefix;
-        if (tile == ntiles2 - 1 && threadIdx.x == 0) {
-            a.cadjp[nc] = pos0 + total;
-            a.ctl->cnnz = pos0 + total;
-        }
-        // ---- pass 2: cadjp and the rows, straight into the final arrays ----
-        for (int32_t g0 = r0; g0 < r1; g0 += kCNT) {
-            const int32_t c = g0 + threadIdx.x;
-            int32_t cntc = 0, ub = 0, slot = 0, o = 0, part = 0;
-            if (single) {
-                cntc = k_cnt;
-                slot = k_slot;
-                ub = k_ub;
-                o = pos0 + k_ex;
-                part = total;
-            } else {
-                if (c < r1) {
-                    cntc = __ldcg(a.cnt + c);
-                    slot = __ldcg(a.off + c) - tbase;
-                    ub = __ldcg(a.off + c + 1) - __ldcg(a.off + c);
-                }
-                const int32_t ex = block_excl_scan<kCNT>(cntc, sm.scan, part);
-                o = pos0 + ex;
-            }
-            if (c < r1) {
-                a.cadjp[c] = o;
-                if (ub <= kWarpNet) {
-                    for (int32_t j = 0; j < cntc; ++j) {
-                        const unsigned long long k = sm.buf[slot + j];
-                        a.cadjncy[o + j] = (int32_t)(k >> 32);
-                        a.cadjwgt[o + j] = (int32_t)(uint32_t)k;
-                    }
-                }
-            }
-            // rows sorted in shared memory by a warp: the warp writes the run heads
-            unsigned mw = __ballot_sync(0xffffffffu, c < r1 && ub > kWarpNet && ub <= kTileArcs);
-            while (mw) {
-                const int src = __ffs(mw) - 1;
-                mw &= mw - 1;
-                const int32_t cw = __shfl_sync(0xffffffffu, c, src);
-                const int32_t sl = __shfl_sync(0xffffffffu, slot, src);
-                const int32_t ow = __shfl_sync(0xffffffffu, o, src);
-                const unsigned long long *keys = sm.buf + sl;
-                const int32_t len = __ldcg(a.rlen + cw);
-                int32_t run = 0;
+                    [&](int32_t v, int32_t &tot) { return warp_excl(v, tot); }, []() { __syncwarp(); });
+                int32_t wr = 0;
                 for (int32_t b0 = 0; b0 < len; b0 += 32) {
                     const int32_t i = b0 + lane;
+                    const unsigned long long kv = i < len ? keys[i] : 0ull;
                     const bool h = i < len && is_head(keys, i);
                     const unsigned hm = __ballot_sync(0xffffffffu, h);
-                    if (h) {
-                        const int32_t pos = ow + run + __popc(hm & lanemask_lt());
-                        a.cadjncy[pos] = (int32_t)(keys[i] >> 32);
-                        a.cadjwgt[pos] = (int32_t)(uint32_t)keys[i];
-                    }
-                    run += __popc(hm);
+                    __syncwarp();
+                    if (h) keys[wr + __popc(hm & lanemask_lt())] = kv;
+                    wr += __popc(hm);
+                    __syncwarp();
                 }
+                if (lane == src) cntc = cc;
             }
-            // a row merged by C1b (at most one per tile, its last row): copied by the CTA
-            const int hub_here = __syncthreads_or(c < r1 && ub > kTileArcs);
-            if (hub_here) {
-                if (c < r1 && ub > kTileArcs) {
-                    sm.hub_c = c;
-                    sm.hub_o = o;
-                }
-                __syncthreads();
-                const int32_t hc = sm.hub_c, oc = sm.hub_o;
-                const unsigned long long *src = a.gkeys + __ldcg(a.off + hc);
-                const int32_t len = __ldcg(a.rlen + hc);
-                int32_t run = 0;
-                for (int32_t b0 = 0; b0 < len; b0 += kCNT) {
-                    const int32_t i = b0 + threadIdx.x;
-                    const bool h = i < len && is_head(src, i);
-                    int32_t tot;
-                    const int32_t ex = block_excl_scan<kCNT>(h ? 1 : 0, sm.scan, tot);
-                    if (h) {
-                        a.cadjncy[oc + run + ex] = (int32_t)(src[i] >> 32);
-                        a.cadjwgt[oc + run + ex] = (int32_t)(uint32_t)src[i];
-                    }
-                    run += tot;
-                }
+            int32_t part;
+            const int32_t ex = warp_excl(cntc, part);
+            if (c < r1) {
+                a.lofs[c] = run + ex;
+                if (ub <= kWB)
+                    for (int32_t j = 0; j < cntc; ++j) __stcs(out + run + ex + j, wb[slot + j]);
             }
-            pos0 += part;
+            // rows merged by C1h: the warp copies them in
+            unsigned mh = __ballot_sync(0xffffffffu, c < r1 && ub > kWB);
+            while (mh) {
+                const int src = __ffs(mh) - 1;
+                mh &= mh - 1;
+                const int32_t cw = __shfl_sync(0xffffffffu, c, src);
+                const int32_t k = __shfl_sync(0xffffffffu, cntc, src);
+                const int32_t pos = run + __shfl_sync(0xffffffffu, ex, src);
+                const unsigned long long *src_keys = a.gkeys + __ldcg(a.off + cw);
+                for (int32_t j = lane; j < k; j += 32) out[pos + j] = __ldcg(src_keys + j);
+            }
+            __syncwarp();
+            run += part;
         }
-        __syncthreads();  // the slots are reused by the next tile
+        if (lane == 0) {
+            a.ttot[wt] = run;
+            atomicAdd(&a.ctl->chunk2[wt / T2], run);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------
+// C2b: cadjp + coalesced copy of the tiles of this CTA's chunk into the final CSR
+// ---------------------------------------------------------------------------------------
+__device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, int32_t ntiles2, int T2) {
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int t_lo = blockIdx.x * T2, t_hi = min(ntiles2, t_lo + T2);
+    if (t_lo >= t_hi) return;
+    int32_t pre = 0, dummy = 0;
+    for (int b = threadIdx.x; b < (int)blockIdx.x; b += kCNT) pre += __ldcg(a.ctl->chunk2 + b);
+    block_sum2(sm, pre, dummy);
+    int32_t *tp = reinterpret_cast<int32_t *>(sm.buf);
+    constexpr int kCap = 2 * kBuf;
+    for (int s_lo = t_lo; s_lo < t_hi; s_lo += kCap) {
+    const int s_hi = min(t_hi, s_lo + kCap);
+    pre += block_scan_list(sm, a.ttot + s_lo, 1, 0, s_hi - s_lo, pre, tp);
+    for (int t = s_lo + wib; t < s_hi; t += kCW) {
+        const int32_t p = tp[t - s_lo];
+        int32_t r0 = 0, r1 = 0;
+        if (lane < 2) r0 = __ldcg(a.tile_start + t + lane);
+        r1 = __shfl_sync(0xffffffffu, r0, 1);
+        r0 = __shfl_sync(0xffffffffu, r0, 0);
+        const int32_t total = __ldcg(a.ttot + t);
+        for (int32_t c = r0 + lane; c < r1; c += 32) a.cadjp[c] = p + __ldcg(a.lofs + c);
+        if (r0 < r1) {
+            const unsigned long long *src = a.tout + __ldcg(a.off + r0);
+            constexpr int kB = 8;
+            for (int32_t j0 = 0; j0 < total; j0 += 32 * kB) {
+                unsigned long long k[kB];
+#pragma unroll
+                for (int q = 0; q < kB; ++q) {
+                    const int32_t j = j0 + q * 32 + lane;
+                    k[q] = j < total ? __ldcs(src + j) : 0ull;
+                }
+#pragma unroll
+                for (int q = 0; q < kB; ++q) {
+                    const int32_t j = j0 + q * 32 + lane;
+                    if (j < total) {
+                        a.cadjncy[p + j] = (int32_t)(k[q] >> 32);
+                        a.cadjwgt[p + j] = (int32_t)(uint32_t)k[q];
+                    }
+                }
+            }
+        }
+        if (t == ntiles2 - 1 && lane == 0) {
+            a.cadjp[nc] = p + total;
+            a.ctl->cnnz = p + total;
+        }
+    }
+    __syncthreads();
     }
 }
 
 __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constant__ ContractArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    ContractSmem &sm = *reinterpret_cast<ContractSmem *>(smem_raw);
+    ContractSmem &sm = *reinterpret_cast<ContractSmem *>(((uintptr_t)smem_raw + 127) & ~(uintptr_t)127);
     ContractCtl *ctl = a.ctl;
     const volatile SizeRec *in = a.in;
     if (in->stop) {  // an earlier level ended the coarsening: propagate and leave
@@ -716,35 +835,47 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
     }
     const int32_t n = in->n;
     const int32_t nnz = in->nnz;
-    const int32_t ntiles2 = nnz > 0 ? (nnz + kTileArcs - 1) / kTileArcs : 0;
+    unsigned bar_epoch = 0;  // grid barriers passed (thread 0)
+    const int nt1 = (n + kVW - 1) / kVW;
+    const int T1 = (nt1 + gridDim.x - 1) / gridDim.x;            // C1b tiles per CTA
+    const int32_t ntiles2 = nnz > 0 ? (nnz + kWB - 1) / kWB : 0;
+    const int T2 = (ntiles2 + gridDim.x - 1) / gridDim.x;        // C2b tiles per CTA
     trace_mark(ctl->trace, 0);
     if (n > 0) {
-        phase_c1(a, sm, n, ntiles2);
+        phase_c1a(a, n, nt1, T1);
         trace_mark(ctl->trace, 1);
-        grid_barrier(ctl->bar);
+        grid_barrier(ctl->bar, bar_epoch);
+        trace_mark(ctl->trace, 2);
+        phase_c1b(a, sm, n, nt1, T1, ntiles2);
+        trace_mark(ctl->trace, 3);
+        grid_barrier(ctl->bar, bar_epoch);
     }
-    trace_mark(ctl->trace, 2);
+    trace_mark(ctl->trace, 4);
     const int32_t nc = *(volatile int32_t *)&ctl->n_coarse;
     const int32_t nh = *(volatile int32_t *)&ctl->n_huge;
     if (nh > 0) {
-        phase_c1b(a, sm, nh);
-        grid_barrier(ctl->bar);
+        phase_c1h(a, sm, nh);
+        grid_barrier(ctl->bar, bar_epoch);
     }
-    trace_mark(ctl->trace, 3);
-    if (ntiles2 > 0) phase_c2(a, sm, nc, nnz, ntiles2);
-    trace_mark(ctl->trace, 4);
-    if (ntiles2 == 0) {  // no arcs: every coarse row is empty
+    trace_mark(ctl->trace, 5);
+    if (ntiles2 > 0) {
+        phase_c2a(a, sm, ntiles2, T2);
+        trace_mark(ctl->trace, 6);
+        grid_barrier(ctl->bar, bar_epoch);
+        trace_mark(ctl->trace, 7);
+        phase_c2b(a, sm, nc, ntiles2, T2);
+    } else {  // no arcs: every coarse row is empty
         for (long long c = (long long)blockIdx.x * kCNT + threadIdx.x; c <= nc; c += (long long)gridDim.x * kCNT)
             a.cadjp[c] = 0;
         if (blockIdx.x == 0 && threadIdx.x == 0) ctl->cnnz = 0;
     }
+    trace_mark(ctl->trace, 8);
     // the last CTA to finish publishes the coarse sizes and the stop decision
-    __shared__ bool last;
     __threadfence();
     __syncthreads();
-    if (threadIdx.x == 0) last = atomicAdd(&ctl->blocks_done, 1u) == gridDim.x - 1;
+    if (threadIdx.x == 0) sm.last = atomicAdd(&ctl->blocks_done, 1u) == gridDim.x - 1;
     __syncthreads();
-    if (last && threadIdx.x == 0) {
+    if (sm.last && threadIdx.x == 0) {
         __threadfence();
         const int32_t ncv = *((volatile int32_t *)&ctl->n_coarse);
         const int32_t cnnz = *((volatile int32_t *)&ctl->cnnz);
@@ -778,20 +909,17 @@ int contract_grid(Ctx *ctx) {
     if (per_sm < 0) {
         int b = 0;
         cudaFuncSetAttribute(k_contract_level, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)sizeof(ContractSmem));
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_contract_level, kCNT, sizeof(ContractSmem));
+                             (int)sizeof(ContractSmem) + 128);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_contract_level, kCNT, sizeof(ContractSmem) + 128);
         per_sm = b > 0 ? (b > 4 ? 4 : b) : 1;
     }
-    return ctx->num_sms * per_sm;
+    const int g = ctx->num_sms * per_sm;
+    return g < kMaxContractCtas ? g : kMaxContractCtas;
 }
 
-size_t contract_status_words(int32_t n, int32_t nnz) {
-    const size_t t1 = (size_t)(n + kCTileV - 1) / kCTileV + 1;
-    const size_t t2 = (size_t)(nnz + kTileArcs - 1) / kTileArcs + 1;
-    return 4 * t1 + 2 * t2;
+size_t contract_tiles(int32_t n, int32_t nnz) {
+    return (size_t)(nnz + kWB - 1) / kWB + 2 * ((size_t)(n + kVW - 1) / kVW) + 8;
 }
-
-size_t contract_tiles(int32_t nnz) { return (size_t)(nnz + kTileArcs - 1) / kTileArcs + 2; }
 
 gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *CM, Graph *cg, ContractCtl *ctl,
                            SizeRec *out_sizes, LevelReport *report, const ContractParams &prm) {
@@ -803,19 +931,16 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
     a.vwgt = lb.vwgt;
     a.M = M;
     a.CM = CM;
-    a.leaders = lb.leaders;
     a.off = lb.off;
     a.cnt = lb.cnt;
     a.tile_start = lb.tile_start;
     a.huge = lb.huge;
-    a.rlen = lb.rlen;
+    a.lofs = lb.lofs;
+    a.tagg1 = lb.tagg1;
+    a.ttot = lb.ttot;
     a.seg = lb.seg;
     a.gkeys = lb.gkeys;
-    a.st1 = ctx->status;
-    a.st2 = ctx->status + 4 * ((size_t)(prm.n_bound + kCTileV - 1) / kCTileV + 1);
-    a.epoch = ctx->epoch;
-    ctx->epoch = (ctx->epoch + 1) & 0x7FFFFFFFu;
-    if (ctx->epoch == 0) ctx->epoch = 1;
+    a.tout = lb.tout;
     a.cadjp = cg->adjp;
     a.cadjncy = cg->adjncy;
     a.cadjwgt = cg->adjwgt;
@@ -828,14 +953,10 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
     a.level = prm.level;
     a.max_levels = prm.max_levels;
     a.report = report;
-    gp_status st = ensure_status(ctx, contract_status_words(prm.n_bound, prm.nnz_bound));
-    if (st != GP_OK) return st;
-    a.st1 = ctx->status;
-    a.st2 = ctx->status + 4 * ((size_t)(prm.n_bound + kCTileV - 1) / kCTileV + 1);
     void *args[] = {&a};
     LaunchScope ls(ctx, GP_K_CONTRACT);
     GP_CUDA(cudaLaunchCooperativeKernel((const void *)k_contract_level, dim3(contract_grid(ctx)), dim3(kCNT), args,
-                                        sizeof(ContractSmem), ctx->stream));
+                                        sizeof(ContractSmem) + 128, ctx->stream));
     ++ctx->launches;
     return GP_OK;
 }

@@ -194,22 +194,25 @@ __device__ __forceinline__ unsigned atom_add_acqrel_u32(unsigned *p, unsigned v)
     return old;
 }
 
-__device__ __forceinline__ void grid_barrier(unsigned *bar) {
+__device__ __forceinline__ void red_release_add_u32(unsigned *p, unsigned v) {
+    asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// bar[0] counts arrivals and only grows within a launch (zeroed before the launch); the
+// k-th barrier of the launch completes when it reaches k * gridDim.x.  The release-add
+// publishes the CTA's writes (bar.sync orders them before thread 0's release; release is
+// cumulative), the acquire poll makes every other CTA's writes visible after it.
+__device__ __forceinline__ void grid_barrier(unsigned *bar, unsigned &epoch) {
     __syncthreads();
     if (threadIdx.x == 0) {
-        const unsigned gen = ld_acquire_u32(bar + 1);
-        __threadfence();
-        if (atom_add_acqrel_u32(bar, 1u) == gridDim.x - 1) {
-            bar[0] = 0;
-            st_release_u32(bar + 1, gen + 1);
-        } else {
-            const long long guard = spin_start();
-            while (ld_acquire_u32(bar + 1) == gen) {
-                __nanosleep(32);
-                spin_check(guard);
-            }
+        ++epoch;
+        const unsigned target = epoch * gridDim.x;
+        red_release_add_u32(bar, 1u);
+        const long long guard = spin_start();
+        while ((int)(ld_acquire_u32(bar) - target) < 0) {
+            __nanosleep(20);
+            spin_check(guard);
         }
-        __threadfence();
     }
     __syncthreads();
 }

@@ -154,10 +154,11 @@ static gp_status alloc_graph_arrays(Ctx *ctx, Graph *g, int32_t n_bound, int32_t
 
 gp_status level_scratch(Ctx *ctx, int32_t n, int32_t nnz, LevelBufs *lb) {
     const size_t nn = (size_t)(n > 0 ? n : 1);
-    const size_t tiles = contract_tiles(nnz);
-    const size_t ints = 14 * nn + 1 + tiles + 16;
+    const size_t tiles = contract_tiles(n, nnz);
+    const size_t ints = 14 * nn + 1 + 3 * tiles + 32;
     const size_t ibytes = ((ints * 4 + 255) / 256) * 256;
-    gp_status st = ensure_scratch(ctx, ibytes + 8 * ((size_t)nnz + 4));
+    const size_t kbytes = ((8 * ((size_t)nnz + 4) + 255) / 256) * 256;
+    gp_status st = ensure_scratch(ctx, ibytes + 2 * kbytes);
     if (st != GP_OK) return st;
     int32_t *p = (int32_t *)ctx->scratch;
     lb->seg = (int4 *)p; p += 4 * nn;  // first: 16-byte aligned
@@ -166,13 +167,16 @@ gp_status level_scratch(Ctx *ctx, int32_t n, int32_t nnz, LevelBufs *lb) {
     lb->L[0] = p; p += nn;
     lb->L[1] = p; p += nn;
     lb->H = p; p += nn;
-    lb->leaders = p; p += nn;
+    lb->S = p; p += nn;
     lb->off = p; p += nn + 1;
     lb->cnt = p; p += nn;
     lb->huge = p; p += nn;
-    lb->rlen = p; p += nn;
+    lb->lofs = p; p += nn;
+    lb->tagg1 = p; p += tiles;
+    lb->ttot = p; p += tiles;
     lb->tile_start = p; p += tiles + 8;
     lb->gkeys = (unsigned long long *)((char *)ctx->scratch + ibytes);
+    lb->tout = (unsigned long long *)((char *)ctx->scratch + ibytes + kbytes);
     return GP_OK;
 }
 
@@ -650,8 +654,9 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
                 const unsigned long long *mt = hd[l].match.trace, *ct = hd[l].contract.trace;
                 fprintf(stderr, "[gp] level %d n=%d nnz=%d rounds=%d | match us:", l, L.n, L.nnz, L.rounds);
                 for (int q = 1; q < kTrace && mt[q]; ++q) fprintf(stderr, " %.1f", (mt[q] - mt[q - 1]) * 1e-3);
-                fprintf(stderr, " | contract us:");
-                for (int q = 1; q < 5 && ct[q]; ++q) fprintf(stderr, " %.1f", (ct[q] - ct[q - 1]) * 1e-3);
+                fprintf(stderr, " | contract us (c1a bar c1b bar hub c2a bar c2b):");
+                for (int q = 1; q < 9; ++q)
+                    fprintf(stderr, " %.1f", ct[q] && ct[q - 1] ? ((long long)ct[q] - (long long)ct[q - 1]) * 1e-3 : 0.0);
                 fprintf(stderr, " | gap to contract %.1f us\n", ct[0] && mt[1] ? ((long long)ct[0] - (long long)mt[0]) * 1e-3 : 0.0);
             }
         }

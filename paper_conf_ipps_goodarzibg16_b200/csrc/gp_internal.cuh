@@ -42,12 +42,16 @@ struct MatchCtl {
     int32_t pad[2];
 };
 
+constexpr int kMaxContractCtas = 1024;  // grid cap of the contraction kernel
+
 struct ContractCtl {
     unsigned long long trace[kTrace];
     unsigned bar[2];
-    unsigned tile_ctr[2];
     int32_t n_coarse, cnnz, n_huge;
     unsigned blocks_done;
+    int32_t chunk1[2 * kMaxContractCtas];  // C1 chunk sums {#leaders, sum ub} per owner CTA
+    int32_t chunk2[kMaxContractCtas];      // C2 chunk sums of merged entries per owner CTA
+    unsigned long long dbg[8];             // debug: slowest C2a warp tile (ns<<32 | tile), paths
 };
 
 // per-graph device size record: the producer of a coarse graph writes it
@@ -73,10 +77,11 @@ struct LevelReport {
 struct LevelBufs {
     const SizeRec *in;  // sizes (+ stop flag) of this level's input graph
     const int32_t *adjp, *adjncy, *adjwgt, *vwgt;
-    int32_t *P[2], *L[2], *H;                         // matching scratch
-    int32_t *leaders, *off, *cnt, *tile_start, *huge, *rlen;  // contraction scratch
+    int32_t *P[2], *L[2], *H, *S;                     // matching scratch
+    int32_t *off, *cnt, *tile_start, *huge, *lofs;  // contraction scratch
+    int32_t *tagg1, *ttot;  // tile aggregates of C1 and tile totals of C2
     int4 *seg;
-    unsigned long long *gkeys;
+    unsigned long long *gkeys, *tout;
 };
 
 }  // namespace gp
@@ -202,8 +207,7 @@ struct ContractParams {
 };
 gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *CM, Graph *coarse, ContractCtl *ctl,
                            SizeRec *out_sizes, LevelReport *report, const ContractParams &prm);
-size_t contract_status_words(int32_t n, int32_t nnz);
-size_t contract_tiles(int32_t nnz);
+size_t contract_tiles(int32_t n, int32_t nnz);
 
 gp_status graph_totals_and_validate(Ctx *ctx, const Graph *g, bool validate);
 

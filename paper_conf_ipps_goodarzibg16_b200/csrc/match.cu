@@ -47,6 +47,7 @@ struct MatchArgs {
     int32_t *P[2];
     int32_t *L[2];
     int32_t *H;  // hub list of the pending hub phase
+    int32_t *S;  // second-heaviest neighbour of the last full scan (NONE = none cached)
     MatchCtl *ctl;
     int32_t max_rounds;
     int32_t leftover;
@@ -67,6 +68,29 @@ struct MatchSmem {
 
 __device__ __forceinline__ int32_t ldcg(const int32_t *p) { return __ldcg(p); }
 
+// Warp-buffered list append (no CTA-wide synchronisation): the lanes with `pred` put `value`
+// into the warp's shared queue; a full queue is flushed with ONE global atomic and a
+// coalesced copy.  `qn` is the warp-uniform queue length.  All 32 lanes must call.
+constexpr int kWQ = 256;
+__device__ __forceinline__ void wq_flush(int32_t *q, int32_t &qn, int32_t *list, int32_t *counter) {
+    const int lane = threadIdx.x & 31;
+    if (qn == 0) return;
+    int32_t base = 0;
+    if (lane == 0) base = atomicAdd(counter, qn);
+    base = __shfl_sync(0xffffffffu, base, 0);
+    __syncwarp();
+    for (int i = lane; i < qn; i += 32) list[base + i] = q[i];
+    __syncwarp();
+    qn = 0;
+}
+__device__ __forceinline__ void wq_push(int32_t *q, int32_t &qn, int32_t *list, int32_t *counter, bool pred,
+                                        int32_t value) {
+    const unsigned m = __ballot_sync(0xffffffffu, pred);
+    if (pred) q[qn + __popc(m & lanemask_lt())] = value;
+    qn += __popc(m);
+    if (qn > kWQ - 32) wq_flush(q, qn, list, counter);
+}
+
 // x is free after round k's commits
 __device__ __forceinline__ bool free_after(int32_t x, const int32_t *M, const int32_t *Pk) {
     if (ldcg(M + x) != kFree) return false;
@@ -74,9 +98,35 @@ __device__ __forceinline__ bool free_after(int32_t x, const int32_t *M, const in
     return !(px >= 0 && ldcg(Pk + px) == x);
 }
 
-template <int G>
-__device__ __forceinline__ unsigned long long gmax(unsigned long long k) {
-    return group_max64<G>(k);
+// top-2 of packed keys (k1 > k2, both 0 = none)
+__device__ __forceinline__ void top2_add(unsigned long long &k1, unsigned long long &k2, unsigned long long k) {
+    if (k > k1) {
+        k2 = k1;
+        k1 = k;
+    } else if (k > k2) {
+        k2 = k;
+    }
+}
+template <int WIDTH>
+__device__ __forceinline__ void group_top2(unsigned long long &k1, unsigned long long &k2) {
+#pragma unroll
+    for (int off = WIDTH / 2; off > 0; off >>= 1) {
+        const unsigned long long o1 = __shfl_xor_sync(0xffffffffu, k1, off, WIDTH);
+        const unsigned long long o2 = __shfl_xor_sync(0xffffffffu, k2, off, WIDTH);
+        const unsigned long long lo = k1 < o1 ? k1 : o1;
+        k1 = k1 > o1 ? k1 : o1;
+        const unsigned long long m2 = k2 > o2 ? k2 : o2;
+        k2 = lo > m2 ? lo : m2;
+    }
+}
+__device__ __forceinline__ void group_top2_rt(unsigned long long &k1, unsigned long long &k2, int G) {
+    switch (G) {
+        case 1: return;
+        case 2: group_top2<2>(k1, k2); return;
+        case 4: group_top2<4>(k1, k2); return;
+        case 8: group_top2<8>(k1, k2); return;
+        default: group_top2<16>(k1, k2); return;
+    }
 }
 
 __device__ __forceinline__ unsigned long long group_max_rt(unsigned long long k, int G) {
@@ -171,27 +221,29 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
                     e = __ldg(a.adjp + v + 1);
                 }
             }
-            unsigned long long key = 0;
+            unsigned long long key = 0, key2 = 0;
             bool hub = false;
             if (fits) {
                 const int32_t *sa = sm.adj[st], *sw = sm.wgt[st];
-                for (int32_t j = s - A0 + gl; j < e - A0; j += G) key = umax64(key, pack_key(sw[j], sa[j]));
+                for (int32_t j = s - A0 + gl; j < e - A0; j += G) top2_add(key, key2, pack_key(sw[j], sa[j]));
             } else if (valid) {
                 if (e - s > kHubDeg) {
                     hub = true;
                 } else {
                     for (int32_t j = s + gl; j < e; j += G)
-                        key = umax64(key, pack_key(__ldg(a.adjwgt + j), __ldg(a.adjncy + j)));
+                        top2_add(key, key2, pack_key(__ldg(a.adjwgt + j), __ldg(a.adjncy + j)));
                 }
             }
-            key = group_max_rt(key, G);
+            group_top2_rt(key, key2, G);
             if (valid && gl == 0) {
                 a.M[v] = kFree;
                 if (hub) {
                     a.H[atomicAdd(&a.ctl->slot[1].nhub, 1)] = (int32_t)v;
+                    a.S[v] = kNone;
                 } else {
                     const int32_t p = key_vertex(key);
                     P1[v] = p;
+                    a.S[v] = key_vertex(key2);  // cached second-heaviest neighbour
                     if (p == kNone) P0[v] = kNone;  // dead vertices: NONE in both buffers
                     scanned += (unsigned long long)(e - s);
                 }
@@ -229,6 +281,7 @@ __device__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool 
             for (int q = 0; q < kNT / 32; ++q) k = umax64(k, sm.red[q]);
             const int32_t p = key_vertex(k);
             Pn[u] = p;
+            a.S[u] = kNone;
             if (p == kNone) {
                 a.P[0][u] = kNone;
                 a.P[1][u] = kNone;
@@ -244,6 +297,29 @@ __device__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool 
 // ---------------------------------------------------------------------------------------
 // phase k >= 1: commit of round k + proposals of round k+1 (lazy rescans)
 // ---------------------------------------------------------------------------------------
+// thread rescan of u's row (<= kThreadDeg arcs) in batches of 8 arcs: every dependent level
+// (arc -> M[x] -> P_k[x] -> P_k[P_k[x]]) is issued for the whole batch at once; top-2 kept
+__device__ __forceinline__ void rescan_thread(const MatchArgs &a, const int32_t *Pk, int32_t s, int32_t e,
+                                              unsigned long long &key, unsigned long long &key2) {
+    key = key2 = 0;
+    for (int32_t j0 = s; j0 < e; j0 += 8) {
+        int32_t x[8], m[8], px[8], pp[8];
+#pragma unroll
+        for (int b = 0; b < 8; ++b) x[b] = (j0 + b < e) ? __ldg(a.adjncy + j0 + b) : -1;
+#pragma unroll
+        for (int b = 0; b < 8; ++b) m[b] = (x[b] >= 0) ? ldcg(a.M + x[b]) : 0;
+#pragma unroll
+        for (int b = 0; b < 8; ++b) px[b] = (x[b] >= 0 && m[b] == kFree) ? ldcg(Pk + x[b]) : -1;
+#pragma unroll
+        for (int b = 0; b < 8; ++b) pp[b] = (px[b] >= 0) ? ldcg(Pk + px[b]) : -1;
+#pragma unroll
+        for (int b = 0; b < 8; ++b)
+            if (x[b] >= 0 && m[b] == kFree && pp[b] != x[b]) top2_add(key, key2, pack_key(__ldg(a.adjwgt + j0 + b), x[b]));
+    }
+}
+
+constexpr int kVL = 4;  // live vertices per lane per step (their dependent loads overlap)
+
 __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, unsigned long long &scanned,
                         unsigned long long &rows, unsigned long long &visits, int32_t &made) {
     const int32_t *Pk = a.P[k & 1];
@@ -253,104 +329,131 @@ __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int
     int32_t *Ln = a.L[(k + 1) & 1];
     RoundSlot *next = &a.ctl->slot[(k + 1) & 3];
     const int lane = threadIdx.x & 31;
-    const long long stride = (long long)gridDim.x * kNT;
-    for (long long base = (long long)blockIdx.x * kNT; base < len; base += stride) {
-        const long long idx = base + threadIdx.x;
-        bool live_next = false, need_warp = false;
-        int32_t u = -1, s = 0, e = 0;
-        if (idx < len) {
-            u = (k == 1) ? (int32_t)idx : ldcg(Lk + idx);
-            const int32_t p = ldcg(Pk + u);
-            if (p != kNone) {
-                ++visits;
-                const int32_t q = ldcg(Pk + p);
-                if (q == u) {
-                    a.M[u] = p;  // handshake: u and p propose each other
-                    Pn[u] = p;
-                    ++made;
-                } else if (!(q >= 0 && ldcg(Pk + q) == p)) {
-                    Pn[u] = p;  // p is still free: still the heaviest free neighbour
-                    live_next = true;
+    int32_t *q = reinterpret_cast<int32_t *>(&sm.adj[0][0]) + (threadIdx.x >> 5) * kWQ;  // phase 0 is over
+    int32_t qn = 0;
+    // warp-uniform grid-stride loop over groups of 32*kVL entries: warps never wait for their CTA
+    const long long wstride = (long long)gridDim.x * kNT * kVL;
+    for (long long base = ((long long)blockIdx.x * kNT + (threadIdx.x & ~31)) * kVL; base < len; base += wstride) {
+        int32_t u[kVL], p[kVL], s2[kVL], qq[kVL], rr[kVL], ms[kVL], ps[kVL], pps[kVL];
+        // level 1: the vertices; level 2: P_k[u] and the cached second candidate S[u]
+#pragma unroll
+        for (int i = 0; i < kVL; ++i) {
+            const long long idx = base + i * 32 + lane;
+            u[i] = idx < len ? ((k == 1) ? (int32_t)idx : ldcg(Lk + idx)) : -1;
+        }
+#pragma unroll
+        for (int i = 0; i < kVL; ++i) {
+            p[i] = u[i] >= 0 ? ldcg(Pk + u[i]) : kNone;
+            s2[i] = (u[i] >= 0 && p[i] != kNone) ? ldcg(a.S + u[i]) : kNone;
+        }
+        // level 3: P_k[p] and the freedom test of the cached candidate (M, P_k)
+#pragma unroll
+        for (int i = 0; i < kVL; ++i) {
+            qq[i] = p[i] != kNone ? ldcg(Pk + p[i]) : kNone;
+            ms[i] = s2[i] != kNone ? ldcg(a.M + s2[i]) : 0;
+            ps[i] = (s2[i] != kNone && ms[i] == kFree) ? ldcg(Pk + s2[i]) : -1;
+        }
+        // level 4: P_k[q] (did p match q?) and P_k[P_k[s2]]
+#pragma unroll
+        for (int i = 0; i < kVL; ++i) {
+            rr[i] = (p[i] != kNone && qq[i] != u[i] && qq[i] >= 0) ? ldcg(Pk + qq[i]) : -1;
+            pps[i] = ps[i] >= 0 ? ldcg(Pk + ps[i]) : -1;
+        }
+        bool need[kVL];
+#pragma unroll
+        for (int i = 0; i < kVL; ++i) {
+            need[i] = false;
+            if (p[i] == kNone) continue;
+            ++visits;
+            if (qq[i] == u[i]) {
+                a.M[u[i]] = p[i];  // handshake: u and p propose each other
+                Pn[u[i]] = p[i];
+                ++made;
+                u[i] = -1;  // done
+            } else if (rr[i] != p[i]) {
+                Pn[u[i]] = p[i];  // p is still free: still the heaviest free neighbour
+            } else if (s2[i] != kNone && ms[i] == kFree && pps[i] != s2[i]) {
+                // the cached second-heaviest neighbour of u's last scan is still free: it is
+                // now u's heaviest free neighbour (the free set only shrinks)
+                Pn[u[i]] = s2[i];
+                a.S[u[i]] = kNone;
+            } else {
+                need[i] = true;  // full rescan
+            }
+        }
+        bool live[kVL];
+#pragma unroll
+        for (int i = 0; i < kVL; ++i) {
+            live[i] = u[i] >= 0 && p[i] != kNone && !need[i];
+            int32_t s = 0, e = 0;
+            bool need_warp = false;
+            if (need[i]) {
+                s = __ldg(a.adjp + u[i]);
+                e = __ldg(a.adjp + u[i] + 1);
+                ++rows;
+                if (e - s <= kThreadDeg) {
+                    unsigned long long key, key2;
+                    rescan_thread(a, Pk, s, e, key, key2);
+                    scanned += (unsigned long long)(e - s);
+                    const int32_t b = key_vertex(key);
+                    Pn[u[i]] = b;
+                    a.S[u[i]] = key_vertex(key2);
+                    if (b == kNone) Pkw[u[i]] = kNone;
+                    live[i] = b != kNone;
+                } else if (e - s <= kHubDeg) {
+                    need_warp = true;
                 } else {
-                    s = __ldg(a.adjp + u);
-                    e = __ldg(a.adjp + u + 1);
-                    ++rows;
-                    if (e - s <= kThreadDeg) {
-                        // batches of 8 arcs: every dependent load level is issued for the
-                        // whole batch at once (arc -> M[x] -> P_k[x] -> P_k[P_k[x]])
-                        unsigned long long key = 0;
-                        for (int32_t j0 = s; j0 < e; j0 += 8) {
-                            int32_t x[8], m[8], px[8], pp[8];
-#pragma unroll
-                            for (int b = 0; b < 8; ++b) x[b] = (j0 + b < e) ? __ldg(a.adjncy + j0 + b) : -1;
-#pragma unroll
-                            for (int b = 0; b < 8; ++b) m[b] = (x[b] >= 0) ? ldcg(a.M + x[b]) : 0;
-#pragma unroll
-                            for (int b = 0; b < 8; ++b) px[b] = (x[b] >= 0 && m[b] == kFree) ? ldcg(Pk + x[b]) : -1;
-#pragma unroll
-                            for (int b = 0; b < 8; ++b) pp[b] = (px[b] >= 0) ? ldcg(Pk + px[b]) : -1;
-#pragma unroll
-                            for (int b = 0; b < 8; ++b)
-                                if (x[b] >= 0 && m[b] == kFree && pp[b] != x[b])
-                                    key = umax64(key, pack_key(__ldg(a.adjwgt + j0 + b), x[b]));
-                        }
-                        scanned += (unsigned long long)(e - s);
-                        const int32_t b = key_vertex(key);
-                        Pn[u] = b;
-                        if (b == kNone) Pkw[u] = kNone;
-                        live_next = b != kNone;
-                    } else if (e - s <= kHubDeg) {
-                        need_warp = true;
-                    } else {
-                        a.H[atomicAdd(&next->nhub, 1)] = u;
-                    }
+                    a.H[atomicAdd(&next->nhub, 1)] = u[i];
                 }
             }
-        }
-        // medium rows: the whole warp rescans one row at a time
-        unsigned mm = __ballot_sync(0xffffffffu, need_warp);
-        while (mm) {
-            const int src = __ffs(mm) - 1;
-            mm &= mm - 1;
-            const int32_t su = __shfl_sync(0xffffffffu, s, src), eu = __shfl_sync(0xffffffffu, e, src);
-            unsigned long long key = 0;
-            for (int32_t j = su + lane; j < eu; j += 32) {
-                const int32_t x = __ldg(a.adjncy + j);
-                if (free_after(x, a.M, Pk)) key = umax64(key, pack_key(__ldg(a.adjwgt + j), x));
+            // medium rows: the whole warp rescans one row at a time
+            unsigned mm = __ballot_sync(0xffffffffu, need_warp);
+            while (mm) {
+                const int src = __ffs(mm) - 1;
+                mm &= mm - 1;
+                const int32_t su = __shfl_sync(0xffffffffu, s, src), eu = __shfl_sync(0xffffffffu, e, src);
+                unsigned long long key = 0, key2 = 0;
+                for (int32_t j = su + lane; j < eu; j += 32) {
+                    const int32_t x = __ldg(a.adjncy + j);
+                    if (free_after(x, a.M, Pk)) top2_add(key, key2, pack_key(__ldg(a.adjwgt + j), x));
+                }
+                group_top2<32>(key, key2);
+                if (lane == src) {
+                    const int32_t b = key_vertex(key);
+                    Pn[u[i]] = b;
+                    a.S[u[i]] = key_vertex(key2);
+                    if (b == kNone) Pkw[u[i]] = kNone;
+                    live[i] = b != kNone;
+                    scanned += (unsigned long long)(eu - su);
+                }
             }
-            key = group_max64<32>(key);
-            if (lane == src) {
-                const int32_t b = key_vertex(key);
-                Pn[u] = b;
-                if (b == kNone) Pkw[u] = kNone;
-                live_next = b != kNone;
-                scanned += (unsigned long long)(eu - su);
-            }
+            wq_push(q, qn, Ln, &next->live, live[i], u[i]);
         }
-        block_append<kNT>(Ln, &next->live, live_next, u, sm.scratch);
     }
+    wq_flush(q, qn, Ln, &next->live);
 }
 
 __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ MatchArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    MatchSmem &sm = *reinterpret_cast<MatchSmem *>(smem_raw);
+    MatchSmem &sm = *reinterpret_cast<MatchSmem *>(((uintptr_t)smem_raw + 127) & ~(uintptr_t)127);
     MatchCtl *ctl = a.ctl;
     const volatile SizeRec *in = a.in;
     if (in->stop) return;  // an earlier level ended the coarsening: nothing to do
     const int32_t n = in->n;
     if (n <= 0) return;
     unsigned long long scanned = 0, rows = 0, visits = 0;
+    unsigned bar_epoch = 0;  // grid barriers passed (thread 0)
     int tr = 0;
     trace_mark(ctl->trace, tr++);
     phase0(a, sm, n, scanned);
     trace_mark(ctl->trace, tr++);
-    grid_barrier(ctl->bar);
+    grid_barrier(ctl->bar, bar_epoch);
     trace_mark(ctl->trace, tr++);
     {
         const int32_t nh = *(volatile int32_t *)&ctl->slot[1].nhub;
         if (nh > 0) {
             hub_phase(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned);
-            grid_barrier(ctl->bar);
+            grid_barrier(ctl->bar, bar_epoch);
         }
     }
     int32_t rounds = 0, maximal = 0;
@@ -368,13 +471,13 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
         made = warp_sum(made);
         if ((threadIdx.x & 31) == 0 && made) atomicAdd(&ctl->slot[k & 3].matches, made);
         trace_mark(ctl->trace, tr++);
-        grid_barrier(ctl->bar);
+        grid_barrier(ctl->bar, bar_epoch);
         trace_mark(ctl->trace, tr++);
         const int32_t nh = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].nhub;
         if (nh > 0) {
             hub_phase(a, sm, nh, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1], &ctl->slot[(k + 1) & 3].live,
                       scanned);
-            grid_barrier(ctl->bar);
+            grid_barrier(ctl->bar, bar_epoch);
         }
         if (*(volatile int32_t *)&ctl->slot[k & 3].matches > 0) ++rounds;
         const int32_t live = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].live;
@@ -419,8 +522,8 @@ int match_grid(Ctx *ctx) {
     static int per_sm = -1;
     if (per_sm < 0) {
         int b = 0;
-        cudaFuncSetAttribute(k_match_level, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(MatchSmem));
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_match_level, kNT, sizeof(MatchSmem));
+        cudaFuncSetAttribute(k_match_level, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(MatchSmem) + 128);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_match_level, kNT, sizeof(MatchSmem) + 128);
         per_sm = b > 0 ? (b > 2 ? 2 : b) : 1;
     }
     return ctx->num_sms * per_sm;
@@ -439,6 +542,7 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     a.L[0] = lb.L[0];
     a.L[1] = lb.L[1];
     a.H = lb.H;
+    a.S = lb.S;
     a.ctl = ctl;
     a.max_rounds = max_rounds;
     a.leftover = leftover ? 1 : 0;
@@ -452,7 +556,7 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     void *args[] = {&a};
     LaunchScope ls(ctx, GP_K_PROPOSE);
     GP_CUDA(cudaLaunchCooperativeKernel((const void *)k_match_level, dim3(match_grid(ctx)), dim3(kNT), args,
-                                        sizeof(MatchSmem), ctx->stream));
+                                        sizeof(MatchSmem) + 128, ctx->stream));
     ++ctx->launches;
     return GP_OK;
 }

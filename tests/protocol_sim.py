@@ -20,18 +20,24 @@ def _key(w, v):
     return (int(w) << 32) | (0xFFFFFFFF - int(v))
 
 
-def simulate_match(adjp, adjncy, adjwgt, seed=0, max_rounds=0):
+def simulate_match(adjp, adjncy, adjwgt, seed=0, max_rounds=0, use_cache=True):
     rng = np.random.default_rng(seed)
     n = len(adjp) - 1
     M = np.full(n, FREE, dtype=np.int64)
     P = [np.full(n, 123456789, dtype=np.int64), np.full(n, 987654321, dtype=np.int64)]  # garbage
-    # phase 0: round-1 proposals of every vertex
+    S = np.full(n, NONE, dtype=np.int64)  # cached second-heaviest neighbour of the last scan
+
+    def vert(k):
+        return NONE if k == 0 else 0xFFFFFFFF - (k & 0xFFFFFFFF)
+
+    # phase 0: round-1 proposals (top-2) of every vertex
     for u in rng.permutation(n):
-        best = 0
-        for j in range(adjp[u], adjp[u + 1]):
-            best = max(best, _key(adjwgt[j], adjncy[j]))
-        p = NONE if best == 0 else 0xFFFFFFFF - (best & 0xFFFFFFFF)
+        keys = sorted((_key(adjwgt[j], adjncy[j]) for j in range(adjp[u], adjp[u + 1])), reverse=True)
+        best = keys[0] if keys else 0
+        second = keys[1] if len(keys) > 1 else 0
+        p = vert(best)
         P[1][u] = p
+        S[u] = vert(second)
         if p == NONE:
             P[0][u] = NONE
     live = [u for u in range(n) if P[1][u] != NONE]
@@ -61,13 +67,15 @@ def simulate_match(adjp, adjncy, adjwgt, seed=0, max_rounds=0):
             elif not (q >= 0 and Pk[q] == p):
                 Pn[u] = p
                 nxt.append(u)
+            elif use_cache and S[u] != NONE and free_after(S[u]):
+                Pn[u] = S[u]
+                S[u] = NONE
+                nxt.append(u)
             else:
-                best = 0
-                for j in range(adjp[u], adjp[u + 1]):
-                    x = adjncy[j]
-                    if free_after(x):
-                        best = max(best, _key(adjwgt[j], x))
-                b = NONE if best == 0 else 0xFFFFFFFF - (best & 0xFFFFFFFF)
+                keys = sorted((_key(adjwgt[j], adjncy[j]) for j in range(adjp[u], adjp[u + 1])
+                               if free_after(adjncy[j])), reverse=True)
+                b = vert(keys[0]) if keys else NONE
+                S[u] = vert(keys[1]) if len(keys) > 1 else NONE
                 Pn[u] = b
                 if b == NONE:
                     Pk[u] = NONE

@@ -23,8 +23,9 @@ def test_fused_round_protocol_equals_oracle(n, m, seed, wmax):
     gn = np_graph(g)
     ref_m, ref_r, ref_max = oracle.match_level(g)
     for order_seed in range(3):
-        sm, sr, smax = simulate_match(gn["adjp"], gn["adjncy"], gn["adjwgt"], seed=order_seed)
-        assert np.array_equal(sm, ref_m) and sr == ref_r and smax == ref_max
+        for cache in (True, False):
+            sm, sr, smax = simulate_match(gn["adjp"], gn["adjncy"], gn["adjwgt"], seed=order_seed, use_cache=cache)
+            assert np.array_equal(sm, ref_m) and sr == ref_r and smax == ref_max
 
 
 @pytest.mark.parametrize("cap", [1, 2, 3])
