@@ -449,7 +449,8 @@ __device__ void phase_c1a(const ContractArgs &a, int32_t n, int nt1, int T1) {
 // ---------------------------------------------------------------------------------------
 // C1b: CM, cvwgt, off, seg, C2 warp-tile starts, huge rows
 // ---------------------------------------------------------------------------------------
-__device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, int nt1, int T1, int32_t ntiles2) {
+__device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, int nt1, int T1, int32_t ntiles2,
+                          int32_t tb) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int t_lo = blockIdx.x * T1, t_hi = min(nt1, t_lo + T1);
     if (t_lo >= t_hi) return;
@@ -522,9 +523,9 @@ __device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, in
                 a.cvwgt[c] = vw[q];
                 a.off[c] = o;
                 a.seg[c] = make_int4(su[q], dl, sv[q], d[i] - dl);
-                // warp tile t2 starts at the first row with off >= t2*kWB: row c+1 for
-                // every t2 with off[c] < t2*kWB <= off[c+1]
-                for (int32_t t2 = o / kWB + 1; t2 <= (o + d[i]) / kWB && t2 < ntiles2; ++t2) a.tile_start[t2] = c + 1;
+                // warp tile t2 starts at the first row with off >= t2*tb: row c+1 for
+                // every t2 with off[c] < t2*tb <= off[c+1]
+                for (int32_t t2 = o / tb + 1; t2 <= (o + d[i]) / tb && t2 < ntiles2; ++t2) a.tile_start[t2] = c + 1;
                 if (d[i] > kWB) a.huge[atomicAdd(&a.ctl->n_huge, 1)] = c;
                 ++c;
                 o += d[i];
@@ -593,11 +594,16 @@ __device__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
 // ---------------------------------------------------------------------------------------
 // C2a: warp tiles: merge every row, write the tile compacted to tout at its ub offset
 // ---------------------------------------------------------------------------------------
-__device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntiles2, int T2) {
+__device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntiles2, int T2, int32_t tb) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int gw = blockIdx.x * kCW + wib, nw = gridDim.x * kCW;
     unsigned long long *wb = sm.buf + wib * 2 * kWB;  // this warp's slots (2*kWB entries)
-    for (int wt = gw; wt < ntiles2; wt += nw) {
+    (void)gw;
+    (void)nw;
+    // warp tiles are claimed dynamically (balances the tail of the phase)
+    for (int wt = (lane == 0) ? (int)atomicAdd(&a.ctl->tile_ctr, 1u) : 0;;) {
+        wt = __shfl_sync(0xffffffffu, wt, 0);
+        if (wt >= ntiles2) break;
         int32_t r0 = 0, r1 = 0;
         if (lane < 2) {
             const int32_t x = __ldcg(a.tile_start + wt + lane);
@@ -605,7 +611,7 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
         }
         r1 = __shfl_sync(0xffffffffu, r0, 1);
         r0 = __shfl_sync(0xffffffffu, r0, 0);
-        const int32_t tbase = wt * kWB;
+        const int32_t tbase = wt * tb;  // slots: a row starting in the tile ends below tb + kWB <= 2kWB
         unsigned long long *out = a.tout + (r0 < r1 ? __ldcg(a.off + r0) : 0);
         int32_t run = 0;
         for (int32_t g0 = r0; g0 < r1; g0 += 32) {
@@ -758,6 +764,7 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
         if (lane == 0) {
             a.ttot[wt] = run;
             atomicAdd(&a.ctl->chunk2[wt / T2], run);
+            wt = (int)atomicAdd(&a.ctl->tile_ctr, 1u);
         }
     }
 }
@@ -838,7 +845,10 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
     unsigned bar_epoch = 0;  // grid barriers passed (thread 0)
     const int nt1 = (n + kVW - 1) / kVW;
     const int T1 = (nt1 + gridDim.x - 1) / gridDim.x;            // C1b tiles per CTA
-    const int32_t ntiles2 = nnz > 0 ? (nnz + kWB - 1) / kWB : 0;
+    // C2 warp-tile budget: kWB, halved (down to 32) while there are < 4 tiles per warp
+    int32_t tb = kWB;
+    while (tb > 32 && (long long)nnz < 4LL * tb * gridDim.x * kCW) tb >>= 1;
+    const int32_t ntiles2 = nnz > 0 ? (nnz + tb - 1) / tb : 0;
     const int T2 = (ntiles2 + gridDim.x - 1) / gridDim.x;        // C2b tiles per CTA
     trace_mark(ctl->trace, 0);
     if (n > 0) {
@@ -846,7 +856,7 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
         trace_mark(ctl->trace, 1);
         grid_barrier(ctl->bar, bar_epoch);
         trace_mark(ctl->trace, 2);
-        phase_c1b(a, sm, n, nt1, T1, ntiles2);
+        phase_c1b(a, sm, n, nt1, T1, ntiles2, tb);
         trace_mark(ctl->trace, 3);
         grid_barrier(ctl->bar, bar_epoch);
     }
@@ -859,7 +869,7 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
     }
     trace_mark(ctl->trace, 5);
     if (ntiles2 > 0) {
-        phase_c2a(a, sm, ntiles2, T2);
+        phase_c2a(a, sm, ntiles2, T2, tb);
         trace_mark(ctl->trace, 6);
         grid_barrier(ctl->bar, bar_epoch);
         trace_mark(ctl->trace, 7);
@@ -918,7 +928,7 @@ int contract_grid(Ctx *ctx) {
 }
 
 size_t contract_tiles(int32_t n, int32_t nnz) {
-    return (size_t)(nnz + kWB - 1) / kWB + 2 * ((size_t)(n + kVW - 1) / kVW) + 8;
+    return (size_t)(nnz + 31) / 32 + 2 * ((size_t)(n + kVW - 1) / kVW) + 8;  // smallest budget: 32
 }
 
 gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *CM, Graph *cg, ContractCtl *ctl,

@@ -36,6 +36,8 @@ constexpr int kTrace = 48;  // phase timestamps per kernel (debug tracing)
 struct MatchCtl {
     unsigned long long trace[kTrace];  // %globaltimer at phase boundaries (block 0; debug)
     unsigned bar[2];   // grid barrier
+    unsigned chunk_ctr;  // dynamic phase-0 chunk claims
+    unsigned pad0;
     RoundSlot slot[4]; // ring by round number
     int32_t rounds, maximal;
     unsigned long long arcs_scanned, rows_scanned, live_visits;
@@ -49,6 +51,8 @@ struct ContractCtl {
     unsigned bar[2];
     int32_t n_coarse, cnnz, n_huge;
     unsigned blocks_done;
+    unsigned tile_ctr;  // dynamic C2a warp-tile claims
+    unsigned pad0;
     int32_t chunk1[2 * kMaxContractCtas];  // C1 chunk sums {#leaders, sum ub} per owner CTA
     int32_t chunk2[kMaxContractCtas];      // C2 chunk sums of merged entries per owner CTA
     unsigned long long dbg[8];             // debug: slowest C2a warp tile (ns<<32 | tile), paths

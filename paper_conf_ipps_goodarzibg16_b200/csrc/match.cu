@@ -61,7 +61,8 @@ struct MatchSmem {
     int32_t ap[kStages][kMaxVch + 8];  // adjp[v0 .. v0+vch] of the staged chunk
     uint64_t bar[kStages];
     int32_t a0[kStages];    // aligned first arc of the staged chunk
-    int32_t fits[kStages];  // 1 staged, 2 empty, 0 fallback
+    int32_t fits[kStages];  // 1 staged, 0 fallback
+    long long cid[kStages]; // chunk staged in the stage (claimed dynamically; >= nchunks: none)
     int32_t scratch[40];
     unsigned long long red[kNT / 32];
 };
@@ -179,26 +180,30 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
     const long long nchunks = ((long long)n + a.vch - 1) / a.vch;
     const int t = threadIdx.x, gl = t % G, grp = t / G;
     int32_t *P1 = a.P[1], *P0 = a.P[0];
-    int32_t nb_s = 0, nb_e = 0;  // thread 0: prefetched bounds of the next chunk to stage
+    // thread 0 claims chunks dynamically (balances the tail) and keeps kStages in flight
+    long long nxt = -1;          // next claimed chunk, bounds prefetched
+    int32_t nb_s = 0, nb_e = 0;
     if (t == 0) {
         for (int q = 0; q < kStages; ++q) mbar_init(&sm.bar[q], 1);
         fence_mbar_init();
         for (int q = 0; q < kStages; ++q) {
-            const long long c = blockIdx.x + (long long)q * gridDim.x;
+            const long long c = atomicAdd(&a.ctl->chunk_ctr, 1u);
+            sm.cid[q] = c;
             if (c < nchunks) {
                 int32_t cs, ce;
                 load_bounds(a, n, nchunks, c, cs, ce);
                 stage_chunk(a, sm, n, c, cs, ce, q);
             }
         }
-        load_bounds(a, n, nchunks, blockIdx.x + (long long)kStages * gridDim.x, nb_s, nb_e);
+        nxt = atomicAdd(&a.ctl->chunk_ctr, 1u);
+        load_bounds(a, n, nchunks, nxt, nb_s, nb_e);
     }
     __syncthreads();
     unsigned uses[kStages] = {};
     for (long long i = 0;; ++i) {
-        const long long c = blockIdx.x + i * gridDim.x;
-        if (c >= nchunks) break;
         const int st = (int)(i % kStages);
+        const long long c = sm.cid[st];
+        if (c >= nchunks) break;  // chunks are claimed in order: later stages are empty too
         const bool fits = sm.fits[st] != 0;
         const int32_t A0 = sm.a0[st];
         if (fits) {
@@ -251,10 +256,14 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
         }
         __syncthreads();  // stage `st` is free again
         if (t == 0) {
-            const long long c2 = blockIdx.x + (i + kStages) * gridDim.x;
-            if (c2 < nchunks) stage_chunk(a, sm, n, c2, nb_s, nb_e, st);
-            load_bounds(a, n, nchunks, c2 + gridDim.x, nb_s, nb_e);  // in flight during the next chunk
+            sm.cid[st] = nxt;
+            if (nxt < nchunks) {
+                stage_chunk(a, sm, n, nxt, nb_s, nb_e, st);
+                nxt = atomicAdd(&a.ctl->chunk_ctr, 1u);
+                load_bounds(a, n, nchunks, nxt, nb_s, nb_e);  // in flight during the next chunk
+            }
         }
+        __syncthreads();
     }
 }
 
@@ -318,10 +327,11 @@ __device__ __forceinline__ void rescan_thread(const MatchArgs &a, const int32_t 
     }
 }
 
-constexpr int kVL = 4;  // live vertices per lane per step (their dependent loads overlap)
-
-__device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, unsigned long long &scanned,
-                        unsigned long long &rows, unsigned long long &visits, int32_t &made) {
+// kVL live vertices per lane per step: their dependent loads overlap.  4 on long lists, 1 on
+// short ones (a wide step would leave most warps idle).
+template <int kVL>
+__device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t len, unsigned long long &scanned,
+                             unsigned long long &rows, unsigned long long &visits, int32_t &made) {
     const int32_t *Pk = a.P[k & 1];
     int32_t *Pn = a.P[(k + 1) & 1];
     int32_t *Pkw = a.P[k & 1];
@@ -433,6 +443,13 @@ __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int
     wq_flush(q, qn, Ln, &next->live);
 }
 
+__device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, unsigned long long &scanned,
+                        unsigned long long &rows, unsigned long long &visits, int32_t &made) {
+    (void)n;
+    if ((long long)len >= 4LL * gridDim.x * kNT) phase_k_impl<4>(a, sm, k, len, scanned, rows, visits, made);
+    else phase_k_impl<1>(a, sm, k, len, scanned, rows, visits, made);
+}
+
 __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ MatchArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     MatchSmem &sm = *reinterpret_cast<MatchSmem *>(((uintptr_t)smem_raw + 127) & ~(uintptr_t)127);
@@ -510,12 +527,12 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
 // host side
 // ---------------------------------------------------------------------------------------
 static int choose_group(double avg_deg) {
-    // lanes per vertex in phase 0: about one arc per lane
-    if (avg_deg <= 1.5) return 1;
-    if (avg_deg <= 3.0) return 2;
-    if (avg_deg <= 6.5) return 4;
-    if (avg_deg <= 13.0) return 8;
-    return 16;
+    // lanes per vertex in phase 0.  The rows come from shared memory, so a thread per row is
+    // cheapest in instructions (no 64-bit top-2 shuffles) up to ~12 arcs per row.
+    if (avg_deg <= 12.0) return 1;
+    if (avg_deg <= 24.0) return 2;
+    if (avg_deg <= 48.0) return 4;
+    return 8;
 }
 
 int match_grid(Ctx *ctx) {
@@ -548,9 +565,12 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     a.leftover = leftover ? 1 : 0;
     a.G = choose_group(avg_deg_hint);
     {
+        // vertices per chunk: ~80 % of a stage at the average degree, a multiple of the
+        // number of vertex groups (kNT / G) so that no group pass runs mostly idle
         const double d = avg_deg_hint > 0.5 ? avg_deg_hint : 0.5;
+        const int ng = kNT / a.G;
         int v = (int)(0.8 * kStageArcs / d);
-        v = (v / 32) * 32;
+        v = v >= ng ? (v / ng) * ng : (v / 32) * 32;
         a.vch = v < 32 ? 32 : (v > kMaxVch ? kMaxVch : v);
     }
     void *args[] = {&a};
