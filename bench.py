@@ -78,6 +78,19 @@ def level_bytes(l) -> dict:
     return {"match": match, "contract": contract}
 
 
+def ncu_traffic(config: str, kernel: str):
+    """DRAM bytes (read + write) per step of `kernel` from the committed ncu launch list
+    (profiles/r1/ncu_traffic_<config>.json, written by scripts/summarize_profiles.py from one
+    profiled gp_coarsen_to), or None when no capture of this config is committed."""
+    path = os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "r1",
+                        f"ncu_traffic_{config}.json")
+    try:
+        j = json.load(open(path))
+        return float(j["kernels"][kernel]["dram_bytes"]), "profiles/r1/" + os.path.basename(path)
+    except Exception:
+        return None
+
+
 # ------------------------------------------------------------------------------------------
 # clocks sampled during the timed region
 # ------------------------------------------------------------------------------------------
@@ -243,6 +256,7 @@ def run_ours(args, rank, world, local_rank):
     peak, peak_kind = peaks()
     achieved = fam_bytes[dom] / (fam_ms[dom] / 1e3) / 1e9 if fam_ms[dom] > 0 else 0.0
     step_bytes = sum(fam_bytes.values())
+    traffic = ncu_traffic(args.config, {"match": "k_match_level", "contract": "k_contract_level"}[dom])
 
     # end-to-end through the C ABI with host buffers
     host = {k: g[k].cpu().pin_memory() for k in ("adjp", "adjncy", "adjwgt", "vwgt")}
@@ -292,7 +306,9 @@ def run_ours(args, rank, world, local_rank):
                    "gen_s": round(gen_s, 2)},
         "hbm_gbs_step": step_bytes / (ms_step / 1e3) / 1e9,
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "peak_kind": peak_kind,
-                     "unit": "GB/s", "frac": achieved / peak, "traffic": None,
+                     "unit": "GB/s", "frac": achieved / peak,
+                     "traffic": traffic[0] if traffic else None,
+                     "traffic_source": traffic[1] if traffic else None,
                      "bytes_per_step": fam_bytes[dom], "ms_per_step": fam_ms[dom]},
         "kernels": {k: {"ms_per_step": fam_ms[k], "GB/s": (fam_bytes[k] / (fam_ms[k] / 1e3) / 1e9) if fam_ms[k] else None,
                         "launches_per_step": kstats[kfam[k]]["launches"] / args.steps} for k in fam_bytes},
