@@ -28,7 +28,7 @@ struct RoundSlot {
     int32_t live;     // live-list length of the round this slot belongs to
     int32_t nhub;     // hub rows waiting for the hub phase
     int32_t matches;  // matches made by the round's commit
-    int32_t pad;
+    int32_t claim;    // phase-k work claims (groups of 32*kVL live entries) beyond the first
 };
 
 constexpr int kTrace = 48;  // phase timestamps per kernel (debug tracing)

@@ -92,9 +92,10 @@ __device__ __forceinline__ void wq_push(int32_t *q, int32_t &qn, int32_t *list, 
     if (qn > kWQ - 32) wq_flush(q, qn, list, counter);
 }
 
-// x is free after round k's commits
-__device__ __forceinline__ bool free_after(int32_t x, const int32_t *M, const int32_t *Pk) {
-    if (ldcg(M + x) != kFree) return false;
+// x is free after round k's commits.  M is not read: a vertex matched in any
+// round <= k has P_k[P_k[x]] == x (matched vertices keep their partner in both proposal
+// buffers), and a dead vertex (P = NONE) never neighbours a vertex that still rescans.
+__device__ __forceinline__ bool free_after(int32_t x, const int32_t *Pk) {
     const int32_t px = ldcg(Pk + x);
     return !(px >= 0 && ldcg(Pk + px) == x);
 }
@@ -280,7 +281,7 @@ __device__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool 
         unsigned long long key = 0;
         for (int32_t j = s + threadIdx.x; j < e; j += kNT) {
             const int32_t x = __ldg(a.adjncy + j);
-            if (!check || free_after(x, a.M, Pk)) key = umax64(key, pack_key(__ldg(a.adjwgt + j), x));
+            if (!check || free_after(x, Pk)) key = umax64(key, pack_key(__ldg(a.adjwgt + j), x));
         }
         key = group_max64<32>(key);
         if (lane == 0) sm.red[wib] = key;
@@ -312,18 +313,16 @@ __device__ __forceinline__ void rescan_thread(const MatchArgs &a, const int32_t 
                                               unsigned long long &key, unsigned long long &key2) {
     key = key2 = 0;
     for (int32_t j0 = s; j0 < e; j0 += 8) {
-        int32_t x[8], m[8], px[8], pp[8];
+        int32_t x[8], px[8], pp[8];
 #pragma unroll
         for (int b = 0; b < 8; ++b) x[b] = (j0 + b < e) ? __ldg(a.adjncy + j0 + b) : -1;
 #pragma unroll
-        for (int b = 0; b < 8; ++b) m[b] = (x[b] >= 0) ? ldcg(a.M + x[b]) : 0;
-#pragma unroll
-        for (int b = 0; b < 8; ++b) px[b] = (x[b] >= 0 && m[b] == kFree) ? ldcg(Pk + x[b]) : -1;
+        for (int b = 0; b < 8; ++b) px[b] = (x[b] >= 0) ? ldcg(Pk + x[b]) : -1;
 #pragma unroll
         for (int b = 0; b < 8; ++b) pp[b] = (px[b] >= 0) ? ldcg(Pk + px[b]) : -1;
 #pragma unroll
         for (int b = 0; b < 8; ++b)
-            if (x[b] >= 0 && m[b] == kFree && pp[b] != x[b]) top2_add(key, key2, pack_key(__ldg(a.adjwgt + j0 + b), x[b]));
+            if (x[b] >= 0 && pp[b] != x[b]) top2_add(key, key2, pack_key(__ldg(a.adjwgt + j0 + b), x[b]));
     }
 }
 
@@ -341,10 +340,23 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
     const int lane = threadIdx.x & 31;
     int32_t *q = reinterpret_cast<int32_t *>(&sm.adj[0][0]) + (threadIdx.x >> 5) * kWQ;  // phase 0 is over
     int32_t qn = 0;
-    // warp-uniform grid-stride loop over groups of 32*kVL entries: warps never wait for their CTA
-    const long long wstride = (long long)gridDim.x * kNT * kVL;
-    for (long long base = ((long long)blockIdx.x * kNT + (threadIdx.x & ~31)) * kVL; base < len; base += wstride) {
-        int32_t u[kVL], p[kVL], s2[kVL], qq[kVL], rr[kVL], ms[kVL], ps[kVL], pps[kVL];
+    // warps claim groups of 32*kVL live entries: the first group by warp id, the rest from a
+    // per-round counter, claimed one group ahead so the atomic's latency overlaps the work.
+    // Warps whose groups need rescans simply claim fewer groups: no barrier tail.
+    const long long ngroups = ((long long)len + 32 * kVL - 1) / (32 * kVL);
+    const long long nwarps = (long long)gridDim.x * (kNT / 32);
+    int32_t *claim = &a.ctl->slot[k & 3].claim;
+    auto claim_next = [&](bool more) -> long long {  // warp-uniform; lane 0 does the atomic
+        long long c = ngroups;
+        if (lane == 0 && more) c = nwarps + atomicAdd(claim, 1);
+        return __shfl_sync(0xffffffffu, c, 0);
+    };
+    long long g = (long long)blockIdx.x * (kNT / 32) + (threadIdx.x >> 5);
+    long long gn = claim_next(g < ngroups);
+    while (g < ngroups) {
+        const long long base = g * 32 * kVL;
+        const long long gafter = claim_next(gn < ngroups);
+        int32_t u[kVL], p[kVL], s2[kVL], qq[kVL], rr[kVL], ps[kVL], pps[kVL];
         // level 1: the vertices; level 2: P_k[u] and the cached second candidate S[u]
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
@@ -356,12 +368,11 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
             p[i] = u[i] >= 0 ? ldcg(Pk + u[i]) : kNone;
             s2[i] = (u[i] >= 0 && p[i] != kNone) ? ldcg(a.S + u[i]) : kNone;
         }
-        // level 3: P_k[p] and the freedom test of the cached candidate (M, P_k)
+        // level 3: P_k[p] and P_k[s2] (freedom test of the cached candidate, P only)
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
             qq[i] = p[i] != kNone ? ldcg(Pk + p[i]) : kNone;
-            ms[i] = s2[i] != kNone ? ldcg(a.M + s2[i]) : 0;
-            ps[i] = (s2[i] != kNone && ms[i] == kFree) ? ldcg(Pk + s2[i]) : -1;
+            ps[i] = s2[i] != kNone ? ldcg(Pk + s2[i]) : -1;
         }
         // level 4: P_k[q] (did p match q?) and P_k[P_k[s2]]
 #pragma unroll
@@ -382,7 +393,7 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
                 u[i] = -1;  // done
             } else if (rr[i] != p[i]) {
                 Pn[u[i]] = p[i];  // p is still free: still the heaviest free neighbour
-            } else if (s2[i] != kNone && ms[i] == kFree && pps[i] != s2[i]) {
+            } else if (s2[i] != kNone && pps[i] != s2[i]) {
                 // the cached second-heaviest neighbour of u's last scan is still free: it is
                 // now u's heaviest free neighbour (the free set only shrinks)
                 Pn[u[i]] = s2[i];
@@ -425,7 +436,7 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
                 unsigned long long key = 0, key2 = 0;
                 for (int32_t j = su + lane; j < eu; j += 32) {
                     const int32_t x = __ldg(a.adjncy + j);
-                    if (free_after(x, a.M, Pk)) top2_add(key, key2, pack_key(__ldg(a.adjwgt + j), x));
+                    if (free_after(x, Pk)) top2_add(key, key2, pack_key(__ldg(a.adjwgt + j), x));
                 }
                 group_top2<32>(key, key2);
                 if (lane == src) {
@@ -439,6 +450,8 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
             }
             wq_push(q, qn, Ln, &next->live, live[i], u[i]);
         }
+        g = gn;
+        gn = gafter;
     }
     wq_flush(q, qn, Ln, &next->live);
 }
@@ -481,6 +494,7 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
             z->live = 0;
             z->nhub = 0;
             z->matches = 0;
+            z->claim = 0;
         }
         const int32_t len = (k == 1) ? n : *(volatile int32_t *)&ctl->slot[k & 3].live;
         int32_t made = 0;

@@ -50,10 +50,14 @@ def simulate_match(adjp, adjncy, adjwgt, seed=0, max_rounds=0, use_cache=True):
         nxt = []
 
         def free_after(x):
-            if M[x] != FREE:
-                return False
+            # P-only test: a vertex matched in any round <= k has
+            # P_k[P_k[x]] == x (matched vertices keep their partner in both buffers); a dead
+            # vertex (P = NONE) never neighbours a vertex that still rescans.  M is not read.
             px = Pk[x]
-            return not (px >= 0 and Pk[px] == x)
+            free = not (px >= 0 and Pk[px] == x)
+            # the test the M array would give (M written immediately in this simulation)
+            assert free == (M[x] == FREE and not (px >= 0 and Pk[px] == x)), (k, x)
+            return free
 
         for u in rng.permutation(live) if live else []:
             p = Pk[u]
