@@ -30,6 +30,7 @@
 //  Rows come out sorted by coarse id (R10) with repeated coarse neighbours summed (R8) and
 //  the collapsed edge dropped (R9).
 #include <cuda_runtime.h>
+#include <stdlib.h>
 
 #include "device_util.cuh"
 #include "gp_internal.cuh"
@@ -47,6 +48,9 @@ constexpr int kWarpNet = 64;     // one-warp register merge capacity
 constexpr int kBuf = 4096;       // shared u64 buffer (warp regions of 2*kWB / C1h rows / C2b)
 constexpr unsigned long long kMaxKey = ~0ull;
 
+// CTAs taking part in this launch: min(grid, ceil(max(n, nnz/4) / vpc)) (see match.cu)
+__shared__ int g_cact;
+
 struct ContractArgs {
     const SizeRec *in;  // device: sizes + stop flag of this level's graph
     const int32_t *adjp, *adjncy, *adjwgt, *vwgt;
@@ -63,6 +67,7 @@ struct ContractArgs {
     int32_t apply_leftover;
     int32_t threshold, stall_pct, level, max_levels;
     LevelReport *report;  // mapped host memory (may be null)
+    int32_t vpc;          // vertices (or 4 arcs) per active CTA
 };
 
 struct ContractSmem {
@@ -415,7 +420,7 @@ __device__ __forceinline__ int32_t warp_excl(int32_t v, int32_t &total) {
 // ---------------------------------------------------------------------------------------
 __device__ void phase_c1a(const ContractArgs &a, int32_t n, int nt1, int T1) {
     const int lane = threadIdx.x & 31;
-    const int gw = blockIdx.x * kCW + (threadIdx.x >> 5), nw = gridDim.x * kCW;
+    const int gw = blockIdx.x * kCW + (threadIdx.x >> 5), nw = g_cact * kCW;
     for (int wt = gw; wt < nt1; wt += nw) {
         const long long base = (long long)wt * kVW;
         int32_t cnt = 0, ubs = 0;
@@ -557,7 +562,7 @@ __device__ __forceinline__ void gather_row(const ContractArgs &a, int32_t c, int
 // C1h: rows with ub > kWB, one CTA each; result compacted at gkeys[off[c]], count cnt[c]
 // ---------------------------------------------------------------------------------------
 __device__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
-    for (int i = blockIdx.x; i < nh; i += gridDim.x) {
+    for (int i = blockIdx.x; i < nh; i += g_cact) {
         const int32_t c = a.huge[i];
         const int32_t o0 = __ldcg(a.off + c);
         const int32_t ub = __ldcg(a.off + c + 1) - o0;
@@ -596,11 +601,13 @@ __device__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
 // ---------------------------------------------------------------------------------------
 __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntiles2, int T2, int32_t tb) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    const int gw = blockIdx.x * kCW + wib, nw = gridDim.x * kCW;
+    const int gw = blockIdx.x * kCW + wib, nw = g_cact * kCW;
     unsigned long long *wb = sm.buf + wib * 2 * kWB;  // this warp's slots (2*kWB entries)
     (void)gw;
     (void)nw;
-    // warp tiles are claimed dynamically (balances the tail of the phase)
+    // warp tiles are claimed dynamically from one global counter: the merge cost of a tile
+    // varies (row mix, C1h copies), and a static split per CTA leaves barrier tails
+    // (measured: +30 % on the phase at small levels)
     for (int wt = (lane == 0) ? (int)atomicAdd(&a.ctl->tile_ctr, 1u) : 0;;) {
         wt = __shfl_sync(0xffffffffu, wt, 0);
         if (wt >= ntiles2) break;
@@ -842,40 +849,48 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
     }
     const int32_t n = in->n;
     const int32_t nnz = in->nnz;
+    {
+        const long long work = (long long)n > (long long)nnz / 4 ? (long long)n : (long long)nnz / 4;
+        const long long want = (work + a.vpc - 1) / a.vpc;
+        const int nact = (int)(want < 1 ? 1 : (want < (long long)gridDim.x ? want : (long long)gridDim.x));
+        if ((int)blockIdx.x >= nact) return;  // retired: this level is too small for it
+        if (threadIdx.x == 0) g_cact = nact;
+        __syncthreads();
+    }
     unsigned bar_epoch = 0;  // grid barriers passed (thread 0)
     const int nt1 = (n + kVW - 1) / kVW;
-    const int T1 = (nt1 + gridDim.x - 1) / gridDim.x;            // C1b tiles per CTA
+    const int T1 = (nt1 + g_cact - 1) / g_cact;            // C1b tiles per CTA
     // C2 warp-tile budget: kWB, halved (down to 32) while there are < 4 tiles per warp
     int32_t tb = kWB;
-    while (tb > 32 && (long long)nnz < 4LL * tb * gridDim.x * kCW) tb >>= 1;
+    while (tb > 32 && (long long)nnz < 4LL * tb * g_cact * kCW) tb >>= 1;
     const int32_t ntiles2 = nnz > 0 ? (nnz + tb - 1) / tb : 0;
-    const int T2 = (ntiles2 + gridDim.x - 1) / gridDim.x;        // C2b tiles per CTA
+    const int T2 = (ntiles2 + g_cact - 1) / g_cact;        // C2b tiles per CTA
     trace_mark(ctl->trace, 0);
     if (n > 0) {
         phase_c1a(a, n, nt1, T1);
         trace_mark(ctl->trace, 1);
-        grid_barrier(ctl->bar, bar_epoch);
+        grid_barrier(ctl->bar, bar_epoch, g_cact);
         trace_mark(ctl->trace, 2);
         phase_c1b(a, sm, n, nt1, T1, ntiles2, tb);
         trace_mark(ctl->trace, 3);
-        grid_barrier(ctl->bar, bar_epoch);
+        grid_barrier(ctl->bar, bar_epoch, g_cact);
     }
     trace_mark(ctl->trace, 4);
     const int32_t nc = *(volatile int32_t *)&ctl->n_coarse;
     const int32_t nh = *(volatile int32_t *)&ctl->n_huge;
     if (nh > 0) {
         phase_c1h(a, sm, nh);
-        grid_barrier(ctl->bar, bar_epoch);
+        grid_barrier(ctl->bar, bar_epoch, g_cact);
     }
     trace_mark(ctl->trace, 5);
     if (ntiles2 > 0) {
         phase_c2a(a, sm, ntiles2, T2, tb);
         trace_mark(ctl->trace, 6);
-        grid_barrier(ctl->bar, bar_epoch);
+        grid_barrier(ctl->bar, bar_epoch, g_cact);
         trace_mark(ctl->trace, 7);
         phase_c2b(a, sm, nc, ntiles2, T2);
     } else {  // no arcs: every coarse row is empty
-        for (long long c = (long long)blockIdx.x * kCNT + threadIdx.x; c <= nc; c += (long long)gridDim.x * kCNT)
+        for (long long c = (long long)blockIdx.x * kCNT + threadIdx.x; c <= nc; c += (long long)g_cact * kCNT)
             a.cadjp[c] = 0;
         if (blockIdx.x == 0 && threadIdx.x == 0) ctl->cnnz = 0;
     }
@@ -883,7 +898,7 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
     // the last CTA to finish publishes the coarse sizes and the stop decision
     __threadfence();
     __syncthreads();
-    if (threadIdx.x == 0) sm.last = atomicAdd(&ctl->blocks_done, 1u) == gridDim.x - 1;
+    if (threadIdx.x == 0) sm.last = atomicAdd(&ctl->blocks_done, 1u) == (unsigned)g_cact - 1;
     __syncthreads();
     if (sm.last && threadIdx.x == 0) {
         __threadfence();
@@ -914,6 +929,16 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
 // ---------------------------------------------------------------------------------------
 // host side
 // ---------------------------------------------------------------------------------------
+static int32_t contract_vpc() {
+    static int32_t v = -1;
+    if (v < 0) {
+        const char *e = getenv("GP_CONTRACT_VPC");  // tuning knob (results never depend on it)
+        v = e ? atoi(e) : 64;
+        if (v < 1) v = 1;
+    }
+    return v;
+}
+
 int contract_grid(Ctx *ctx) {
     static int per_sm = -1;
     if (per_sm < 0) {
@@ -963,6 +988,7 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
     a.level = prm.level;
     a.max_levels = prm.max_levels;
     a.report = report;
+    a.vpc = contract_vpc();
     void *args[] = {&a};
     LaunchScope ls(ctx, GP_K_CONTRACT);
     GP_CUDA(cudaLaunchCooperativeKernel((const void *)k_contract_level, dim3(contract_grid(ctx)), dim3(kCNT), args,

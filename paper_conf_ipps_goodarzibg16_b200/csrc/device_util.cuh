@@ -199,14 +199,15 @@ __device__ __forceinline__ void red_release_add_u32(unsigned *p, unsigned v) {
 }
 
 // bar[0] counts arrivals and only grows within a launch (zeroed before the launch); the
-// k-th barrier of the launch completes when it reaches k * gridDim.x.  The release-add
+// k-th barrier of the launch completes when it reaches k * nblocks (the CTAs that take part:
+// a level kernel retires the CTAs its level is too small to use).  The release-add
 // publishes the CTA's writes (bar.sync orders them before thread 0's release; release is
 // cumulative), the acquire poll makes every other CTA's writes visible after it.
-__device__ __forceinline__ void grid_barrier(unsigned *bar, unsigned &epoch) {
+__device__ __forceinline__ void grid_barrier(unsigned *bar, unsigned &epoch, unsigned nblocks) {
     __syncthreads();
     if (threadIdx.x == 0) {
         ++epoch;
-        const unsigned target = epoch * gridDim.x;
+        const unsigned target = epoch * nblocks;
         red_release_add_u32(bar, 1u);
         const long long guard = spin_start();
         while ((int)(ld_acquire_u32(bar) - target) < 0) {

@@ -27,6 +27,7 @@
 //  * Worklists are appended with one atomic per CTA (block-aggregated), round counters
 //    live in a 4-slot ring so no counter is reset while another CTA may still read it.
 #include <cuda_runtime.h>
+#include <stdlib.h>
 
 #include "device_util.cuh"
 #include "gp_internal.cuh"
@@ -39,6 +40,11 @@ constexpr int kStages = 3;          // TMA pipeline depth of phase 0
 constexpr int kMaxVch = 1024;       // vertices per phase-0 chunk (adjp slice staged too)
 constexpr int kThreadDeg = 32;      // phase-k rescans up to this many arcs: one thread
 constexpr int kHubDeg = 4096;       // rows longer than this: one CTA each (hub phase)
+
+// CTAs taking part in this launch: min(grid, ceil(n / vpc)).  The host launches the full
+// persistent grid before the level's size is known; the level's kernel retires the CTAs a
+// small level cannot use, which makes its grid barriers and claim counters cheaper.
+__shared__ int g_nact;
 
 struct MatchArgs {
     const SizeRec *in;  // device: sizes + stop flag of this level's graph
@@ -53,6 +59,7 @@ struct MatchArgs {
     int32_t leftover;
     int32_t G;    // lanes per vertex in phase 0 (1, 2, 4, 8 or 16)
     int32_t vch;  // vertices per phase-0 chunk (about 80 % of a stage at the average degree)
+    int32_t vpc;  // vertices per active CTA (small levels run on fewer CTAs)
 };
 
 struct MatchSmem {
@@ -64,7 +71,9 @@ struct MatchSmem {
     int32_t fits[kStages];  // 1 staged, 0 fallback
     long long cid[kStages]; // chunk staged in the stage (claimed dynamically; >= nchunks: none)
     int32_t scratch[40];
+    int32_t claim;  // phase-k group claims of this CTA
     unsigned long long red[kNT / 32];
+    unsigned long long cnt3[3][kNT / 32];
 };
 
 __device__ __forceinline__ int32_t ldcg(const int32_t *p) { return __ldcg(p); }
@@ -275,7 +284,7 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
 __device__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool check, const int32_t *Pk,
                           int32_t *Pn, int32_t *Lnext, int32_t *live_next, unsigned long long &scanned) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    for (int i = blockIdx.x; i < nhub; i += gridDim.x) {
+    for (int i = blockIdx.x; i < nhub; i += g_nact) {
         const int32_t u = a.H[i];
         const int32_t s = __ldg(a.adjp + u), e = __ldg(a.adjp + u + 1);
         unsigned long long key = 0;
@@ -337,25 +346,24 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
     const int32_t *Lk = a.L[k & 1];
     int32_t *Ln = a.L[(k + 1) & 1];
     RoundSlot *next = &a.ctl->slot[(k + 1) & 3];
-    const int lane = threadIdx.x & 31;
-    int32_t *q = reinterpret_cast<int32_t *>(&sm.adj[0][0]) + (threadIdx.x >> 5) * kWQ;  // phase 0 is over
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    int32_t *q = reinterpret_cast<int32_t *>(&sm.adj[0][0]) + wib * kWQ;  // phase 0 is over
     int32_t qn = 0;
-    // warps claim groups of 32*kVL live entries: the first group by warp id, the rest from a
-    // per-round counter, claimed one group ahead so the atomic's latency overlaps the work.
-    // Warps whose groups need rescans simply claim fewer groups: no barrier tail.
+    // CTA b owns the contiguous groups [g_lo, g_hi) of 32*kVL live entries; its warps claim
+    // them from a shared-memory counter.  No global atomics on a shared address: thousands
+    // of warps hitting one L2 atomic unit serialise (~0.5 ns each), which dominated the
+    // rounds of small levels.
     const long long ngroups = ((long long)len + 32 * kVL - 1) / (32 * kVL);
-    const long long nwarps = (long long)gridDim.x * (kNT / 32);
-    int32_t *claim = &a.ctl->slot[k & 3].claim;
-    auto claim_next = [&](bool more) -> long long {  // warp-uniform; lane 0 does the atomic
-        long long c = ngroups;
-        if (lane == 0 && more) c = nwarps + atomicAdd(claim, 1);
-        return __shfl_sync(0xffffffffu, c, 0);
+    const long long g_lo = ngroups * blockIdx.x / g_nact, g_hi = ngroups * (blockIdx.x + 1) / g_nact;
+    if (threadIdx.x == 0) sm.claim = 0;
+    __syncthreads();
+    auto claim_next = [&]() -> long long {  // warp-uniform
+        int c = 0;
+        if (lane == 0) c = atomicAdd(&sm.claim, 1);
+        return g_lo + __shfl_sync(0xffffffffu, c, 0);
     };
-    long long g = (long long)blockIdx.x * (kNT / 32) + (threadIdx.x >> 5);
-    long long gn = claim_next(g < ngroups);
-    while (g < ngroups) {
+    for (long long g = claim_next(); g < g_hi; g = claim_next()) {
         const long long base = g * 32 * kVL;
-        const long long gafter = claim_next(gn < ngroups);
         int32_t u[kVL], p[kVL], s2[kVL], qq[kVL], rr[kVL], ps[kVL], pps[kVL];
         // level 1: the vertices; level 2: P_k[u] and the cached second candidate S[u]
 #pragma unroll
@@ -450,16 +458,30 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
             }
             wq_push(q, qn, Ln, &next->live, live[i], u[i]);
         }
-        g = gn;
-        gn = gafter;
     }
-    wq_flush(q, qn, Ln, &next->live);
+    // CTA-aggregated final flush: one global atomic per CTA
+    if (lane == 0) sm.scratch[wib] = qn;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int32_t tot = 0;
+        for (int w = 0; w < kNT / 32; ++w) {
+            const int32_t c = sm.scratch[w];
+            sm.scratch[w] = tot;
+            tot += c;
+        }
+        sm.scratch[kNT / 32] = tot ? atomicAdd(&next->live, tot) : 0;
+    }
+    __syncthreads();
+    {
+        const int32_t base = sm.scratch[kNT / 32] + sm.scratch[wib];
+        for (int i = lane; i < qn; i += 32) Ln[base + i] = q[i];
+    }
 }
 
 __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, unsigned long long &scanned,
                         unsigned long long &rows, unsigned long long &visits, int32_t &made) {
     (void)n;
-    if ((long long)len >= 4LL * gridDim.x * kNT) phase_k_impl<4>(a, sm, k, len, scanned, rows, visits, made);
+    if ((long long)len >= 4LL * g_nact * kNT) phase_k_impl<4>(a, sm, k, len, scanned, rows, visits, made);
     else phase_k_impl<1>(a, sm, k, len, scanned, rows, visits, made);
 }
 
@@ -471,19 +493,26 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
     if (in->stop) return;  // an earlier level ended the coarsening: nothing to do
     const int32_t n = in->n;
     if (n <= 0) return;
+    {
+        const long long want = ((long long)n + a.vpc - 1) / a.vpc;
+        const int nact = (int)(want < 1 ? 1 : (want < (long long)gridDim.x ? want : (long long)gridDim.x));
+        if ((int)blockIdx.x >= nact) return;  // retired: this level is too small for it
+        if (threadIdx.x == 0) g_nact = nact;
+        __syncthreads();
+    }
     unsigned long long scanned = 0, rows = 0, visits = 0;
     unsigned bar_epoch = 0;  // grid barriers passed (thread 0)
     int tr = 0;
     trace_mark(ctl->trace, tr++);
     phase0(a, sm, n, scanned);
     trace_mark(ctl->trace, tr++);
-    grid_barrier(ctl->bar, bar_epoch);
+    grid_barrier(ctl->bar, bar_epoch, g_nact);
     trace_mark(ctl->trace, tr++);
     {
         const int32_t nh = *(volatile int32_t *)&ctl->slot[1].nhub;
         if (nh > 0) {
             hub_phase(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned);
-            grid_barrier(ctl->bar, bar_epoch);
+            grid_barrier(ctl->bar, bar_epoch, g_nact);
         }
     }
     int32_t rounds = 0, maximal = 0;
@@ -499,16 +528,16 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
         const int32_t len = (k == 1) ? n : *(volatile int32_t *)&ctl->slot[k & 3].live;
         int32_t made = 0;
         phase_k(a, sm, n, k, len, scanned, rows, visits, made);
-        made = warp_sum(made);
-        if ((threadIdx.x & 31) == 0 && made) atomicAdd(&ctl->slot[k & 3].matches, made);
+        // any match this round: one flag store per CTA (only "> 0" is used)
+        if (__syncthreads_or(made > 0) && threadIdx.x == 0) *(volatile int32_t *)&ctl->slot[k & 3].matches = 1;
         trace_mark(ctl->trace, tr++);
-        grid_barrier(ctl->bar, bar_epoch);
+        grid_barrier(ctl->bar, bar_epoch, g_nact);
         trace_mark(ctl->trace, tr++);
         const int32_t nh = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].nhub;
         if (nh > 0) {
             hub_phase(a, sm, nh, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1], &ctl->slot[(k + 1) & 3].live,
                       scanned);
-            grid_barrier(ctl->bar, bar_epoch);
+            grid_barrier(ctl->bar, bar_epoch, g_nact);
         }
         if (*(volatile int32_t *)&ctl->slot[k & 3].matches > 0) ++rounds;
         const int32_t live = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].live;
@@ -520,16 +549,22 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
     }
     trace_mark(ctl->trace, tr++);
     if (a.leftover) {
-        for (long long u = (long long)blockIdx.x * kNT + threadIdx.x; u < n; u += (long long)gridDim.x * kNT)
+        for (long long u = (long long)blockIdx.x * kNT + threadIdx.x; u < n; u += (long long)g_nact * kNT)
             if (a.M[u] == kFree) a.M[u] = (int32_t)u;
     }
     scanned = warp_sum64(scanned);
     rows = warp_sum64(rows);
     visits = warp_sum64(visits);
     if ((threadIdx.x & 31) == 0) {
-        if (scanned) atomicAdd(&ctl->arcs_scanned, scanned);
-        if (rows) atomicAdd(&ctl->rows_scanned, rows);
-        if (visits) atomicAdd(&ctl->live_visits, visits);
+        sm.cnt3[0][threadIdx.x >> 5] = scanned;
+        sm.cnt3[1][threadIdx.x >> 5] = rows;
+        sm.cnt3[2][threadIdx.x >> 5] = visits;
+    }
+    __syncthreads();
+    if (threadIdx.x < 3) {  // one atomic per CTA and counter
+        unsigned long long t = 0;
+        for (int w = 0; w < kNT / 32; ++w) t += sm.cnt3[threadIdx.x][w];
+        if (t) atomicAdd(threadIdx.x == 0 ? &ctl->arcs_scanned : threadIdx.x == 1 ? &ctl->rows_scanned : &ctl->live_visits, t);
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         ctl->rounds = rounds;
@@ -547,6 +582,16 @@ static int choose_group(double avg_deg) {
     if (avg_deg <= 24.0) return 2;
     if (avg_deg <= 48.0) return 4;
     return 8;
+}
+
+static int32_t match_vpc() {
+    static int32_t v = -1;
+    if (v < 0) {
+        const char *e = getenv("GP_MATCH_VPC");  // tuning knob (results never depend on it)
+        v = e ? atoi(e) : 128;
+        if (v < 1) v = 1;
+    }
+    return v;
 }
 
 int match_grid(Ctx *ctx) {
@@ -578,6 +623,7 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     a.max_rounds = max_rounds;
     a.leftover = leftover ? 1 : 0;
     a.G = choose_group(avg_deg_hint);
+    a.vpc = match_vpc();
     {
         // vertices per chunk: ~80 % of a stage at the average degree, a multiple of the
         // number of vertex groups (kNT / G) so that no group pass runs mostly idle
