@@ -157,13 +157,63 @@ typedef struct {
     const gp_vid *d_match;   /* device int32[n]                                            */
     const gp_vid *d_cmap;    /* device int32[n]                                            */
     gp_graph coarse;         /* borrowed: do not gp_free                                   */
+    /* sharded hierarchies (gp_ctx_create_dist): n, nnz, n_coarse, cnnz, rounds are GLOBAL;
+     * d_match / d_cmap / coarse are this rank's piece: the fine vertices
+     * [v_begin, v_begin + n_local) and the coarse vertices [cv_begin, cv_begin + n_coarse_local)
+     * (coarse ids stay globally contiguous per rank and equal to the 1-GPU numbering).
+     * Loopback contexts hold every piece: those three are NULL, use the download calls.
+     * Single GPU: v_begin = cv_begin = 0, n_local = n, n_coarse_local = n_coarse.            */
+    gp_vid v_begin, n_local, cv_begin, n_coarse_local;
 } gp_level;
 
 gp_status gp_hier_num_levels(gp_hier h, int32_t *out);
 gp_status gp_hier_level(gp_hier h, int32_t i, gp_level *out);
 
-/* Copy a level's M and CM to caller-owned host buffers (either may be NULL).  Synchronous. */
+/* Copy a level's M and CM to caller-owned host buffers (either may be NULL).  Synchronous.
+ * Sharded hierarchies: this rank's piece (n_local entries); loopback: all n entries. */
 gp_status gp_hier_download_level(gp_hier h, int32_t i, gp_vid *h_match, gp_vid *h_cmap);
+
+/* Copy a level's coarse graph to caller-owned host buffers (any may be NULL): adjp
+ * [n_coarse_local + 1], adjncy / adjwgt [its arcs], vwgt [n_coarse_local]; column ids are
+ * global coarse ids.  Loopback: the whole coarse graph (pieces concatenated).  Synchronous.
+ * *n_out / *nnz_out (nullable) receive the row and arc counts of what is copied. */
+gp_status gp_hier_download_coarse(gp_hier h, int32_t i, gp_vid *h_adjp, gp_vid *h_adjncy, gp_wgt *h_adjwgt,
+                                  gp_wgt *h_vwgt, gp_vid *n_out, gp_vid *nnz_out);
+
+/* ---- sharded coarsening over several GPUs -------------------
+ * Vertex ranges are sharded over the ranks of one node (one process per GPU).  Each rank
+ * owns the contiguous global ids [v_begin, v_end) and holds their CSR rows with GLOBAL
+ * column ids.  Every handshake round ends with an all-gather of the boundary proposals
+ * (a vertex with a neighbour on another rank publishes (v, P[v], P[P[v]] when P[v] is its
+ * own)); per level the leader counts are all-gathered into the rank offsets of the coarse
+ * ids (the north_star's "allreduce'd prefix"), the boundary CM values are all-gathered and
+ * the rows of non-leader partners are sent to their leader's rank, already mapped to coarse
+ * ids.  All results are bit-identical to the 1-GPU path for any number of ranks.
+ *
+ * gp_nccl_unique_id   rank 0 creates the NCCL id (128 bytes) and broadcasts it (e.g. with
+ *                     torch.distributed); GP_ERR_NCCL when libnccl.so.2 cannot be loaded.
+ * gp_ctx_create_dist  collective over the nranks processes; `device` is this rank's GPU.
+ * gp_ctx_create_loopback  one process, one GPU, `nranks` simulated ranks: every collective
+ *                     becomes device-to-device copies between the ranks' private buffers
+ *                     (the same kernels and the same exchange layout as NCCL).  For tests and
+ *                     for single-GPU runs of the sharded protocol.
+ * gp_graph_create_dist  (NCCL contexts) this rank's shard: n_global vertices in total, rows
+ *                     v_begin..v_end-1 given by adjp_local[v_end - v_begin + 1] (local offsets,
+ *                     adjp_local[0] = 0), adjncy/adjwgt (global ids), vwgt.  Collective: the
+ *                     shards must tile [0, n_global) in rank order.  Flags as gp_graph_create.
+ *                     On a loopback context, gp_graph_create makes the whole graph and
+ *                     gp_coarsen_to splits it into nranks equal vertex ranges.
+ * gp_coarsen_to on a sharded graph (or any graph of a loopback context) runs the sharded
+ *                     driver; collective. */
+gp_status gp_nccl_unique_id(void *out_128_bytes);
+gp_status gp_ctx_create_dist(int device, void *cuda_stream, const void *nccl_unique_id, int rank, int nranks,
+                             gp_ctx *out);
+gp_status gp_ctx_create_loopback(int device, void *cuda_stream, int nranks, gp_ctx *out);
+/* rank / nranks of a context: single GPU 0 / 1; NCCL rank / nranks; loopback -1 / nranks. */
+gp_status gp_ctx_dist_info(gp_ctx ctx, int32_t *rank, int32_t *nranks);
+gp_status gp_graph_create_dist(gp_ctx ctx, gp_vid n_global, gp_vid v_begin, gp_vid v_end, const gp_vid *adjp_local,
+                               const gp_vid *adjncy, const gp_wgt *adjwgt, const gp_wgt *vwgt, uint32_t flags,
+                               gp_graph *out);
 
 /* Release any gp_ctx / gp_graph / gp_hier (handles are tagged); NULL is a no-op.
  * Levels borrowed from a hierarchy are released with the hierarchy. */

@@ -41,7 +41,7 @@ constexpr int kCNT = 256;        // threads per CTA (4 co-resident CTAs per SM)
 constexpr int kCW = kCNT / 32;   // warps per CTA
 constexpr int kCItems = 8;       // vertices per lane of a C1 warp tile
 constexpr int kVW = 32 * kCItems;  // 256 vertices per C1 warp tile
-constexpr int kWB = 256;         // C2 warp-tile budget (upper-bound entries)
+constexpr int kWB = kContractTileBudget;  // C2 warp-tile budget (upper-bound entries)
 constexpr int kCtaRow = 4096;    // C1h: rows up to this bound are merged in shared memory
 constexpr int kNet = 16;         // one-thread merge capacity
 constexpr int kWarpNet = 64;     // one-warp register merge capacity
@@ -68,6 +68,11 @@ struct ContractArgs {
     int32_t threshold, stall_pct, level, max_levels;
     LevelReport *report;  // mapped host memory (may be null)
     int32_t vpc;          // vertices (or 4 arcs) per active CTA
+    // sharded levels (dist.cu): C1 ran as separate kernels (seg, off, cvwgt, CM, tile starts,
+    // huge rows and ctl->n_coarse / n_huge are given); coarse row c has the global id
+    // cbase + c; adjncy/adjwgt hold the local rows followed by the shipped partner rows; the
+    // host takes the stop decision.  Single GPU: dist = 0, cbase = 0.
+    int32_t dist, cbase, tb_fixed, nnz_ub;
 };
 
 struct ContractSmem {
@@ -553,7 +558,7 @@ __device__ __forceinline__ void gather_row(const ContractArgs &a, int32_t c, int
         const int32_t s = side ? sg.z : sg.x, e = s + (side ? sg.w : sg.y);
         for (int32_t j = s + tid; j < e; j += nthr) {
             const int32_t cx = __ldcg(a.CM + __ldcs(a.adjncy + j));
-            if (cx != c) dst[claim()] = ckey(cx, __ldcs(a.adjwgt + j));  // drop the collapsed edge (R9)
+            if (cx != c + a.cbase) dst[claim()] = ckey(cx, __ldcs(a.adjwgt + j));  // drop the collapsed edge (R9)
         }
     }
 }
@@ -670,7 +675,7 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
 #pragma unroll
                     for (int k = 0; k < kB; ++k)
                         if (jj[k] >= 0)  // collapsed edge dropped (R9)
-                            wb[b0 + k * 32 + lane] = (cx[k] != rc[k]) ? ckey(cx[k], w[k]) : kMaxKey;
+                            wb[b0 + k * 32 + lane] = (cx[k] != rc[k] + a.cbase) ? ckey(cx[k], w[k]) : kMaxKey;
                 }
                 __syncwarp();
             }
@@ -848,7 +853,11 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
         return;
     }
     const int32_t n = in->n;
-    const int32_t nnz = in->nnz;
+    // load the volatile size first: a conditional "a.dist ? a.nnz_ub : in->nnz" compiles to
+    // ONE load from a selected address, and a generic load of a __grid_constant__ parameter's
+    // address faults (observed with nvcc 12.9 / sm_100a)
+    const int32_t nnz_in = in->nnz;
+    const int32_t nnz = a.dist ? a.nnz_ub : nnz_in;
     {
         const long long work = (long long)n > (long long)nnz / 4 ? (long long)n : (long long)nnz / 4;
         const long long want = (work + a.vpc - 1) / a.vpc;
@@ -863,10 +872,11 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
     // C2 warp-tile budget: kWB, halved (down to 32) while there are < 4 tiles per warp
     int32_t tb = kWB;
     while (tb > 32 && (long long)nnz < 4LL * tb * g_cact * kCW) tb >>= 1;
+    if (a.dist) tb = a.tb_fixed;
     const int32_t ntiles2 = nnz > 0 ? (nnz + tb - 1) / tb : 0;
     const int T2 = (ntiles2 + g_cact - 1) / g_cact;        // C2b tiles per CTA
     trace_mark(ctl->trace, 0);
-    if (n > 0) {
+    if (n > 0 && !a.dist) {
         phase_c1a(a, n, nt1, T1);
         trace_mark(ctl->trace, 1);
         grid_barrier(ctl->bar, bar_epoch, g_cact);
@@ -906,7 +916,8 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
         const int32_t cnnz = *((volatile int32_t *)&ctl->cnnz);
         // stop rule (P12.s30, P20.s30; R12, R13): stall first, then threshold, then levels
         int32_t reason = GP_STOP_NONE;
-        if (100LL * ncv > (long long)a.stall_pct * n) reason = GP_STOP_STALL;
+        if (a.dist) reason = GP_STOP_NONE;  // global decision on the host (dist.cu)
+        else if (100LL * ncv > (long long)a.stall_pct * n) reason = GP_STOP_STALL;
         else if (ncv <= a.threshold) reason = GP_STOP_THRESHOLD;
         else if (a.level + 1 >= a.max_levels) reason = GP_STOP_MAX_LEVELS;
         a.out->n = ncv;
@@ -989,6 +1000,10 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
     a.max_levels = prm.max_levels;
     a.report = report;
     a.vpc = contract_vpc();
+    a.dist = prm.dist;
+    a.cbase = prm.cbase;
+    a.tb_fixed = prm.tb;
+    a.nnz_ub = prm.nnz_ub;
     void *args[] = {&a};
     LaunchScope ls(ctx, GP_K_CONTRACT);
     GP_CUDA(cudaLaunchCooperativeKernel((const void *)k_contract_level, dim3(contract_grid(ctx)), dim3(kCNT), args,

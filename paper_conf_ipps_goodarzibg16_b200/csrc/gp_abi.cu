@@ -8,6 +8,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <vector>
 
 #include "gp_internal.cuh"
 
@@ -117,7 +118,7 @@ static void drain_events(Ctx *ctx) {
     ctx->pending.clear();
 }
 
-static void graph_release(Graph *g) {
+void graph_release(Graph *g) {
     if (!g) return;
     Ctx *ctx = g->ctx;
     dev_free(ctx, g->adjp);
@@ -129,12 +130,17 @@ static void graph_release(Graph *g) {
     delete g;
 }
 
-static void hier_release(Hier *h) {
+void hier_release(Hier *h) {
     if (!h) return;
     for (auto &l : h->levels) {
         dev_free(h->ctx, l.match);
         dev_free(h->ctx, l.cmap);
         graph_release(l.coarse);
+        for (auto &p : l.pieces) {
+            dev_free(h->ctx, p.M);
+            dev_free(h->ctx, p.CM);
+            graph_release(p.coarse);
+        }
     }
     dev_free(h->ctx, h->levdev);
     h->tag = 0;
@@ -142,7 +148,7 @@ static void hier_release(Hier *h) {
 }
 
 // graph arrays with 4 ints of padding (TMA bulk copies round ranges up to 16 bytes)
-static gp_status alloc_graph_arrays(Ctx *ctx, Graph *g, int32_t n_bound, int32_t nnz_bound, bool own_sizes) {
+gp_status alloc_graph_arrays(Ctx *ctx, Graph *g, int32_t n_bound, int32_t nnz_bound, bool own_sizes) {
     gp_status st = dev_alloc(ctx, (void **)&g->adjp, sizeof(int32_t) * ((size_t)n_bound + 4));
     if (st == GP_OK) st = dev_alloc(ctx, (void **)&g->vwgt, sizeof(int32_t) * ((size_t)n_bound + 4));
     if (st == GP_OK) st = dev_alloc(ctx, (void **)&g->adjncy, sizeof(int32_t) * ((size_t)nnz_bound + 4));
@@ -421,6 +427,10 @@ gp_status gp_match_level(gp_graph g, gp_vid *d_match, int32_t max_rounds, int32_
     }
     GP_TRY_BEGIN
     Ctx *ctx = g->ctx;
+    if (ctx->comm) {
+        set_error("gp_match_level: per-level calls are single-GPU; sharded graphs use gp_coarsen_to");
+        return GP_ERR_INVALID_ARG;
+    }
     if (g->n == 0) {
         if (rounds_out) *rounds_out = 0;
         return GP_OK;
@@ -459,6 +469,10 @@ gp_status gp_contract_level(gp_graph g, const gp_vid *d_match, gp_vid *d_cmap, g
     }
     GP_TRY_BEGIN
     Ctx *ctx = g->ctx;
+    if (ctx->comm) {
+        set_error("gp_contract_level: per-level calls are single-GPU; sharded graphs use gp_coarsen_to");
+        return GP_ERR_INVALID_ARG;
+    }
     LevelBufs lb;
     gp_status st = level_scratch(ctx, g->n, g->nnz, &lb);
     if (st != GP_OK) return st;
@@ -536,6 +550,7 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
     }
     GP_TRY_BEGIN
     Ctx *ctx = g->ctx;
+    if (ctx->comm) return dist_coarsen_to(g, opts, out);  // sharded path (dist.cu)
     const int32_t pct = opts->stall_ratio_pct ? opts->stall_ratio_pct : 95;
     int32_t max_levels = opts->max_levels ? opts->max_levels : 64;
     if (max_levels > ctx->max_reports) max_levels = ctx->max_reports;
@@ -713,6 +728,25 @@ gp_status gp_hier_level(gp_hier h, int32_t i, gp_level *out) {
     o.d_match = l.match;
     o.d_cmap = l.cmap;
     o.coarse = l.coarse;
+    o.v_begin = 0;
+    o.n_local = l.n;
+    o.cv_begin = 0;
+    o.n_coarse_local = l.n_coarse;
+    if (!l.pieces.empty()) {  // sharded level
+        o.d_match = nullptr;
+        o.d_cmap = nullptr;
+        o.coarse = nullptr;
+        if (l.pieces.size() == 1) {  // NCCL: this rank's piece
+            const DistPiece &p = l.pieces[0];
+            o.d_match = p.M + p.vbase;
+            o.d_cmap = p.CM + p.vbase;
+            o.coarse = p.coarse;
+            o.v_begin = p.vbase;
+            o.n_local = p.nloc;
+            o.cv_begin = p.coarse ? p.coarse->vbase : 0;
+            o.n_coarse_local = p.coarse ? p.coarse->n : 0;
+        }
+    }
     *out = o;
     return GP_OK;
 }
@@ -724,10 +758,165 @@ gp_status gp_hier_download_level(gp_hier h, int32_t i, gp_vid *h_match, gp_vid *
     }
     const Level &l = h->levels[i];
     cudaStream_t s = h->ctx->stream;
+    if (!l.pieces.empty()) {  // sharded: the pieces' owned slices, in rank order
+        size_t o = 0;
+        for (const DistPiece &p : l.pieces) {
+            if (h_match && p.nloc)
+                GP_CUDA(cudaMemcpyAsync(h_match + o, p.M + p.vbase, sizeof(int32_t) * (size_t)p.nloc,
+                                        cudaMemcpyDeviceToHost, s));
+            if (h_cmap && p.nloc)
+                GP_CUDA(cudaMemcpyAsync(h_cmap + o, p.CM + p.vbase, sizeof(int32_t) * (size_t)p.nloc,
+                                        cudaMemcpyDeviceToHost, s));
+            o += (size_t)p.nloc;
+        }
+        GP_CUDA(cudaStreamSynchronize(s));
+        return GP_OK;
+    }
     if (h_match && l.n) GP_CUDA(cudaMemcpyAsync(h_match, l.match, sizeof(int32_t) * (size_t)l.n, cudaMemcpyDeviceToHost, s));
     if (h_cmap && l.n) GP_CUDA(cudaMemcpyAsync(h_cmap, l.cmap, sizeof(int32_t) * (size_t)l.n, cudaMemcpyDeviceToHost, s));
     GP_CUDA(cudaStreamSynchronize(s));
     return GP_OK;
+}
+
+gp_status gp_hier_download_coarse(gp_hier h, int32_t i, gp_vid *h_adjp, gp_vid *h_adjncy, gp_wgt *h_adjwgt,
+                                  gp_wgt *h_vwgt, gp_vid *n_out, gp_vid *nnz_out) {
+    if (!tagged<Hier>(h, kTagHier) || i < 0 || i >= (int32_t)h->levels.size()) {
+        set_error("gp_hier_download_coarse: bad handle or level index");
+        return GP_ERR_INVALID_ARG;
+    }
+    GP_TRY_BEGIN
+    const Level &l = h->levels[i];
+    std::vector<const Graph *> parts;
+    if (l.pieces.empty()) parts.push_back(l.coarse);
+    else
+        for (const DistPiece &p : l.pieces) parts.push_back(p.coarse);
+    cudaStream_t s = h->ctx->stream;
+    int32_t rows = 0, arcs = 0;
+    for (const Graph *c : parts) {
+        if (!c) {
+            set_error("gp_hier_download_coarse: level has no coarse graph");
+            return GP_ERR_INTERNAL;
+        }
+        if (h_adjp) {
+            GP_CUDA(cudaMemcpyAsync(h_adjp + rows, c->adjp, sizeof(int32_t) * ((size_t)c->n + 1), cudaMemcpyDeviceToHost, s));
+        }
+        if (h_adjncy && c->nnz)
+            GP_CUDA(cudaMemcpyAsync(h_adjncy + arcs, c->adjncy, sizeof(int32_t) * (size_t)c->nnz, cudaMemcpyDeviceToHost, s));
+        if (h_adjwgt && c->nnz)
+            GP_CUDA(cudaMemcpyAsync(h_adjwgt + arcs, c->adjwgt, sizeof(int32_t) * (size_t)c->nnz, cudaMemcpyDeviceToHost, s));
+        if (h_vwgt && c->n)
+            GP_CUDA(cudaMemcpyAsync(h_vwgt + rows, c->vwgt, sizeof(int32_t) * (size_t)c->n, cudaMemcpyDeviceToHost, s));
+        GP_CUDA(cudaStreamSynchronize(s));
+        if (h_adjp)  // piece offsets are local: shift them to the concatenation
+            for (int32_t r = 0; r <= c->n; ++r) h_adjp[rows + r] += arcs;
+        rows += c->n;
+        arcs += c->nnz;
+    }
+    if (n_out) *n_out = rows;
+    if (nnz_out) *nnz_out = arcs;
+    return GP_OK;
+    GP_TRY_END
+}
+
+gp_status gp_nccl_unique_id(void *out128) {
+    if (!out128) return GP_ERR_INVALID_ARG;
+    return dist_unique_id(out128);
+}
+
+static gp_status attach_comm(gp_ctx ctx, gp_status st) {
+    if (st != GP_OK) {
+        std::string keep = g_last_error;
+        gp_free(ctx);
+        g_last_error = keep;
+    }
+    return st;
+}
+
+gp_status gp_ctx_create_dist(int device, void *cuda_stream, const void *nccl_unique_id, int rank, int nranks,
+                             gp_ctx *out) {
+    if (!out || !nccl_unique_id || nranks < 1 || rank < 0 || rank >= nranks) {
+        set_error("gp_ctx_create_dist: bad id, rank or nranks");
+        if (out) *out = nullptr;
+        return GP_ERR_INVALID_ARG;
+    }
+    gp_status st = gp_ctx_create(device, cuda_stream, out);
+    if (st != GP_OK) return st;
+    st = attach_comm(*out, dist_comm_create_nccl(*out, nccl_unique_id, rank, nranks));
+    if (st != GP_OK) *out = nullptr;
+    return st;
+}
+
+gp_status gp_ctx_create_loopback(int device, void *cuda_stream, int nranks, gp_ctx *out) {
+    if (!out || nranks < 1) {
+        set_error("gp_ctx_create_loopback: bad nranks");
+        if (out) *out = nullptr;
+        return GP_ERR_INVALID_ARG;
+    }
+    gp_status st = gp_ctx_create(device, cuda_stream, out);
+    if (st != GP_OK) return st;
+    st = attach_comm(*out, dist_comm_create_loopback(*out, nranks));
+    if (st != GP_OK) *out = nullptr;
+    return st;
+}
+
+gp_status gp_ctx_dist_info(gp_ctx ctx, int32_t *rank, int32_t *nranks) {
+    if (!tagged<Ctx>(ctx, kTagCtx)) return GP_ERR_INVALID_ARG;
+    if (rank) *rank = dist_rank(ctx);
+    if (nranks) *nranks = dist_nranks(ctx);
+    return GP_OK;
+}
+
+gp_status gp_graph_create_dist(gp_ctx ctx, gp_vid n_global, gp_vid v_begin, gp_vid v_end, const gp_vid *adjp_local,
+                               const gp_vid *adjncy, const gp_wgt *adjwgt, const gp_wgt *vwgt, uint32_t flags,
+                               gp_graph *out) {
+    if (out) *out = nullptr;
+    if (!tagged<Ctx>(ctx, kTagCtx) || !out || !ctx->comm || dist_rank(ctx) < 0 || n_global < 0 || v_begin < 0 ||
+        v_end < v_begin || v_end > n_global) {
+        set_error("gp_graph_create_dist: needs an NCCL context and 0 <= v_begin <= v_end <= n_global");
+        return GP_ERR_INVALID_ARG;
+    }
+    if (flags & GP_VALIDATE) {
+        set_error("gp_graph_create_dist: GP_VALIDATE checks whole graphs (use a single-GPU context)");
+        return GP_ERR_INVALID_ARG;
+    }
+    GP_TRY_BEGIN
+    gp_graph g = nullptr;
+    gp_status st = gp_graph_create(ctx, v_end - v_begin, adjp_local, adjncy, adjwgt, vwgt, flags, &g);
+    if (st != GP_OK) return st;
+    const int G = dist_nranks(ctx), me = dist_rank(ctx);
+    int32_t mine[3] = {v_begin, v_end, g->nnz};
+    std::vector<int32_t> all(3 * (size_t)G);
+    st = dist_allgather_i32(ctx, mine, 3, all.data());
+    long long nnz = 0;
+    std::vector<int32_t> ranges(G + 1);
+    for (int r = 0; st == GP_OK && r < G; ++r) {
+        ranges[r] = all[3 * r];
+        nnz += all[3 * r + 2];
+        if (all[3 * r] != (r == 0 ? 0 : all[3 * (r - 1) + 1]) || (r == G - 1 && all[3 * r + 1] != n_global)) {
+            set_error("gp_graph_create_dist: the shards do not tile [0, n_global) in rank order");
+            st = GP_ERR_INVALID_ARG;
+        }
+    }
+    if (st == GP_OK && nnz > INT32_MAX) {
+        set_error("gp_graph_create_dist: total arcs exceed INT32_MAX");
+        st = GP_ERR_OVERFLOW;
+    }
+    if (st != GP_OK) {
+        std::string keep = g_last_error;
+        gp_free(g);
+        g_last_error = keep;
+        return st;
+    }
+    ranges[G] = n_global;
+    g->dist = true;
+    g->rank = me;
+    g->vbase = v_begin;
+    g->n_global = n_global;
+    g->nnz_global = (int32_t)nnz;
+    g->ranges = ranges;
+    *out = g;
+    return GP_OK;
+    GP_TRY_END
 }
 
 void gp_free(void *handle) {
@@ -741,6 +930,7 @@ void gp_free(void *handle) {
     } else if (tag == kTagCtx) {
         Ctx *ctx = static_cast<Ctx *>(handle);
         cudaStreamSynchronize(ctx->stream);
+        dist_comm_destroy(ctx);
         drain_events(ctx);
         for (auto e : ctx->event_pool) cudaEventDestroy(e);
         dev_free(ctx, ctx->scratch);

@@ -106,6 +106,16 @@ struct TimedLaunch {
     cudaEvent_t a, b;
 };
 struct Level;
+struct DistComm;  // dist.cu: NCCL or loopback collectives of the sharded path
+// one rank's piece of a sharded level: M / CM are indexed by GLOBAL fine vertex id (length =
+// the level's n_global; only [vbase, vbase + nloc) is this rank's), coarse is the rank's
+// shard of the coarse graph
+struct DistPiece {
+    int rank = 0;
+    int32_t vbase = 0, nloc = 0;
+    int32_t *M = nullptr, *CM = nullptr;
+    ::gp_graph_s *coarse = nullptr;
+};
 }  // namespace gp
 
 struct gp_graph_s {
@@ -116,6 +126,12 @@ struct gp_graph_s {
     gp::SizeRec *sizes = nullptr;  // device copy of {n, nnz, stop}
     bool owns_sizes = true;
     bool borrowed = false;  // owned by a hierarchy
+    // sharded graphs (NCCL contexts): this rank's rows are the global vertices
+    // [vbase, vbase + n); ranges[r] .. ranges[r+1] is rank r's range; adjncy holds global ids
+    bool dist = false;
+    int rank = 0;
+    int32_t vbase = 0, n_global = 0, nnz_global = 0;
+    std::vector<int32_t> ranges;
 };
 
 namespace gp {
@@ -124,6 +140,7 @@ struct Level {
     int64_t arcs_scanned = 0, rows_scanned = 0, live_visits = 0;
     int32_t *match = nullptr, *cmap = nullptr;
     Graph *coarse = nullptr;
+    std::vector<DistPiece> pieces;  // sharded levels: one piece per local rank
 };
 }  // namespace gp
 
@@ -154,6 +171,9 @@ struct gp_ctx_s {
     unsigned long long *status = nullptr;  // look-back tile status words
     size_t status_words = 0;
     uint32_t epoch = 1;  // look-back epoch (no memset between scans)
+
+    // sharded path: NCCL (one local rank) or loopback (all ranks simulated); null = 1 GPU
+    gp::DistComm *comm = nullptr;
 
     // instrumentation
     bool timing = false;
@@ -200,20 +220,43 @@ inline int persistent_grid(const Ctx *ctx, int blocks_per_sm) { return ctx->num_
 // level pipeline entry points (implemented in match.cu / contract.cu / validate.cu)
 // ---------------------------------------------------------------------------------------
 
-// enqueue the persistent matching kernel of one level (A1-A4; leftover optional)
+// enqueue the persistent matching kernel of one level (A1-A4; leftover optional).
+// mode: kMatchWhole (everything in one launch) or one phase per launch for the sharded
+// driver (dist.cu), whose rows are the vertices [vbase, vbase + n) of a larger graph.
+constexpr int kMatchWhole = 0;   // phase 0, every round and the leftover pass in one launch
+constexpr int kMatchPhase0 = 1;  // phase 0 (+ its hub rows): the round-1 proposals
+constexpr int kMatchRound = 2;   // commit of round k + proposals of round k+1 (+ hub rows)
+constexpr int kMatchFinish = 3;  // leftover self-matches + statistics
 gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl, int32_t max_rounds, bool leftover,
-                        double avg_deg_hint);
+                        double avg_deg_hint, int32_t vbase = 0, int mode = kMatchWhole, int k = 0);
 // enqueue the persistent contraction kernel of one level (A4 leftover + A5-A8)
 struct ContractParams {
     bool leftover;
     int32_t threshold, stall_pct, level, max_levels;
     int32_t n_bound, nnz_bound;
+    // sharded levels only (see ContractArgs in contract.cu)
+    int32_t dist = 0, cbase = 0, tb = 0, nnz_ub = 0;
 };
+constexpr int kContractTileBudget = 256;  // C2 warp-tile budget (upper-bound entries), kWB
+int contract_grid(Ctx *ctx);
 gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *CM, Graph *coarse, ContractCtl *ctl,
                            SizeRec *out_sizes, LevelReport *report, const ContractParams &prm);
 size_t contract_tiles(int32_t n, int32_t nnz);
 
 gp_status graph_totals_and_validate(Ctx *ctx, const Graph *g, bool validate);
+
+// sharded path (dist.cu)
+gp_status dist_coarsen_to(Graph *g, const gp_coarsen_opts *opts, Hier **out);
+gp_status dist_comm_create_nccl(Ctx *ctx, const void *uid, int rank, int nranks);
+gp_status dist_comm_create_loopback(Ctx *ctx, int nranks);
+void dist_comm_destroy(Ctx *ctx);
+gp_status dist_unique_id(void *out128);
+int dist_rank(const Ctx *ctx);    // -1 loopback, else the rank
+int dist_nranks(const Ctx *ctx);  // 1 without a communicator
+gp_status dist_allgather_i32(Ctx *ctx, const int32_t *h_send, int32_t count, int32_t *h_recv);  // host values
+void graph_release(Graph *g);
+void hier_release(Hier *h);
+gp_status alloc_graph_arrays(Ctx *ctx, Graph *g, int32_t n_bound, int32_t nnz_bound, bool own_sizes);
 
 gp_status ensure_scratch(Ctx *ctx, size_t bytes);
 // carve one level's scratch pointers out of ctx->scratch (sized for n, nnz)

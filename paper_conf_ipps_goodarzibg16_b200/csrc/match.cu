@@ -60,7 +60,14 @@ struct MatchArgs {
     int32_t G;    // lanes per vertex in phase 0 (1, 2, 4, 8 or 16)
     int32_t vch;  // vertices per phase-0 chunk (about 80 % of a stage at the average degree)
     int32_t vpc;  // vertices per active CTA (small levels run on fewer CTAs)
+    // sharded levels (dist.cu): the rows are the vertices [vbase, vbase + n) of a graph of
+    // n_global vertices; P, S and M are indexed by global vertex id (ghost entries are
+    // filled by the exchange between launches).  Single GPU: vbase = 0.
+    int32_t vbase;
+    int32_t mode;  // kMatchWhole, or one launch per phase for the sharded path
+    int32_t k;     // round of a kMatchRound launch
 };
+
 
 struct MatchSmem {
     int32_t adj[kStages][kStageArcs];
@@ -251,15 +258,16 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
             }
             group_top2_rt(key, key2, G);
             if (valid && gl == 0) {
-                a.M[v] = kFree;
+                const int32_t x = a.vbase + (int32_t)v;  // row v is vertex vbase + v
+                a.M[x] = kFree;
                 if (hub) {
-                    a.H[atomicAdd(&a.ctl->slot[1].nhub, 1)] = (int32_t)v;
-                    a.S[v] = kNone;
+                    a.H[atomicAdd(&a.ctl->slot[1].nhub, 1)] = x;
+                    a.S[x] = kNone;
                 } else {
                     const int32_t p = key_vertex(key);
-                    P1[v] = p;
-                    a.S[v] = key_vertex(key2);  // cached second-heaviest neighbour
-                    if (p == kNone) P0[v] = kNone;  // dead vertices: NONE in both buffers
+                    P1[x] = p;
+                    a.S[x] = key_vertex(key2);  // cached second-heaviest neighbour
+                    if (p == kNone) P0[x] = kNone;  // dead vertices: NONE in both buffers
                     scanned += (unsigned long long)(e - s);
                 }
             }
@@ -286,7 +294,7 @@ __device__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool 
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     for (int i = blockIdx.x; i < nhub; i += g_nact) {
         const int32_t u = a.H[i];
-        const int32_t s = __ldg(a.adjp + u), e = __ldg(a.adjp + u + 1);
+        const int32_t s = __ldg(a.adjp + (u - a.vbase)), e = __ldg(a.adjp + (u - a.vbase) + 1);
         unsigned long long key = 0;
         for (int32_t j = s + threadIdx.x; j < e; j += kNT) {
             const int32_t x = __ldg(a.adjncy + j);
@@ -369,7 +377,7 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
             const long long idx = base + i * 32 + lane;
-            u[i] = idx < len ? ((k == 1) ? (int32_t)idx : ldcg(Lk + idx)) : -1;
+            u[i] = idx < len ? ((k == 1) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
         }
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
@@ -417,8 +425,8 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
             int32_t s = 0, e = 0;
             bool need_warp = false;
             if (need[i]) {
-                s = __ldg(a.adjp + u[i]);
-                e = __ldg(a.adjp + u[i] + 1);
+                s = __ldg(a.adjp + (u[i] - a.vbase));
+                e = __ldg(a.adjp + (u[i] - a.vbase) + 1);
                 ++rows;
                 if (e - s <= kThreadDeg) {
                     unsigned long long key, key2;
@@ -503,54 +511,59 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
     unsigned long long scanned = 0, rows = 0, visits = 0;
     unsigned bar_epoch = 0;  // grid barriers passed (thread 0)
     int tr = 0;
-    trace_mark(ctl->trace, tr++);
-    phase0(a, sm, n, scanned);
-    trace_mark(ctl->trace, tr++);
-    grid_barrier(ctl->bar, bar_epoch, g_nact);
-    trace_mark(ctl->trace, tr++);
-    {
-        const int32_t nh = *(volatile int32_t *)&ctl->slot[1].nhub;
-        if (nh > 0) {
-            hub_phase(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned);
-            grid_barrier(ctl->bar, bar_epoch, g_nact);
-        }
-    }
-    int32_t rounds = 0, maximal = 0;
-    for (int k = 1;; ++k) {
-        if (k > n + 2) __trap();  // every round matches >= 1 pair: a bug
-        if (blockIdx.x == 0 && threadIdx.x == 0) {
-            RoundSlot *z = &ctl->slot[(k + 2) & 3];  // last read two phases ago
-            z->live = 0;
-            z->nhub = 0;
-            z->matches = 0;
-            z->claim = 0;
-        }
-        const int32_t len = (k == 1) ? n : *(volatile int32_t *)&ctl->slot[k & 3].live;
-        int32_t made = 0;
-        phase_k(a, sm, n, k, len, scanned, rows, visits, made);
-        // any match this round: one flag store per CTA (only "> 0" is used)
-        if (__syncthreads_or(made > 0) && threadIdx.x == 0) *(volatile int32_t *)&ctl->slot[k & 3].matches = 1;
+    if (a.mode == kMatchWhole || a.mode == kMatchPhase0) {
+        trace_mark(ctl->trace, tr++);
+        phase0(a, sm, n, scanned);
         trace_mark(ctl->trace, tr++);
         grid_barrier(ctl->bar, bar_epoch, g_nact);
         trace_mark(ctl->trace, tr++);
-        const int32_t nh = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].nhub;
+        const int32_t nh = *(volatile int32_t *)&ctl->slot[1].nhub;
         if (nh > 0) {
-            hub_phase(a, sm, nh, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1], &ctl->slot[(k + 1) & 3].live,
-                      scanned);
+            hub_phase(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned);
+            if (a.mode == kMatchWhole) grid_barrier(ctl->bar, bar_epoch, g_nact);
+        }
+    }
+    int32_t rounds = 0, maximal = 0;
+    if (a.mode == kMatchWhole || a.mode == kMatchRound) {
+        // kMatchWhole: the device-side round loop; kMatchRound: round a.k only (the sharded
+        // driver exchanges the boundary proposals between launches and decides termination)
+        for (int k = (a.mode == kMatchRound) ? a.k : 1;; ++k) {
+            if (k > n + 2 && a.mode == kMatchWhole) __trap();  // each round matches >= 1 pair
+            if (blockIdx.x == 0 && threadIdx.x == 0) {
+                RoundSlot *z = &ctl->slot[(k + 2) & 3];  // last read two phases ago
+                z->live = 0;
+                z->nhub = 0;
+                z->matches = 0;
+                z->claim = 0;
+            }
+            const int32_t len = (k == 1) ? n : *(volatile int32_t *)&ctl->slot[k & 3].live;
+            int32_t made = 0;
+            phase_k(a, sm, n, k, len, scanned, rows, visits, made);
+            // any match this round: one flag store per CTA (only "> 0" is used)
+            if (__syncthreads_or(made > 0) && threadIdx.x == 0) *(volatile int32_t *)&ctl->slot[k & 3].matches = 1;
+            trace_mark(ctl->trace, tr++);
             grid_barrier(ctl->bar, bar_epoch, g_nact);
+            trace_mark(ctl->trace, tr++);
+            const int32_t nh = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].nhub;
+            if (nh > 0) {
+                hub_phase(a, sm, nh, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1],
+                          &ctl->slot[(k + 1) & 3].live, scanned);
+                grid_barrier(ctl->bar, bar_epoch, g_nact);
+            }
+            if (a.mode == kMatchRound) break;
+            if (*(volatile int32_t *)&ctl->slot[k & 3].matches > 0) ++rounds;
+            const int32_t live = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].live;
+            if (live == 0) {
+                maximal = 1;
+                break;
+            }
+            if (a.max_rounds > 0 && rounds >= a.max_rounds) break;
         }
-        if (*(volatile int32_t *)&ctl->slot[k & 3].matches > 0) ++rounds;
-        const int32_t live = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].live;
-        if (live == 0) {
-            maximal = 1;
-            break;
-        }
-        if (a.max_rounds > 0 && rounds >= a.max_rounds) break;
     }
     trace_mark(ctl->trace, tr++);
-    if (a.leftover) {
+    if (a.leftover && (a.mode == kMatchWhole || a.mode == kMatchFinish)) {
         for (long long u = (long long)blockIdx.x * kNT + threadIdx.x; u < n; u += (long long)g_nact * kNT)
-            if (a.M[u] == kFree) a.M[u] = (int32_t)u;
+            if (a.M[a.vbase + u] == kFree) a.M[a.vbase + u] = a.vbase + (int32_t)u;
     }
     scanned = warp_sum64(scanned);
     rows = warp_sum64(rows);
@@ -566,7 +579,7 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
         for (int w = 0; w < kNT / 32; ++w) t += sm.cnt3[threadIdx.x][w];
         if (t) atomicAdd(threadIdx.x == 0 ? &ctl->arcs_scanned : threadIdx.x == 1 ? &ctl->rows_scanned : &ctl->live_visits, t);
     }
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
+    if (blockIdx.x == 0 && threadIdx.x == 0 && a.mode == kMatchWhole) {
         ctl->rounds = rounds;
         ctl->maximal = maximal;
     }
@@ -606,8 +619,11 @@ int match_grid(Ctx *ctx) {
 }
 
 gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl, int32_t max_rounds,
-                        bool leftover, double avg_deg_hint) {
+                        bool leftover, double avg_deg_hint, int32_t vbase, int mode, int k) {
     MatchArgs a;
+    a.vbase = vbase;
+    a.mode = mode;
+    a.k = k;
     a.in = lb.in;
     a.adjp = lb.adjp;
     a.adjncy = lb.adjncy;

@@ -55,7 +55,8 @@ class Level(ctypes.Structure):
     _fields_ = [("n", _i32), ("nnz", _i32), ("n_coarse", _i32), ("cnnz", _i32), ("rounds", _i32),
                 ("maximal", _i32), ("stop_reason", _i32), ("reserved", _i32),
                 ("arcs_scanned", ctypes.c_int64), ("rows_scanned", ctypes.c_int64),
-                ("live_visits", ctypes.c_int64), ("d_match", _vp), ("d_cmap", _vp), ("coarse", _vp)]
+                ("live_visits", ctypes.c_int64), ("d_match", _vp), ("d_cmap", _vp), ("coarse", _vp),
+                ("v_begin", _i32), ("n_local", _i32), ("cv_begin", _i32), ("n_coarse_local", _i32)]
 
 
 class KernelStats(ctypes.Structure):
@@ -83,6 +84,13 @@ _sig("gp_coarsen_to", ctypes.c_int, [_vp, ctypes.POINTER(CoarsenOpts), ctypes.PO
 _sig("gp_hier_num_levels", ctypes.c_int, [_vp, _i32p])
 _sig("gp_hier_level", ctypes.c_int, [_vp, _i32, ctypes.POINTER(Level)])
 _sig("gp_hier_download_level", ctypes.c_int, [_vp, _i32, _vp, _vp])
+_sig("gp_hier_download_coarse", ctypes.c_int, [_vp, _i32, _vp, _vp, _vp, _vp, _i32p, _i32p])
+_sig("gp_nccl_unique_id", ctypes.c_int, [_vp])
+_sig("gp_ctx_create_dist", ctypes.c_int, [ctypes.c_int, _vp, _vp, ctypes.c_int, ctypes.c_int, ctypes.POINTER(_vp)])
+_sig("gp_ctx_create_loopback", ctypes.c_int, [ctypes.c_int, _vp, ctypes.c_int, ctypes.POINTER(_vp)])
+_sig("gp_ctx_dist_info", ctypes.c_int, [_vp, _i32p, _i32p])
+_sig("gp_graph_create_dist", ctypes.c_int, [_vp, _i32, _i32, _i32, _vp, _vp, _vp, _vp, ctypes.c_uint32,
+                                            ctypes.POINTER(_vp)])
 _sig("gp_free", None, [_vp])
 _sig("gp_ctx_set_timing", ctypes.c_int, [_vp, _i32])
 _sig("gp_ctx_kernel_stats", ctypes.c_int, [_vp, ctypes.c_int, ctypes.POINTER(KernelStats)])
@@ -102,17 +110,44 @@ def _ptr(t: Optional[torch.Tensor]):
     return t.data_ptr()
 
 
-class Context:
-    """gp_ctx on a CUDA device, enqueuing on the given (default: current) torch stream."""
+def nccl_unique_id() -> bytes:
+    """gp_nccl_unique_id: the 128-byte NCCL id rank 0 creates and broadcasts."""
+    buf = ctypes.create_string_buffer(128)
+    _check(_lib.gp_nccl_unique_id(buf), "gp_nccl_unique_id")
+    return buf.raw
 
-    def __init__(self, device: int = 0, stream: Optional[torch.cuda.Stream] = None):
+
+class Context:
+    """gp_ctx on a CUDA device, enqueuing on the given (default: current) torch stream.
+
+    Context(dev)                           single GPU
+    Context(dev, loopback=G)               G simulated ranks of the sharded path on one GPU
+    Context(dev, nccl_id=id, rank=r, nranks=G)   rank r of G processes (one per GPU, NCCL)
+    """
+
+    def __init__(self, device: int = 0, stream: Optional[torch.cuda.Stream] = None, *, loopback: int = 0,
+                 nccl_id: Optional[bytes] = None, rank: int = 0, nranks: int = 1):
         if not torch.cuda.is_available():
             raise RuntimeError("no CUDA device: the coarsening path has no CPU fallback")
         self.device = device
         self.stream = stream if stream is not None else torch.cuda.current_stream(device)
         h = _vp()
-        _check(_lib.gp_ctx_create(device, self.stream.cuda_stream, ctypes.byref(h)), "gp_ctx_create")
+        if nccl_id is not None:
+            idbuf = ctypes.create_string_buffer(bytes(nccl_id), 128)
+            _check(_lib.gp_ctx_create_dist(device, self.stream.cuda_stream, idbuf, rank, nranks, ctypes.byref(h)),
+                   "gp_ctx_create_dist")
+        elif loopback:
+            _check(_lib.gp_ctx_create_loopback(device, self.stream.cuda_stream, loopback, ctypes.byref(h)),
+                   "gp_ctx_create_loopback")
+        else:
+            _check(_lib.gp_ctx_create(device, self.stream.cuda_stream, ctypes.byref(h)), "gp_ctx_create")
         self.handle = h
+
+    def dist_info(self):
+        """(rank, nranks): (0, 1) single GPU, (-1, G) loopback."""
+        r, g = _i32(), _i32()
+        _check(_lib.gp_ctx_dist_info(self.handle, ctypes.byref(r), ctypes.byref(g)), "gp_ctx_dist_info")
+        return r.value, g.value
 
     def close(self) -> None:
         if self.handle is not None and self.handle.value:
@@ -173,6 +208,19 @@ class Graph:
         h = _vp()
         _check(_lib.gp_graph_create(ctx.handle, n, _ptr(adjp), _ptr(adjncy), _ptr(adjwgt), _ptr(vwgt), flags,
                                     ctypes.byref(h)), "gp_graph_create")
+        return cls(ctx, h)
+
+    @classmethod
+    def create_dist(cls, ctx: Context, n_global: int, v_begin: int, adjp_local: torch.Tensor,
+                    adjncy: torch.Tensor, adjwgt: Optional[torch.Tensor] = None,
+                    vwgt: Optional[torch.Tensor] = None) -> "Graph":
+        """gp_graph_create_dist: this rank's rows [v_begin, v_begin + len(adjp_local) - 1)
+        with local offsets and global column ids (collective over the NCCL context)."""
+        v_end = v_begin + adjp_local.numel() - 1
+        flags = GP_INPUT_DEVICE if adjp_local.is_cuda else 0
+        h = _vp()
+        _check(_lib.gp_graph_create_dist(ctx.handle, n_global, v_begin, v_end, _ptr(adjp_local), _ptr(adjncy),
+                                         _ptr(adjwgt), _ptr(vwgt), flags, ctypes.byref(h)), "gp_graph_create_dist")
         return cls(ctx, h)
 
     def close(self) -> None:
@@ -246,6 +294,10 @@ class LevelInfo:
     rows_scanned: int
     live_visits: int
     coarse: Graph
+    v_begin: int = 0
+    n_local: int = 0
+    cv_begin: int = 0
+    n_coarse_local: int = 0
 
 
 class Hierarchy:
@@ -275,7 +327,8 @@ class Hierarchy:
         l = Level()
         _check(_lib.gp_hier_level(self.handle, i, ctypes.byref(l)), "gp_hier_level")
         return LevelInfo(l.n, l.nnz, l.n_coarse, l.cnnz, l.rounds, bool(l.maximal), l.stop_reason,
-                         l.arcs_scanned, l.rows_scanned, l.live_visits, Graph(self.ctx, _vp(l.coarse), owned=False))
+                         l.arcs_scanned, l.rows_scanned, l.live_visits, Graph(self.ctx, _vp(l.coarse), owned=False),
+                         l.v_begin, l.n_local, l.cv_begin, l.n_coarse_local)
 
     def levels(self) -> List[LevelInfo]:
         return [self.level(i) for i in range(len(self))]
@@ -285,11 +338,32 @@ class Hierarchy:
         """(match, cmap) of level i as host int32 tensors (optionally preallocated/pinned);
         want_match=False skips the match copy and returns (None, cmap)."""
         info = self.level(i)
-        m = None if not want_match else (match if match is not None else torch.empty(info.n, dtype=torch.int32))
-        c = cmap if cmap is not None else torch.empty(info.n, dtype=torch.int32)
+        rank, _ = self.ctx.dist_info()
+        n = info.n_local if rank >= 0 else info.n  # NCCL rank: its piece; loopback / 1 GPU: all
+        m = None if not want_match else (match if match is not None else torch.empty(n, dtype=torch.int32))
+        c = cmap if cmap is not None else torch.empty(n, dtype=torch.int32)
         _check(_lib.gp_hier_download_level(self.handle, i, m.data_ptr() if m is not None else None, c.data_ptr()),
                "gp_hier_download_level")
         return m, c
+
+
+    def download_coarse(self, i: int) -> Dict[str, torch.Tensor]:
+        """Coarse graph of level i as host int32 tensors (gp_hier_download_coarse): the whole
+        graph on one GPU / loopback, this rank's piece (global column ids) on an NCCL rank."""
+        info = self.level(i)
+        rank, _ = self.ctx.dist_info()
+        n = info.n_coarse_local if rank >= 0 else info.n_coarse
+        out = {"adjp": torch.empty(n + 1, dtype=torch.int32), "adjncy": torch.empty(max(info.cnnz, 1), dtype=torch.int32),
+               "adjwgt": torch.empty(max(info.cnnz, 1), dtype=torch.int32), "vwgt": torch.empty(max(n, 1), dtype=torch.int32)}
+        rows, arcs = _i32(), _i32()
+        _check(_lib.gp_hier_download_coarse(self.handle, i, out["adjp"].data_ptr(), out["adjncy"].data_ptr(),
+                                            out["adjwgt"].data_ptr(), out["vwgt"].data_ptr(), ctypes.byref(rows),
+                                            ctypes.byref(arcs)), "gp_hier_download_coarse")
+        out["adjncy"] = out["adjncy"][:arcs.value]
+        out["adjwgt"] = out["adjwgt"][:arcs.value]
+        out["vwgt"] = out["vwgt"][:rows.value]
+        out["n"], out["nnz"] = rows.value, arcs.value
+        return out
 
 
 def exported_symbols():

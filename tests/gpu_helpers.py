@@ -22,7 +22,7 @@ def gpu_coarsen(gp, ctx, g: Dict, threshold: int, **kw) -> List[Dict]:
     out = []
     for i, info in enumerate(H.levels()):
         m, c = H.download_level(i)
-        coarse = info.coarse.download()
+        coarse = H.download_coarse(i)
         out.append({"n": info.n, "nnz": info.nnz, "n_coarse": info.n_coarse, "rounds": info.rounds,
                     "maximal": info.maximal, "stop_reason": info.stop_reason, "match": m.numpy(),
                     "cmap": c.numpy(), "coarse": {k: coarse[k].numpy() for k in ("adjp", "adjncy", "adjwgt", "vwgt")},
