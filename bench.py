@@ -193,9 +193,23 @@ def run_ours(args, rank, world, local_rank):
     name, threshold = WORKLOADS[args.config]
     g, gen_s = make_graph(args.config, dev)
     n, nnz = g["n"], g["nnz"]
-    ctx = gp.Context(local_rank)
+    sharded = world > 1   # N GPUs: the sharded path over NCCL (strong scaling: one graph)
+    if sharded:
+        uid = [gp.nccl_unique_id() if rank == 0 else None]
+        torch.distributed.broadcast_object_list(uid, src=0)
+        ctx = gp.Context(local_rank, nccl_id=uid[0], rank=rank, nranks=world)
+        vb, ve = n * rank // world, n * (rank + 1) // world   # this rank's vertex range
+        a0, a1 = int(g["adjp"][vb]), int(g["adjp"][ve])
+        shard = {"adjp": (g["adjp"][vb:ve + 1] - a0).contiguous(), "adjncy": g["adjncy"][a0:a1].contiguous(),
+                 "adjwgt": g["adjwgt"][a0:a1].contiguous(), "vwgt": g["vwgt"][vb:ve].contiguous()}
+        graph = gp.Graph.create_dist(ctx, n, vb, shard["adjp"], shard["adjncy"], shard["adjwgt"], shard["vwgt"])
+    elif args.loopback > 1:  # the sharded protocol simulated on this one GPU (tests / profiling)
+        ctx = gp.Context(local_rank, loopback=args.loopback)
+        graph = gp.Graph.create(ctx, g["adjp"], g["adjncy"], g["adjwgt"], g["vwgt"])
+    else:
+        ctx = gp.Context(local_rank)
+        graph = gp.Graph.create(ctx, g["adjp"], g["adjncy"], g["adjwgt"], g["vwgt"])
     stream = ctx.stream
-    graph = gp.Graph.create(ctx, g["adjp"], g["adjncy"], g["adjwgt"], g["vwgt"])
 
     def step():
         return graph.coarsen_to(threshold)
@@ -250,6 +264,8 @@ def run_ours(args, rank, world, local_rank):
     for l in levels:
         for k, v in level_bytes(l).items():
             fam_bytes[k] = fam_bytes.get(k, 0) + v
+    if sharded:  # global sizes / world: the bytes one rank's kernels move (rows split evenly)
+        fam_bytes = {k: v / world for k, v in fam_bytes.items()}
     kfam = {"match": "propose", "contract": "contract"}   # gp_kernel_kind of each family
     fam_ms = {k: kstats[kfam[k]]["ms"] / args.steps for k in fam_bytes}
     dom = max(fam_ms, key=lambda k: fam_ms[k])
@@ -259,16 +275,11 @@ def run_ours(args, rank, world, local_rank):
     traffic = ncu_traffic(args.config, {"match": "k_match_level", "contract": "k_contract_level"}[dom])
 
     # end-to-end through the C ABI with host buffers
-    host = {k: g[k].cpu().pin_memory() for k in ("adjp", "adjncy", "adjwgt", "vwgt")}
+    host = {k: (shard if sharded else g)[k].cpu().pin_memory() for k in ("adjp", "adjncy", "adjwgt", "vwgt")}
     h2d = sum(t.numel() * 4 for t in host.values())
     # pinned result buffers sized from the warm-up hierarchy (what a partitioner keeps:
     # every level's CM for projection, and the coarsest graph)
-    cm_bufs = [torch.empty(l["n"], dtype=torch.int32).pin_memory() for l in levels]
-    last_l = levels[-1]
-    last_bufs = {"adjp": torch.empty(last_l["n_coarse"] + 1, dtype=torch.int32).pin_memory(),
-                 "adjncy": torch.empty(last_l["cnnz"], dtype=torch.int32).pin_memory(),
-                 "adjwgt": torch.empty(last_l["cnnz"], dtype=torch.int32).pin_memory(),
-                 "vwgt": torch.empty(last_l["n_coarse"], dtype=torch.int32).pin_memory()}
+    cm_bufs = [torch.empty(l["n_local"] if sharded else l["n"], dtype=torch.int32).pin_memory() for l in levels]
     e2e_ms = []
     d2h = 0
     for it in range(max(2, min(args.steps, 5)) + 1):
@@ -276,13 +287,16 @@ def run_ours(args, rank, world, local_rank):
         a = torch.cuda.Event(enable_timing=True)
         b = torch.cuda.Event(enable_timing=True)
         a.record(stream)
-        gh = gp.Graph.create(ctx, host["adjp"], host["adjncy"], host["adjwgt"], host["vwgt"])
+        if sharded:
+            gh = gp.Graph.create_dist(ctx, n, vb, host["adjp"], host["adjncy"], host["adjwgt"], host["vwgt"])
+        else:
+            gh = gp.Graph.create(ctx, host["adjp"], host["adjncy"], host["adjwgt"], host["vwgt"])
         hh = gh.coarsen_to(threshold)
         nb = 0
         for i in range(len(hh)):
             _, c = hh.download_level(i, cmap=cm_bufs[i], want_match=False)
             nb += c.numel() * 4
-        last = hh.level(len(hh) - 1).coarse.download(out=last_bufs)
+        last = hh.download_coarse(len(hh) - 1)
         nb += sum(last[k].numel() * 4 for k in ("adjp", "adjncy", "adjwgt", "vwgt"))
         b.record(stream)
         torch.cuda.synchronize()
@@ -294,15 +308,17 @@ def run_ours(args, rank, world, local_rank):
     e2e_step = min(e2e_ms)
 
     line = {
-        "metric": METRIC, "value": world * edges_per_step / (ms_step / 1e3), "unit": UNIT, "n_gpus": world,
+        "metric": METRIC, "value": edges_per_step / (ms_step / 1e3), "unit": UNIT, "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "scaling": "strong" if sharded else "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
         "config": {"workload": f"{args.config}:{name}", "n": n, "edges": nnz // 2, "threshold": threshold,
                    "levels": len(levels), "edges_all_levels": edges_per_step,
                    "level0_edges_per_s": (nnz // 2) / (ms_step / 1e3),
                    "t_full_ms": ms_step, "rounds": [l["rounds"] for l in levels],
                    "l2": f"L0 input {(4 * (2 * nnz + 2 * n)) / 2**20:.0f} MiB > L2 126 MiB (no flush)",
-                   "parallelism": "single GPU" if world == 1 else f"replicas x{world} (sharded path not built)",
+                   "parallelism": (f"sharded x{world}: vertex ranges, NCCL all-gather per handshake round"
+                                   if sharded else f"loopback x{args.loopback} on 1 GPU (sharded protocol simulated)"
+                                   if args.loopback > 1 else "single GPU"),
                    "gen_s": round(gen_s, 2)},
         "hbm_gbs_step": step_bytes / (ms_step / 1e3) / 1e9,
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "peak_kind": peak_kind,
@@ -312,7 +328,7 @@ def run_ours(args, rank, world, local_rank):
                      "bytes_per_step": fam_bytes[dom], "ms_per_step": fam_ms[dom]},
         "kernels": {k: {"ms_per_step": fam_ms[k], "GB/s": (fam_bytes[k] / (fam_ms[k] / 1e3) / 1e9) if fam_ms[k] else None,
                         "launches_per_step": kstats[kfam[k]]["launches"] / args.steps} for k in fam_bytes},
-        "e2e": {"value": world * edges_per_step / (e2e_step / 1e3), "unit": UNIT, "ms_per_step": e2e_step,
+        "e2e": {"value": edges_per_step / (e2e_step / 1e3), "unit": UNIT, "ms_per_step": e2e_step,
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
         "gpu_launches": launches,
         "clocks": clk.summary(),
@@ -360,6 +376,8 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--config", choices=sorted(WORKLOADS), default="C3")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--loopback", type=int, default=0,
+                    help="run the sharded protocol with this many simulated ranks on one GPU")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3) if args.impl == "ours" else args.warmup
 
