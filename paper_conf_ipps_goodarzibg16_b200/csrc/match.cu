@@ -64,6 +64,9 @@ struct MatchArgs {
     // n_global vertices; P, S and M are indexed by global vertex id (ghost entries are
     // filled by the exchange between launches).  Single GPU: vbase = 0.
     int32_t vbase;
+    int32_t lanes_mode;  // 1: short live lists use G lanes per vertex (phase_k_lanes)
+    int32_t tail_live;   // live lists this short are finished by CTA 0 alone
+    int32_t interleave;  // phase-k groups dealt to CTAs round-robin (1) or in contiguous ranges (0)
     int32_t mode;  // kMatchWhole, or one launch per phase for the sharded path
     int32_t k;     // round of a kMatchRound launch
 };
@@ -330,17 +333,148 @@ __device__ __forceinline__ void rescan_thread(const MatchArgs &a, const int32_t 
                                               unsigned long long &key, unsigned long long &key2) {
     key = key2 = 0;
     for (int32_t j0 = s; j0 < e; j0 += 8) {
-        int32_t x[8], px[8], pp[8];
+        int32_t x[8], w[8], px[8], pp[8];
 #pragma unroll
-        for (int b = 0; b < 8; ++b) x[b] = (j0 + b < e) ? __ldg(a.adjncy + j0 + b) : -1;
+        for (int b = 0; b < 8; ++b) {
+            x[b] = (j0 + b < e) ? __ldg(a.adjncy + j0 + b) : -1;
+            w[b] = (j0 + b < e) ? __ldg(a.adjwgt + j0 + b) : 0;
+        }
 #pragma unroll
         for (int b = 0; b < 8; ++b) px[b] = (x[b] >= 0) ? ldcg(Pk + x[b]) : -1;
 #pragma unroll
         for (int b = 0; b < 8; ++b) pp[b] = (px[b] >= 0) ? ldcg(Pk + px[b]) : -1;
 #pragma unroll
         for (int b = 0; b < 8; ++b)
-            if (x[b] >= 0 && pp[b] != x[b]) top2_add(key, key2, pack_key(__ldg(a.adjwgt + j0 + b), x[b]));
+            if (x[b] >= 0 && pp[b] != x[b]) top2_add(key, key2, pack_key(w[b], x[b]));
     }
+}
+
+// CTA-aggregated final flush of the warps' list queues: one global atomic per CTA.  All
+// threads of the CTA call.
+__device__ __forceinline__ void cta_flush(MatchSmem &sm, const int32_t *q, int32_t qn, int32_t *list,
+                                          int32_t *counter) {
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    if (lane == 0) sm.scratch[wib] = qn;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int32_t tot = 0;
+        for (int w = 0; w < kNT / 32; ++w) {
+            const int32_t c = sm.scratch[w];
+            sm.scratch[w] = tot;
+            tot += c;
+        }
+        sm.scratch[kNT / 32] = tot ? atomicAdd(counter, tot) : 0;
+    }
+    __syncthreads();
+    const int32_t base = sm.scratch[kNT / 32] + sm.scratch[wib];
+    for (int i = lane; i < qn; i += 32) list[base + i] = q[i];
+}
+
+// Short live lists (small levels, late rounds): G lanes per live vertex, so a warp covers
+// 32/G vertices and a rescan reads G*4 arcs per dependent step instead of 8 per thread.
+// The round's critical path is then ~8 dependent loads whatever the row length (<= kHubDeg).
+// Same decisions as phase_k_impl (commit / keep p / cached second choice / rescan).
+template <int G>
+__device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t len, unsigned long long &scanned,
+                              unsigned long long &rows, unsigned long long &visits, int32_t &made) {
+    constexpr int VPW = 32 / G;  // live vertices per warp step
+    const int32_t *Pk = a.P[k & 1];
+    int32_t *Pn = a.P[(k + 1) & 1];
+    int32_t *Pkw = a.P[k & 1];
+    const int32_t *Lk = a.L[k & 1];
+    int32_t *Ln = a.L[(k + 1) & 1];
+    RoundSlot *next = &a.ctl->slot[(k + 1) & 3];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5, gl = lane % G;
+    int32_t *q = reinterpret_cast<int32_t *>(&sm.adj[0][0]) + wib * kWQ;
+    int32_t qn = 0;
+    const long long ngroups = ((long long)len + VPW - 1) / VPW;
+    const long long g_lo = ngroups * blockIdx.x / g_nact, g_hi = ngroups * (blockIdx.x + 1) / g_nact;
+    if (threadIdx.x == 0) sm.claim = 0;
+    __syncthreads();
+    auto claim_next = [&]() -> long long {
+        int c = 0;
+        if (lane == 0) c = atomicAdd(&sm.claim, 1);
+        c = __shfl_sync(0xffffffffu, c, 0);
+        // interleaved (group c of CTA b = b + c * nact): a spatial cluster of rescans is
+        // spread over all CTAs instead of landing on one; contiguous with GP_MATCH_CONTIG=1
+        return a.interleave ? (long long)blockIdx.x + (long long)c * g_nact : g_lo + c;
+    };
+    for (long long g = claim_next(); g < (a.interleave ? ngroups : g_hi); g = claim_next()) {
+        const long long idx = g * VPW + lane / G;
+        int32_t u = idx < len ? ((k == 1) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
+        const int32_t p = u >= 0 ? ldcg(Pk + u) : kNone;
+        const int32_t s2 = (u >= 0 && p != kNone) ? ldcg(a.S + u) : kNone;
+        const int32_t qq = p != kNone ? ldcg(Pk + p) : kNone;
+        const int32_t ps = s2 != kNone ? ldcg(Pk + s2) : -1;
+        const int32_t rr = (p != kNone && qq != u && qq >= 0) ? ldcg(Pk + qq) : -1;
+        const int32_t pps = ps >= 0 ? ldcg(Pk + ps) : -1;
+        bool need = false, live = false;
+        if (p != kNone) {
+            if (gl == 0) ++visits;
+            if (qq == u) {
+                if (gl == 0) {
+                    a.M[u] = p;  // handshake
+                    Pn[u] = p;
+                    ++made;
+                }
+            } else if (rr != p) {
+                if (gl == 0) Pn[u] = p;  // p still free: still the heaviest free neighbour
+                live = true;
+            } else if (s2 != kNone && pps != s2) {
+                if (gl == 0) {
+                    Pn[u] = s2;  // cached second choice still free
+                    a.S[u] = kNone;
+                }
+                live = true;
+            } else {
+                need = true;
+            }
+        }
+        int32_t s = 0, e = 0;
+        if (need) {
+            s = __ldg(a.adjp + (u - a.vbase));
+            e = __ldg(a.adjp + (u - a.vbase) + 1);
+            if (e - s > kHubDeg) {
+                if (gl == 0) a.H[atomicAdd(&next->nhub, 1)] = u;
+                need = false;
+                e = s;
+            } else if (gl == 0) {
+                ++rows;
+                scanned += (unsigned long long)(e - s);
+            }
+        }
+        // warp-uniform trip count keeps the width-G shuffles converged
+        int32_t trips = need ? (e - s + 4 * G - 1) / (4 * G) : 0;
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) trips = max(trips, __shfl_xor_sync(0xffffffffu, trips, off));
+        unsigned long long key = 0, key2 = 0;
+        for (int t = 0; t < trips; ++t) {
+            int32_t x[4], w[4], px[4], pp[4];
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                const int32_t j = s + (t * 4 + b) * G + gl;
+                x[b] = (need && j < e) ? __ldg(a.adjncy + j) : -1;
+                w[b] = (need && j < e) ? __ldg(a.adjwgt + j) : 0;
+            }
+#pragma unroll
+            for (int b = 0; b < 4; ++b) px[b] = x[b] >= 0 ? ldcg(Pk + x[b]) : -1;
+#pragma unroll
+            for (int b = 0; b < 4; ++b) pp[b] = px[b] >= 0 ? ldcg(Pk + px[b]) : -1;
+#pragma unroll
+            for (int b = 0; b < 4; ++b)
+                if (x[b] >= 0 && pp[b] != x[b]) top2_add(key, key2, pack_key(w[b], x[b]));  // x free after round k
+        }
+        if (trips > 0) group_top2<G>(key, key2);
+        if (need && gl == 0) {
+            const int32_t b = key_vertex(key);
+            Pn[u] = b;
+            a.S[u] = key_vertex(key2);
+            if (b == kNone) Pkw[u] = kNone;  // dead: NONE in both buffers
+            live = b != kNone;
+        }
+        wq_push(q, qn, Ln, &next->live, live && gl == 0, u);
+    }
+    cta_flush(sm, q, qn, Ln, &next->live);
 }
 
 // kVL live vertices per lane per step: their dependent loads overlap.  4 on long lists, 1 on
@@ -368,9 +502,12 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
     auto claim_next = [&]() -> long long {  // warp-uniform
         int c = 0;
         if (lane == 0) c = atomicAdd(&sm.claim, 1);
-        return g_lo + __shfl_sync(0xffffffffu, c, 0);
+        c = __shfl_sync(0xffffffffu, c, 0);
+        // interleaved (group c of CTA b = b + c * nact): a spatial cluster of rescans is
+        // spread over all CTAs instead of landing on one; contiguous with GP_MATCH_CONTIG=1
+        return a.interleave ? (long long)blockIdx.x + (long long)c * g_nact : g_lo + c;
     };
-    for (long long g = claim_next(); g < g_hi; g = claim_next()) {
+    for (long long g = claim_next(); g < (a.interleave ? ngroups : g_hi); g = claim_next()) {
         const long long base = g * 32 * kVL;
         int32_t u[kVL], p[kVL], s2[kVL], qq[kVL], rr[kVL], ps[kVL], pps[kVL];
         // level 1: the vertices; level 2: P_k[u] and the cached second candidate S[u]
@@ -467,30 +604,18 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
             wq_push(q, qn, Ln, &next->live, live[i], u[i]);
         }
     }
-    // CTA-aggregated final flush: one global atomic per CTA
-    if (lane == 0) sm.scratch[wib] = qn;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        int32_t tot = 0;
-        for (int w = 0; w < kNT / 32; ++w) {
-            const int32_t c = sm.scratch[w];
-            sm.scratch[w] = tot;
-            tot += c;
-        }
-        sm.scratch[kNT / 32] = tot ? atomicAdd(&next->live, tot) : 0;
-    }
-    __syncthreads();
-    {
-        const int32_t base = sm.scratch[kNT / 32] + sm.scratch[wib];
-        for (int i = lane; i < qn; i += 32) Ln[base + i] = q[i];
-    }
+    cta_flush(sm, q, qn, Ln, &next->live);
 }
 
 __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, unsigned long long &scanned,
                         unsigned long long &rows, unsigned long long &visits, int32_t &made) {
     (void)n;
-    if ((long long)len >= 4LL * g_nact * kNT) phase_k_impl<4>(a, sm, k, len, scanned, rows, visits, made);
-    else phase_k_impl<1>(a, sm, k, len, scanned, rows, visits, made);
+    const long long threads = (long long)g_nact * kNT;
+    if ((long long)len >= 4LL * threads) phase_k_impl<4>(a, sm, k, len, scanned, rows, visits, made);
+    else if (a.lanes_mode == 0 || (long long)len * 2 > threads) phase_k_impl<1>(a, sm, k, len, scanned, rows, visits, made);
+    else if ((long long)len * 8 <= threads) phase_k_lanes<8>(a, sm, k, len, scanned, rows, visits, made);
+    else if ((long long)len * 4 <= threads) phase_k_lanes<4>(a, sm, k, len, scanned, rows, visits, made);
+    else phase_k_lanes<2>(a, sm, k, len, scanned, rows, visits, made);
 }
 
 __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ MatchArgs a) {
@@ -524,6 +649,8 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
         }
     }
     int32_t rounds = 0, maximal = 0;
+    const int nact_all = g_nact;  // CTAs of this launch (g_nact drops to 1 in the tail)
+    bool tail = false;            // CTA 0 alone runs the remaining (short) rounds
     if (a.mode == kMatchWhole || a.mode == kMatchRound) {
         // kMatchWhole: the device-side round loop; kMatchRound: round a.k only (the sharded
         // driver exchanges the boundary proposals between launches and decides termination)
@@ -542,13 +669,15 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
             // any match this round: one flag store per CTA (only "> 0" is used)
             if (__syncthreads_or(made > 0) && threadIdx.x == 0) *(volatile int32_t *)&ctl->slot[k & 3].matches = 1;
             trace_mark(ctl->trace, tr++);
-            grid_barrier(ctl->bar, bar_epoch, g_nact);
+            if (tail) __syncthreads();  // one CTA: the block barrier orders the round
+            else grid_barrier(ctl->bar, bar_epoch, nact_all);
             trace_mark(ctl->trace, tr++);
             const int32_t nh = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].nhub;
             if (nh > 0) {
                 hub_phase(a, sm, nh, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1],
                           &ctl->slot[(k + 1) & 3].live, scanned);
-                grid_barrier(ctl->bar, bar_epoch, g_nact);
+                if (tail) __syncthreads();
+                else grid_barrier(ctl->bar, bar_epoch, nact_all);
             }
             if (a.mode == kMatchRound) break;
             if (*(volatile int32_t *)&ctl->slot[k & 3].matches > 0) ++rounds;
@@ -558,6 +687,20 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
                 break;
             }
             if (a.max_rounds > 0 && rounds >= a.max_rounds) break;
+            // short live list: the grid barriers (not the work) would dominate the remaining
+            // rounds, so CTA 0 finishes them alone; the others wait at the barrier below
+            if (!tail && nact_all > 1 && live <= a.tail_live) {
+                tail = true;
+                if (blockIdx.x != 0) break;
+                __syncthreads();
+                if (threadIdx.x == 0) g_nact = 1;
+                __syncthreads();
+            }
+        }
+        if (tail) {
+            __syncthreads();
+            if (threadIdx.x == 0) g_nact = nact_all;
+            grid_barrier(ctl->bar, bar_epoch, nact_all);  // CTA 0's rounds are done
         }
     }
     trace_mark(ctl->trace, tr++);
@@ -640,6 +783,26 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     a.leftover = leftover ? 1 : 0;
     a.G = choose_group(avg_deg_hint);
     a.vpc = match_vpc();
+    {
+        static int lm = -1;
+        if (lm < 0) {
+            const char *e = getenv("GP_MATCH_LANES");  // tuning knob (results never depend on it)
+            lm = e ? atoi(e) : 1;
+        }
+        a.lanes_mode = lm;
+        static int tl = -1;
+        if (tl < 0) {
+            const char *e = getenv("GP_TAIL_LIVE");  // tuning knob (results never depend on it)
+            tl = e ? atoi(e) : 2048;
+        }
+        a.tail_live = tl;
+        static int il = -1;
+        if (il < 0) {
+            const char *e = getenv("GP_MATCH_CONTIG");  // tuning knob (results never depend on it)
+            il = (e && atoi(e) == 1) ? 0 : 1;
+        }
+        a.interleave = il;
+    }
     {
         // vertices per chunk: ~80 % of a stage at the average degree, a multiple of the
         // number of vertex groups (kNT / G) so that no group pass runs mostly idle
