@@ -153,3 +153,25 @@ def coarsen_to(g: Dict, threshold: int, stall_ratio_pct: int = 95, max_levels: i
     if levels and levels[-1]["stop_reason"] == 0:
         levels[-1]["stop_reason"] = STOP_THRESHOLD if cur["n"] <= threshold else STOP_MAX_LEVELS
     return levels
+
+
+def project(levels: List[Dict], part_coarse, from_level: Optional[int] = None, to_level: int = 0) -> np.ndarray:
+    """Projection of un-coarsening (P12: "the coarser graph is projected back to the finer
+    graph by transferring the partition assignment of each vertex to the corresponding
+    vertices in the finer graph"; P20-P22: "each thread specify the partition labels of
+    the projected vertices in the finer graph by considering the CM array").
+
+    part_coarse labels the coarse graph produced by level `from_level` (default: the last
+    level, i.e. the coarsest graph).  Level by level, finest last:
+        part_l[u] = part_{l+1}[CM_l[u]]      for l = from_level, ..., to_level
+    Returns the labels of level `to_level`'s fine graph.  Plain numpy gathers, one level at
+    a time in the paper's order (coarse to fine).
+    """
+    if from_level is None:
+        from_level = len(levels) - 1
+    part = np.asarray(part_coarse, dtype=np.int64)
+    for l in range(from_level, to_level - 1, -1):
+        cm = np.asarray(levels[l]["cmap"], dtype=np.int64)
+        assert len(part) == levels[l]["n_coarse"]
+        part = part[cm]
+    return part.astype(np.int32)
