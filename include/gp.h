@@ -180,6 +180,19 @@ gp_status gp_hier_download_level(gp_hier h, int32_t i, gp_vid *h_match, gp_vid *
 gp_status gp_hier_download_coarse(gp_hier h, int32_t i, gp_vid *h_adjp, gp_vid *h_adjncy, gp_wgt *h_adjwgt,
                                   gp_wgt *h_vwgt, gp_vid *n_out, gp_vid *nnz_out);
 
+/* Projection of un-coarsening (P12 "the coarser graph is projected back to the finer graph
+ * by transferring the partition assignment of each vertex"; P20-P22 "by considering the CM
+ * array and saved pointer arrays"): labels of the coarse graph made by level from_level
+ * are carried down to level to_level's fine graph,
+ *     part_l[u] = part_{l+1}[CM_l[u]]   for l = from_level, ..., to_level
+ * in ONE kernel launch (no intermediate level's labels are written).
+ *   d_part_coarse  device int32[n_coarse of from_level] (any label values)
+ *   d_part_fine    device int32[n of to_level], caller-owned, written
+ * 0 <= to_level <= from_level < levels.  Asynchronous (context stream).  Single-GPU
+ * hierarchies only (GP_ERR_INVALID_ARG for sharded ones). */
+gp_status gp_project(gp_hier h, int32_t from_level, int32_t to_level, const gp_vid *d_part_coarse,
+                     gp_vid *d_part_fine);
+
 /* ---- sharded coarsening over several GPUs -------------------
  * Vertex ranges are sharded over the ranks of one node (one process per GPU).  Each rank
  * owns the contiguous global ids [v_begin, v_end) and holds their CSR rows with GLOBAL

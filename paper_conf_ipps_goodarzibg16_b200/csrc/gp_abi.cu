@@ -818,6 +818,26 @@ gp_status gp_hier_download_coarse(gp_hier h, int32_t i, gp_vid *h_adjp, gp_vid *
     GP_TRY_END
 }
 
+gp_status gp_project(gp_hier h, int32_t from_level, int32_t to_level, const gp_vid *d_part_coarse,
+                     gp_vid *d_part_fine) {
+    if (!tagged<Hier>(h, kTagHier) || to_level < 0 || from_level < to_level ||
+        from_level >= (int32_t)h->levels.size() || !d_part_coarse || !d_part_fine) {
+        set_error("gp_project: bad handle, level range or buffers");
+        return GP_ERR_INVALID_ARG;
+    }
+    GP_TRY_BEGIN
+    std::vector<const int32_t *> cms;
+    for (int32_t l = to_level; l <= from_level; ++l) {
+        if (!h->levels[l].pieces.empty()) {
+            set_error("gp_project: single-GPU hierarchies only");
+            return GP_ERR_INVALID_ARG;
+        }
+        cms.push_back(h->levels[l].cmap);
+    }
+    return enqueue_project(h->ctx, cms.data(), (int)cms.size(), h->levels[to_level].n, d_part_coarse, d_part_fine);
+    GP_TRY_END
+}
+
 gp_status gp_nccl_unique_id(void *out128) {
     if (!out128) return GP_ERR_INVALID_ARG;
     return dist_unique_id(out128);

@@ -245,6 +245,10 @@ size_t contract_tiles(int32_t n, int32_t nnz);
 
 gp_status graph_totals_and_validate(Ctx *ctx, const Graph *g, bool validate);
 
+// projection of un-coarsening (project.cu): cms = CM of levels to..from (fine to coarse)
+gp_status enqueue_project(Ctx *ctx, const int32_t *const *cms, int nlev, int32_t n, const int32_t *part_c,
+                          int32_t *part_f);
+
 // sharded path (dist.cu)
 gp_status dist_coarsen_to(Graph *g, const gp_coarsen_opts *opts, Hier **out);
 gp_status dist_comm_create_nccl(Ctx *ctx, const void *uid, int rank, int nranks);

@@ -86,6 +86,7 @@ _sig("gp_hier_level", ctypes.c_int, [_vp, _i32, ctypes.POINTER(Level)])
 _sig("gp_hier_download_level", ctypes.c_int, [_vp, _i32, _vp, _vp])
 _sig("gp_hier_download_coarse", ctypes.c_int, [_vp, _i32, _vp, _vp, _vp, _vp, _i32p, _i32p])
 _sig("gp_nccl_unique_id", ctypes.c_int, [_vp])
+_sig("gp_project", ctypes.c_int, [_vp, _i32, _i32, _vp, _vp])
 _sig("gp_ctx_create_dist", ctypes.c_int, [ctypes.c_int, _vp, _vp, ctypes.c_int, ctypes.c_int, ctypes.POINTER(_vp)])
 _sig("gp_ctx_create_loopback", ctypes.c_int, [ctypes.c_int, _vp, ctypes.c_int, ctypes.POINTER(_vp)])
 _sig("gp_ctx_dist_info", ctypes.c_int, [_vp, _i32p, _i32p])
@@ -346,6 +347,15 @@ class Hierarchy:
                "gp_hier_download_level")
         return m, c
 
+
+    def project(self, part_coarse: torch.Tensor, part_fine: torch.Tensor, from_level: Optional[int] = None,
+                to_level: int = 0) -> torch.Tensor:
+        """gp_project: labels of level from_level's coarse graph (default: the coarsest)
+        carried down to level to_level's fine graph, written into part_fine (device)."""
+        if from_level is None:
+            from_level = len(self) - 1
+        _check(_lib.gp_project(self.handle, from_level, to_level, _ptr(part_coarse), _ptr(part_fine)), "gp_project")
+        return part_fine
 
     def download_coarse(self, i: int) -> Dict[str, torch.Tensor]:
         """Coarse graph of level i as host int32 tensors (gp_hier_download_coarse): the whole
