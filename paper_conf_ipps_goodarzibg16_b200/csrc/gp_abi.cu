@@ -673,6 +673,13 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
                 for (int q = 1; q < 9; ++q)
                     fprintf(stderr, " %.1f", ct[q] && ct[q - 1] ? ((long long)ct[q] - (long long)ct[q - 1]) * 1e-3 : 0.0);
                 fprintf(stderr, " | gap to contract %.1f us\n", ct[0] && mt[1] ? ((long long)ct[0] - (long long)mt[0]) * 1e-3 : 0.0);
+                if (hd[l].match.lens[1]) {
+                    fprintf(stderr, "[gp]   per round (live | slowest warp us | rows rescanned thread / warp):");
+                    for (int k = 1; k < 16 && hd[l].match.lens[k]; ++k)
+                        fprintf(stderr, " [%d %.1f %d/%d]", hd[l].match.lens[k], hd[l].match.wmax[k] * 1e-3,
+                                hd[l].match.trows[k], hd[l].match.wrows[k]);
+                    fprintf(stderr, "\n");
+                }
             }
         }
     }

@@ -24,7 +24,7 @@ constexpr int kBlock = 256;  // threads per CTA of the streaming kernels
 // ---------------------------------------------------------------------------------------
 // device-side control blocks of one level (zeroed once per gp_coarsen_to call)
 // ---------------------------------------------------------------------------------------
-struct RoundSlot {
+struct alignas(16) RoundSlot {  // read as one 16-byte load
     int32_t live;     // live-list length of the round this slot belongs to
     int32_t nhub;     // hub rows waiting for the hub phase
     int32_t matches;  // matches made by the round's commit
@@ -42,6 +42,10 @@ struct MatchCtl {
     int32_t rounds, maximal;
     unsigned long long arcs_scanned, rows_scanned, live_visits;
     int32_t pad[2];
+    // GP_PROF=1 only: per round k < 16, the slowest warp's phase-k time (ns), the live-list
+    // length and the rows rescanned by a thread / by a whole warp
+    unsigned long long wmax[16];
+    int32_t lens[16], trows[16], wrows[16];
 };
 
 constexpr int kMaxContractCtas = 1024;  // grid cap of the contraction kernel

@@ -67,6 +67,7 @@ struct MatchArgs {
     int32_t lanes_mode;  // 1: short live lists use G lanes per vertex (phase_k_lanes)
     int32_t tail_live;   // live lists this short are finished by CTA 0 alone
     int32_t interleave;  // phase-k groups dealt to CTAs round-robin (1) or in contiguous ranges (0)
+    int32_t prof;        // GP_PROF=1: per-round slowest-warp times and rescan counts (MatchCtl)
     int32_t mode;  // kMatchWhole, or one launch per phase for the sharded path
     int32_t k;     // round of a kMatchRound launch
 };
@@ -82,11 +83,19 @@ struct MatchSmem {
     long long cid[kStages]; // chunk staged in the stage (claimed dynamically; >= nchunks: none)
     int32_t scratch[40];
     int32_t claim;  // phase-k group claims of this CTA
+    int32_t trows;  // GP_PROF: rows rescanned by this CTA's threads in the round
+    unsigned long long tmax;  // GP_PROF: slowest warp of this CTA in the round (ns)
     unsigned long long red[kNT / 32];
     unsigned long long cnt3[3][kNT / 32];
 };
 
 __device__ __forceinline__ int32_t ldcg(const int32_t *p) { return __ldcg(p); }
+__device__ __forceinline__ int4 ld_volatile_v4(const int4 *p) {
+    int4 v;
+    asm volatile("ld.volatile.global.v4.s32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p)
+                 : "memory");
+    return v;
+}
 
 // Warp-buffered list append (no CTA-wide synchronisation): the lanes with `pred` put `value`
 // into the warp's shared queue; a full queue is flushed with ONE global atomic and a
@@ -356,14 +365,20 @@ __device__ __forceinline__ void cta_flush(MatchSmem &sm, const int32_t *q, int32
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     if (lane == 0) sm.scratch[wib] = qn;
     __syncthreads();
-    if (threadIdx.x == 0) {
-        int32_t tot = 0;
-        for (int w = 0; w < kNT / 32; ++w) {
-            const int32_t c = sm.scratch[w];
-            sm.scratch[w] = tot;
-            tot += c;
+    if (wib == 0) {  // warp 0 scans the 16 queue lengths; one atomic for the CTA
+        const int32_t c = lane < kNT / 32 ? sm.scratch[lane] : 0;
+        int32_t inc = c;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const int32_t t = __shfl_up_sync(0xffffffffu, inc, off);
+            if (lane >= off) inc += t;
         }
-        sm.scratch[kNT / 32] = tot ? atomicAdd(counter, tot) : 0;
+        const int32_t tot = __shfl_sync(0xffffffffu, inc, 31);
+        int32_t base = 0;
+        if (lane == 0 && tot) base = atomicAdd(counter, tot);
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (lane < kNT / 32) sm.scratch[lane] = inc - c;
+        if (lane == 0) sm.scratch[kNT / 32] = base;
     }
     __syncthreads();
     const int32_t base = sm.scratch[kNT / 32] + sm.scratch[wib];
@@ -586,6 +601,7 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
                 const int src = __ffs(mm) - 1;
                 mm &= mm - 1;
                 const int32_t su = __shfl_sync(0xffffffffu, s, src), eu = __shfl_sync(0xffffffffu, e, src);
+                if (a.prof && lane == 0 && k < 16) atomicAdd(&a.ctl->wrows[k], 1);
                 unsigned long long key = 0, key2 = 0;
                 for (int32_t j = su + lane; j < eu; j += 32) {
                     const int32_t x = __ldg(a.adjncy + j);
@@ -610,12 +626,33 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
 __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, unsigned long long &scanned,
                         unsigned long long &rows, unsigned long long &visits, int32_t &made) {
     (void)n;
+    unsigned long long t0 = 0, rows0 = rows;
+    if (a.prof) {
+        if (threadIdx.x == 0) sm.tmax = 0;
+        __syncthreads();
+        t0 = globaltimer();
+    }
     const long long threads = (long long)g_nact * kNT;
     if ((long long)len >= 4LL * threads) phase_k_impl<4>(a, sm, k, len, scanned, rows, visits, made);
     else if (a.lanes_mode == 0 || (long long)len * 2 > threads) phase_k_impl<1>(a, sm, k, len, scanned, rows, visits, made);
     else if ((long long)len * 8 <= threads) phase_k_lanes<8>(a, sm, k, len, scanned, rows, visits, made);
     else if ((long long)len * 4 <= threads) phase_k_lanes<4>(a, sm, k, len, scanned, rows, visits, made);
     else phase_k_lanes<2>(a, sm, k, len, scanned, rows, visits, made);
+    if (a.prof && k < 16) {  // one shared atomic per warp, one global atomic per CTA
+        const unsigned long long dt = globaltimer() - t0;
+        const int32_t dr = warp_sum((int32_t)(rows - rows0));
+        if ((threadIdx.x & 31) == 0) {
+            atomicMax(&sm.tmax, dt);
+            if (dr) atomicAdd(&sm.trows, dr);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            atomicMax(&a.ctl->wmax[k], sm.tmax);
+            if (sm.trows) atomicAdd(&a.ctl->trows[k], sm.trows);
+            sm.trows = 0;
+            if (blockIdx.x == 0) a.ctl->lens[k] = len;
+        }
+    }
 }
 
 __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ MatchArgs a) {
@@ -651,6 +688,7 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
     int32_t rounds = 0, maximal = 0;
     const int nact_all = g_nact;  // CTAs of this launch (g_nact drops to 1 in the tail)
     bool tail = false;            // CTA 0 alone runs the remaining (short) rounds
+    int32_t known_len = -1;       // next round's live-list length, read at the end of a round
     if (a.mode == kMatchWhole || a.mode == kMatchRound) {
         // kMatchWhole: the device-side round loop; kMatchRound: round a.k only (the sharded
         // driver exchanges the boundary proposals between launches and decides termination)
@@ -663,7 +701,7 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
                 z->matches = 0;
                 z->claim = 0;
             }
-            const int32_t len = (k == 1) ? n : *(volatile int32_t *)&ctl->slot[k & 3].live;
+            const int32_t len = (k == 1) ? n : known_len >= 0 ? known_len : *(volatile int32_t *)&ctl->slot[k & 3].live;
             int32_t made = 0;
             phase_k(a, sm, n, k, len, scanned, rows, visits, made);
             // any match this round: one flag store per CTA (only "> 0" is used)
@@ -672,16 +710,21 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
             if (tail) __syncthreads();  // one CTA: the block barrier orders the round
             else grid_barrier(ctl->bar, bar_epoch, nact_all);
             trace_mark(ctl->trace, tr++);
-            const int32_t nh = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].nhub;
-            if (nh > 0) {
-                hub_phase(a, sm, nh, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1],
+            // the next slot {live, nhub} and this round's match flag: two independent loads
+            // in flight together (one L2 round trip instead of three)
+            const int4 nxt = ld_volatile_v4(reinterpret_cast<const int4 *>(&ctl->slot[(k + 1) & 3]));
+            const int32_t made_any = *(volatile int32_t *)&ctl->slot[k & 3].matches;
+            int32_t live = nxt.x;
+            if (nxt.y > 0) {
+                hub_phase(a, sm, nxt.y, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1],
                           &ctl->slot[(k + 1) & 3].live, scanned);
                 if (tail) __syncthreads();
                 else grid_barrier(ctl->bar, bar_epoch, nact_all);
+                live = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].live;  // hub rows may stay live
             }
             if (a.mode == kMatchRound) break;
-            if (*(volatile int32_t *)&ctl->slot[k & 3].matches > 0) ++rounds;
-            const int32_t live = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].live;
+            if (made_any > 0) ++rounds;
+            known_len = live;
             if (live == 0) {
                 maximal = 1;
                 break;
@@ -802,6 +845,12 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
             il = (e && atoi(e) == 1) ? 0 : 1;
         }
         a.interleave = il;
+        static int pf = -1;
+        if (pf < 0) {
+            const char *e = getenv("GP_PROF");
+            pf = (e && atoi(e) == 1) ? 1 : 0;
+        }
+        a.prof = pf;
     }
     {
         // vertices per chunk: ~80 % of a stage at the average degree, a multiple of the
