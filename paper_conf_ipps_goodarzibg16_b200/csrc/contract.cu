@@ -462,6 +462,7 @@ __device__ void phase_c1a(const ContractArgs &a, int32_t n, int nt1, int T1) {
 __device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, int nt1, int T1, int32_t ntiles2,
                           int32_t tb) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int tb_log = 31 - __clz(tb);
     const int t_lo = blockIdx.x * T1, t_hi = min(nt1, t_lo + T1);
     if (t_lo >= t_hi) return;
     int32_t pc = 0, pu = 0;
@@ -477,70 +478,62 @@ __device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, in
     pc += block_scan_list(sm, a.tagg1 + 2 * s_lo, 2, 0, s_hi - s_lo, pc, tpc);
     pu += block_scan_list(sm, a.tagg1 + 2 * s_lo, 2, 1, s_hi - s_lo, pu, tpu);
     for (int t = s_lo + wib; t < s_hi; t += kCW) {
-        // lane owns the contiguous vertices base + lane*8 .. +7 (scan order)
-        const long long base = (long long)t * kVW + (long long)lane * kCItems;
-        int32_t m[kCItems], d[kCItems];
-        int32_t cnt = 0, ubs = 0;
-        // counts: M first, then the degrees of leader and partner (loads hoisted per level)
-#pragma unroll
-        for (int i = 0; i < kCItems; ++i) m[i] = (base + i < n) ? __ldcg(a.M + base + i) : -2;
+        // step i of the tile covers the vertices tbase + i*32 + lane: every load and the CM
+        // store are coalesced; the scan runs step by step (ballot for the leader ranks, a
+        // warp scan for the upper bounds) with running totals
+        const long long tbase = (long long)t * kVW;
+        int32_t m[kCItems];
 #pragma unroll
         for (int i = 0; i < kCItems; ++i) {
-            const long long u = base + i;
+            const long long u = tbase + i * 32 + lane;
+            m[i] = u < n ? a.M[u] : -2;  // L1-cached: the grid barrier's acquire invalidated L1
+        }
+        int32_t su[kCItems], du[kCItems], sv[kCItems], dv[kCItems], vw[kCItems];
+#pragma unroll
+        for (int i = 0; i < kCItems; ++i) {
+            const long long u = tbase + i * 32 + lane;
             const bool lead = u < n && u <= m[i];
             const bool pair = u < n && u < m[i];
-            const int32_t v = pair ? m[i] : 0;
-            const int32_t a0 = lead ? __ldg(a.adjp + u) : 0, a1 = lead ? __ldg(a.adjp + u + 1) : 0;
-            const int32_t b0 = pair ? __ldg(a.adjp + v) : 0, b1 = pair ? __ldg(a.adjp + v + 1) : 0;
-            d[i] = (a1 - a0) + (b1 - b0);  // P20.s6-8
-            cnt += lead;
-            ubs += d[i];
+            su[i] = lead ? __ldg(a.adjp + u) : 0;
+            du[i] = lead ? __ldg(a.adjp + u + 1) : 0;
+            sv[i] = pair ? __ldg(a.adjp + m[i]) : 0;
+            dv[i] = pair ? __ldg(a.adjp + m[i] + 1) : 0;
+            vw[i] = (lead ? __ldg(a.vwgt + u) : 0) + (pair ? __ldg(a.vwgt + m[i]) : 0);  // P12.s27
         }
-        int32_t tc, tu;
-        int32_t c = tpc[t - s_lo] + warp_excl(cnt, tc);
-        int32_t o = tpu[t - s_lo] + warp_excl(ubs, tu);
+        int32_t c = tpc[t - s_lo], o = tpu[t - s_lo];
         if (t == 0 && lane == 0) a.tile_start[0] = 0;
-        if (t == nt1 - 1 && lane == 0) {
-            const int32_t nc = tpc[t - s_lo] + tc;
-            a.ctl->n_coarse = nc;
-            a.off[nc] = tpu[t - s_lo] + tu;  // = nnz
-            a.tile_start[ntiles2] = nc;
-        }
-        // stores in two halves; each half gathers everything it needs before any store
+        const unsigned lt = lanemask_lt();
 #pragma unroll
-        for (int h = 0; h < kCItems; h += kCItems / 2) {
-            int32_t su[kCItems / 2], ep[kCItems / 2], sv[kCItems / 2], vw[kCItems / 2];
-#pragma unroll
-            for (int q = 0; q < kCItems / 2; ++q) {
-                const int i = h + q;
-                const long long u = base + i;
-                const bool lead = u < n && u <= m[i];
-                const bool pair = u < n && u < m[i];
-                su[q] = lead ? __ldg(a.adjp + u) : 0;
-                ep[q] = lead ? __ldg(a.adjp + u + 1) : 0;
-                sv[q] = pair ? __ldg(a.adjp + m[i]) : 0;
-                vw[q] = (lead ? __ldg(a.vwgt + u) : 0) + (pair ? __ldg(a.vwgt + m[i]) : 0);  // P12.s27
-            }
-#pragma unroll
-        for (int q = 0; q < kCItems / 2; ++q) {
-            const int i = h + q;
-            const long long u = base + i;
-            if (u < n && u <= m[i]) {
+        for (int i = 0; i < kCItems; ++i) {
+            const long long u = tbase + i * 32 + lane;
+            const bool lead = u < n && u <= m[i];
+            const int32_t dl = du[i] - su[i];
+            const int32_t d = lead ? dl + (dv[i] - sv[i]) : 0;  // P20.s6-8
+            const unsigned bl = __ballot_sync(0xffffffffu, lead);
+            int32_t dtot;
+            const int32_t dex = warp_excl(d, dtot);
+            if (lead) {
+                const int32_t cc = c + __popc(bl & lt);  // exclusive scan = inclusive - 1 (P18.s20-24)
+                const int32_t oo = o + dex;
                 const int32_t v = m[i];
-                const int32_t dl = ep[q] - su[q];
-                a.CM[u] = c;              // exclusive scan = inclusive - 1 (P18.s20-24)
-                if (v != u) a.CM[v] = c;  // partner copies its leader's id (P18.s26)
-                a.cvwgt[c] = vw[q];
-                a.off[c] = o;
-                a.seg[c] = make_int4(su[q], dl, sv[q], d[i] - dl);
-                // warp tile t2 starts at the first row with off >= t2*tb: row c+1 for
-                // every t2 with off[c] < t2*tb <= off[c+1]
-                for (int32_t t2 = o / tb + 1; t2 <= (o + d[i]) / tb && t2 < ntiles2; ++t2) a.tile_start[t2] = c + 1;
-                if (d[i] > kWB) a.huge[atomicAdd(&a.ctl->n_huge, 1)] = c;
-                ++c;
-                o += d[i];
+                a.CM[u] = cc;
+                if (v != u) a.CM[v] = cc;  // partner copies its leader's id (P18.s26)
+                a.cvwgt[cc] = vw[i];
+                a.off[cc] = oo;
+                a.seg[cc] = make_int4(su[i], dl, sv[i], d - dl);
+                // C2 warp tile t2 starts at the first row with off >= t2*tb: row cc+1 for
+                // every t2 with oo < t2*tb <= oo + d (tb is a power of two)
+                for (int32_t t2 = (oo >> tb_log) + 1; t2 <= ((oo + d) >> tb_log) && t2 < ntiles2; ++t2)
+                    a.tile_start[t2] = cc + 1;
+                if (d > kWB) a.huge[atomicAdd(&a.ctl->n_huge, 1)] = cc;
             }
+            c += __popc(bl);
+            o += dtot;
         }
+        if (t == nt1 - 1 && lane == 0) {
+            a.ctl->n_coarse = c;
+            a.off[c] = o;  // = nnz
+            a.tile_start[ntiles2] = c;
         }
     }
     __syncthreads();  // the prefix arrays are rewritten by the next segment
