@@ -73,6 +73,8 @@ struct ContractArgs {
     // cbase + c; adjncy/adjwgt hold the local rows followed by the shipped partner rows; the
     // host takes the stop decision.  Single GPU: dist = 0, cbase = 0.
     int32_t dist, cbase, tb_fixed, nnz_ub;
+    int32_t prof;    // GP_PROF=1: slowest C2a warp tile (ctl->dbg)
+    int32_t tb_min;  // smallest C2 warp-tile budget (GP_TB_MIN tuning knob; results never depend on it)
 };
 
 struct ContractSmem {
@@ -609,6 +611,8 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
     for (int wt = (lane == 0) ? (int)atomicAdd(&a.ctl->tile_ctr, 1u) : 0;;) {
         wt = __shfl_sync(0xffffffffu, wt, 0);
         if (wt >= ntiles2) break;
+        const unsigned long long tt0 = a.prof ? globaltimer() : 0ull;
+        int32_t nw64 = 0;
         int32_t r0 = 0, r1 = 0;
         if (lane < 2) {
             const int32_t x = __ldcg(a.tile_start + wt + lane);
@@ -698,6 +702,7 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
             }
             // rows of 17..64 entries: the warp, registers + shuffles, keys from the slot
             unsigned m64 = __ballot_sync(0xffffffffu, c < r1 && ub > kNet && ub <= kWarpNet);
+            nw64 += __popc(m64);
             while (m64) {
                 const int src = __ffs(m64) - 1;
                 m64 &= m64 - 1;
@@ -765,6 +770,15 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
             }
             __syncwarp();
             run += part;
+        }
+        if (a.prof && lane == 0) {
+            const unsigned long long dt = globaltimer() - tt0;
+            atomicMax(&a.ctl->dbg[0], (dt << 32) | (unsigned)wt);
+            atomicMax(&a.ctl->dbg[1], ((unsigned long long)nw64 << 32) | (unsigned)wt);
+            atomicMax(&a.ctl->dbg[2], ((unsigned long long)(r1 - r0) << 32) | (unsigned)wt);
+            atomicAdd(&a.ctl->dbg[3], dt);
+            atomicAdd(&a.ctl->dbg[4], 1ull);
+            atomicAdd(&a.ctl->dbg[5], (unsigned long long)nw64);
         }
         if (lane == 0) {
             a.ttot[wt] = run;
@@ -864,7 +878,7 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
     const int T1 = (nt1 + g_cact - 1) / g_cact;            // C1b tiles per CTA
     // C2 warp-tile budget: kWB, halved (down to 32) while there are < 4 tiles per warp
     int32_t tb = kWB;
-    while (tb > 32 && (long long)nnz < 4LL * tb * g_cact * kCW) tb >>= 1;
+    while (tb > a.tb_min && (long long)nnz < 4LL * tb * g_cact * kCW) tb >>= 1;
     if (a.dist) tb = a.tb_fixed;
     const int32_t ntiles2 = nnz > 0 ? (nnz + tb - 1) / tb : 0;
     const int T2 = (ntiles2 + g_cact - 1) / g_cact;        // C2b tiles per CTA
@@ -997,6 +1011,22 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
     a.cbase = prm.cbase;
     a.tb_fixed = prm.tb;
     a.nnz_ub = prm.nnz_ub;
+    {
+        static int tm = -1;
+        if (tm < 0) {
+            const char *e = getenv("GP_TB_MIN");  // tuning knob (results never depend on it)
+            tm = e ? atoi(e) : 32;
+            if (tm < 32) tm = 32;
+            if (tm > kWB) tm = kWB;
+        }
+        a.tb_min = tm;
+        static int pf = -1;
+        if (pf < 0) {
+            const char *e = getenv("GP_PROF");
+            pf = (e && atoi(e) == 1) ? 1 : 0;
+        }
+        a.prof = pf;
+    }
     void *args[] = {&a};
     LaunchScope ls(ctx, GP_K_CONTRACT);
     GP_CUDA(cudaLaunchCooperativeKernel((const void *)k_contract_level, dim3(contract_grid(ctx)), dim3(kCNT), args,

@@ -673,6 +673,12 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
                 for (int q = 1; q < 9; ++q)
                     fprintf(stderr, " %.1f", ct[q] && ct[q - 1] ? ((long long)ct[q] - (long long)ct[q - 1]) * 1e-3 : 0.0);
                 fprintf(stderr, " | gap to contract %.1f us\n", ct[0] && mt[1] ? ((long long)ct[0] - (long long)mt[0]) * 1e-3 : 0.0);
+                if (hd[l].contract.dbg[4]) {
+                    const unsigned long long *d = hd[l].contract.dbg;
+                    fprintf(stderr, "[gp]   c2a tiles %llu: slowest %.1f us (tile %llu), mean %.2f us, max warp-merged rows %llu (tile %llu), max rows %llu, warp-merged rows %llu\n",
+                            d[4], (d[0] >> 32) * 1e-3, d[0] & 0xffffffffull, d[3] * 1e-3 / d[4], d[1] >> 32,
+                            d[1] & 0xffffffffull, d[2] >> 32, d[5]);
+                }
                 if (hd[l].match.lens[1]) {
                     fprintf(stderr, "[gp]   per round (live | slowest warp us | rows rescanned thread / warp):");
                     for (int k = 1; k < 16 && hd[l].match.lens[k]; ++k)
