@@ -842,7 +842,9 @@ __device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, i
 
 __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constant__ ContractArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    ContractSmem &sm = *reinterpret_cast<ContractSmem *>(((uintptr_t)smem_raw + 127) & ~(uintptr_t)127);
+    // 128-byte alignment by POINTER arithmetic on the __shared__ symbol: the compiler keeps the
+    // shared address space (LDS/STS/ATOMS); an integer round trip made every access generic
+    ContractSmem &sm = *reinterpret_cast<ContractSmem *>(smem_raw + ((128u - (unsigned)__cvta_generic_to_shared(smem_raw)) & 127u));
     ContractCtl *ctl = a.ctl;
     const volatile SizeRec *in = a.in;
     if (in->stop) {  // an earlier level ended the coarsening: propagate and leave

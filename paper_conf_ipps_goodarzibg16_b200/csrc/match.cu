@@ -38,7 +38,6 @@ constexpr int kNT = 512;            // threads per CTA of the persistent kernels
 constexpr int kStageArcs = 4096;    // arcs per TMA stage (adjncy + adjwgt = 32 KB)
 constexpr int kStages = 3;          // TMA pipeline depth of phase 0
 constexpr int kMaxVch = 1024;       // vertices per phase-0 chunk (adjp slice staged too)
-constexpr int kThreadDeg = 32;      // phase-k rescans up to this many arcs: one thread
 constexpr int kHubDeg = 4096;       // rows longer than this: one CTA each (hub phase)
 
 // CTAs taking part in this launch: min(grid, ceil(n / vpc)).  The host launches the full
@@ -336,28 +335,6 @@ __device__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool 
 // ---------------------------------------------------------------------------------------
 // phase k >= 1: commit of round k + proposals of round k+1 (lazy rescans)
 // ---------------------------------------------------------------------------------------
-// thread rescan of u's row (<= kThreadDeg arcs) in batches of 8 arcs: every dependent level
-// (arc -> M[x] -> P_k[x] -> P_k[P_k[x]]) is issued for the whole batch at once; top-2 kept
-__device__ __forceinline__ void rescan_thread(const MatchArgs &a, const int32_t *Pk, int32_t s, int32_t e,
-                                              unsigned long long &key, unsigned long long &key2) {
-    key = key2 = 0;
-    for (int32_t j0 = s; j0 < e; j0 += 8) {
-        int32_t x[8], w[8], px[8], pp[8];
-#pragma unroll
-        for (int b = 0; b < 8; ++b) {
-            x[b] = (j0 + b < e) ? __ldg(a.adjncy + j0 + b) : -1;
-            w[b] = (j0 + b < e) ? __ldg(a.adjwgt + j0 + b) : 0;
-        }
-#pragma unroll
-        for (int b = 0; b < 8; ++b) px[b] = (x[b] >= 0) ? ldcg(Pk + x[b]) : -1;
-#pragma unroll
-        for (int b = 0; b < 8; ++b) pp[b] = (px[b] >= 0) ? ldcg(Pk + px[b]) : -1;
-#pragma unroll
-        for (int b = 0; b < 8; ++b)
-            if (x[b] >= 0 && pp[b] != x[b]) top2_add(key, key2, pack_key(w[b], x[b]));
-    }
-}
-
 // CTA-aggregated final flush of the warps' list queues: one global atomic per CTA.  All
 // threads of the CTA call.
 __device__ __forceinline__ void cta_flush(MatchSmem &sm, const int32_t *q, int32_t qn, int32_t *list,
@@ -492,6 +469,158 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
     cta_flush(sm, q, qn, Ln, &next->live);
 }
 
+// Warp-cooperative rescan of every row of a phase-k group that needs one (lazy rescan,
+// DESIGN.md §4.2): the rows' arcs are flattened into one item space (warp scan of the
+// degrees) and each lane takes kFB items at a time, so the dependent loads of ALL rows
+// (arc -> P_k[x] -> P_k[P_k[x]]) are in flight together instead of one row after another.
+// Top-2 per row by shared-memory 64-bit atomicMax (keys are distinct: one per neighbour).
+// Rows longer than kHubDeg go to the hub list.  All 32 lanes call; fq lives in the phase-0
+// staging buffers (idle in phase k).
+constexpr int kFQ = 128;  // queue entries per warp (32 lanes x kVL <= 4)
+constexpr int kFB = 4;    // flat items per lane per batch
+struct FlatQ {
+    union {
+        struct {
+            unsigned long long k1[kFQ], k2[kFQ];  // top-2 keys (multi-batch: 64-bit CAS atomics)
+        };
+        struct {
+            uint32_t w1[kFQ], n1[kFQ], w2[kFQ], n2[kFQ];  // single batch: native 32-bit max on (w, ~v)
+        };
+    };
+    int32_t s[kFQ];
+    int32_t off[kFQ + 2];
+};
+static_assert(sizeof(FlatQ) * (kNT / 32) <= sizeof(int32_t) * ((kStages - 1) * kStageArcs + kStages * kStageArcs),
+              "flat rescan queues must fit the idle phase-0 buffers");
+
+template <int kVL>
+__device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, const int32_t *Pk, int32_t *Pn,
+                                            int32_t *Pkw, RoundSlot *next, const int32_t (&u)[kVL],
+                                            bool (&need)[kVL], bool (&live)[kVL], unsigned long long &scanned,
+                                            unsigned long long &rows) {
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    FlatQ &fq = *(reinterpret_cast<FlatQ *>(&sm.adj[1][0]) + wib);
+    int32_t rs[kVL], re[kVL], rpos[kVL];
+#pragma unroll
+    for (int i = 0; i < kVL; ++i) {  // row bounds of every vertex to rescan: one load level
+        rs[i] = re[i] = 0;
+        if (need[i]) {
+            rs[i] = __ldg(a.adjp + (u[i] - a.vbase));
+            re[i] = __ldg(a.adjp + (u[i] - a.vbase) + 1);
+        }
+    }
+    int32_t qn = 0, T = 0;
+#pragma unroll
+    for (int i = 0; i < kVL; ++i) {
+        int32_t d = need[i] ? re[i] - rs[i] : 0;
+        if (need[i]) ++rows;
+        if (need[i] && d > kHubDeg) {
+            a.H[atomicAdd(&next->nhub, 1)] = u[i];
+            need[i] = false;
+            d = 0;
+        }
+        const unsigned b = __ballot_sync(0xffffffffu, need[i]);
+        const int32_t inc = warp_incl_scan(d);
+        const int32_t tot = __shfl_sync(0xffffffffu, inc, 31);
+        rpos[i] = qn + __popc(b & lanemask_lt());
+        if (need[i]) {
+            fq.s[rpos[i]] = rs[i];
+            fq.off[rpos[i]] = T + inc - d;
+            scanned += (unsigned long long)d;
+        }
+        qn += __popc(b);
+        T += tot;
+    }
+    if (qn == 0) return;  // warp-uniform
+    const bool one = T <= 32 * kFB;  // every item in registers at once: top-1 and top-2 in one pass
+    for (int r = lane; r < qn; r += 32) {  // the union's active view
+        if (one) {
+            fq.w1[r] = fq.n1[r] = fq.w2[r] = fq.n2[r] = 0u;
+        } else {
+            fq.k1[r] = 0ull;
+            fq.k2[r] = 0ull;
+        }
+    }
+    __syncwarp();
+    for (int pass = 0; pass < (one ? 1 : 2); ++pass) {
+        for (int32_t b0 = 0; b0 < T; b0 += 32 * kFB) {
+            int32_t e[kFB], x[kFB], w[kFB], px[kFB];
+            unsigned long long key[kFB];
+#pragma unroll
+            for (int b = 0; b < kFB; ++b) {
+                const int32_t f = b0 + b * 32 + lane;
+                e[b] = -1;
+                x[b] = -1;
+                w[b] = 0;
+                if (f < T) {  // entry of item f: the last row with off <= f
+                    int32_t r = 0;
+#pragma unroll
+                    for (int step = kFQ / 2; step > 0; step >>= 1)
+                        if (r + step < qn && fq.off[r + step] <= f) r += step;
+                    e[b] = r;
+                    const int32_t j = fq.s[r] + (f - fq.off[r]);
+                    x[b] = __ldg(a.adjncy + j);
+                    w[b] = __ldg(a.adjwgt + j);
+                }
+            }
+#pragma unroll
+            for (int b = 0; b < kFB; ++b) px[b] = x[b] >= 0 ? ldcg(Pk + x[b]) : -1;
+#pragma unroll
+            for (int b = 0; b < kFB; ++b) {
+                const int32_t pp = px[b] >= 0 ? ldcg(Pk + px[b]) : -1;
+                key[b] = (x[b] >= 0 && pp != x[b]) ? pack_key(w[b], x[b]) : 0ull;  // x free after round k
+            }
+            if (one) {
+                // top-2 of (w, ~x) per row with native 32-bit shared atomics, field by field
+                // (a 64-bit shared atomicMax is a CAS loop): heaviest weight, then the lowest
+                // id at that weight; the same among the row's other keys
+                const uint32_t NOK = 0u;
+#pragma unroll
+                for (int b = 0; b < kFB; ++b)
+                    if (key[b]) atomicMax(&fq.w1[e[b]], (uint32_t)w[b]);
+                __syncwarp();
+#pragma unroll
+                for (int b = 0; b < kFB; ++b)
+                    if (key[b] && (uint32_t)w[b] == fq.w1[e[b]]) atomicMax(&fq.n1[e[b]], ~(uint32_t)x[b]);
+                __syncwarp();
+#pragma unroll
+                for (int b = 0; b < kFB; ++b) {
+                    const bool top = key[b] && (uint32_t)w[b] == fq.w1[e[b]] && ~(uint32_t)x[b] == fq.n1[e[b]];
+                    if (key[b] && !top) atomicMax(&fq.w2[e[b]], (uint32_t)w[b]);
+                    else key[b] = NOK;  // not a second-choice candidate
+                }
+                __syncwarp();
+#pragma unroll
+                for (int b = 0; b < kFB; ++b)
+                    if (key[b] && (uint32_t)w[b] == fq.w2[e[b]]) atomicMax(&fq.n2[e[b]], ~(uint32_t)x[b]);
+            } else if (pass == 0) {
+#pragma unroll
+                for (int b = 0; b < kFB; ++b)
+                    if (key[b]) atomicMax(&fq.k1[e[b]], key[b]);
+            } else {
+#pragma unroll
+                for (int b = 0; b < kFB; ++b)
+                    if (key[b] && key[b] != fq.k1[e[b]]) atomicMax(&fq.k2[e[b]], key[b]);
+            }
+        }
+        __syncwarp();
+    }
+#pragma unroll
+    for (int i = 0; i < kVL; ++i) {
+        if (need[i]) {
+            const int32_t r = rpos[i];
+            const unsigned long long k1 = one ? (((unsigned long long)fq.w1[r] << 32) | fq.n1[r]) : fq.k1[r];
+            const unsigned long long k2 = one ? (((unsigned long long)fq.w2[r] << 32) | fq.n2[r]) : fq.k2[r];
+            const int32_t bv = key_vertex(fq.w1[r] || !one ? k1 : 0ull);
+            Pn[u[i]] = bv;
+            a.S[u[i]] = key_vertex(!one || fq.w2[r] ? k2 : 0ull);
+            if (bv == kNone) Pkw[u[i]] = kNone;  // dead: NONE in both buffers
+            live[i] = bv != kNone;
+        }
+    }
+    __syncwarp();  // fq is rebuilt by the warp's next group
+}
+
 // kVL live vertices per lane per step: their dependent loads overlap.  4 on long lists, 1 on
 // short ones (a wide step would leave most warps idle).
 template <int kVL>
@@ -572,53 +701,10 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
         }
         bool live[kVL];
 #pragma unroll
-        for (int i = 0; i < kVL; ++i) {
-            live[i] = u[i] >= 0 && p[i] != kNone && !need[i];
-            int32_t s = 0, e = 0;
-            bool need_warp = false;
-            if (need[i]) {
-                s = __ldg(a.adjp + (u[i] - a.vbase));
-                e = __ldg(a.adjp + (u[i] - a.vbase) + 1);
-                ++rows;
-                if (e - s <= kThreadDeg) {
-                    unsigned long long key, key2;
-                    rescan_thread(a, Pk, s, e, key, key2);
-                    scanned += (unsigned long long)(e - s);
-                    const int32_t b = key_vertex(key);
-                    Pn[u[i]] = b;
-                    a.S[u[i]] = key_vertex(key2);
-                    if (b == kNone) Pkw[u[i]] = kNone;
-                    live[i] = b != kNone;
-                } else if (e - s <= kHubDeg) {
-                    need_warp = true;
-                } else {
-                    a.H[atomicAdd(&next->nhub, 1)] = u[i];
-                }
-            }
-            // medium rows: the whole warp rescans one row at a time
-            unsigned mm = __ballot_sync(0xffffffffu, need_warp);
-            while (mm) {
-                const int src = __ffs(mm) - 1;
-                mm &= mm - 1;
-                const int32_t su = __shfl_sync(0xffffffffu, s, src), eu = __shfl_sync(0xffffffffu, e, src);
-                if (a.prof && lane == 0 && k < 16) atomicAdd(&a.ctl->wrows[k], 1);
-                unsigned long long key = 0, key2 = 0;
-                for (int32_t j = su + lane; j < eu; j += 32) {
-                    const int32_t x = __ldg(a.adjncy + j);
-                    if (free_after(x, Pk)) top2_add(key, key2, pack_key(__ldg(a.adjwgt + j), x));
-                }
-                group_top2<32>(key, key2);
-                if (lane == src) {
-                    const int32_t b = key_vertex(key);
-                    Pn[u[i]] = b;
-                    a.S[u[i]] = key_vertex(key2);
-                    if (b == kNone) Pkw[u[i]] = kNone;
-                    live[i] = b != kNone;
-                    scanned += (unsigned long long)(eu - su);
-                }
-            }
-            wq_push(q, qn, Ln, &next->live, live[i], u[i]);
-        }
+        for (int i = 0; i < kVL; ++i) live[i] = u[i] >= 0 && p[i] != kNone && !need[i];
+        flat_rescan<kVL>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows);
+#pragma unroll
+        for (int i = 0; i < kVL; ++i) wq_push(q, qn, Ln, &next->live, live[i], u[i]);
     }
     cta_flush(sm, q, qn, Ln, &next->live);
 }
@@ -657,7 +743,9 @@ __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int
 
 __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ MatchArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    MatchSmem &sm = *reinterpret_cast<MatchSmem *>(((uintptr_t)smem_raw + 127) & ~(uintptr_t)127);
+    // 128-byte alignment by POINTER arithmetic on the __shared__ symbol: the compiler keeps the
+    // shared address space (LDS/STS/ATOMS); an integer round trip made every access generic
+    MatchSmem &sm = *reinterpret_cast<MatchSmem *>(smem_raw + ((128u - (unsigned)__cvta_generic_to_shared(smem_raw)) & 127u));
     MatchCtl *ctl = a.ctl;
     const volatile SizeRec *in = a.in;
     if (in->stop) return;  // an earlier level ended the coarsening: nothing to do
@@ -671,6 +759,7 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
         __syncthreads();
     }
     unsigned long long scanned = 0, rows = 0, visits = 0;
+    if (threadIdx.x == 0) sm.trows = 0;  // GP_PROF counter (published after the first barrier)
     unsigned bar_epoch = 0;  // grid barriers passed (thread 0)
     int tr = 0;
     if (a.mode == kMatchWhole || a.mode == kMatchPhase0) {

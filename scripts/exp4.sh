@@ -1,0 +1,9 @@
+M=paper_conf_ipps_goodarzibg16_b200/csrc/match.cu
+C=paper_conf_ipps_goodarzibg16_b200/csrc/contract.cu
+cp $M /tmp/m.cu; cp $C /tmp/c.cu
+run() { python -c "import __graft_entry__ as e; e.build()" > gpurun_out/build.log 2>&1 || { echo BUILD FAIL; return; }; timeout 60 python -u scripts/dbg_case.py 5000 10000 5 5 2>&1 | tail -1; timeout 60 python -u scripts/dbg_case.py 1000 8000 12 5 2>&1 | tail -1; }
+echo "== A current"; run
+echo "== B match generic smem"; sed -i 's|MatchSmem \&sm = \*reinterpret_cast<MatchSmem \*>(smem_raw + .*|MatchSmem \&sm = *reinterpret_cast<MatchSmem *>(((uintptr_t)smem_raw + 127) \& ~(uintptr_t)127);|' $M; grep -n "MatchSmem &sm" $M; run
+cp /tmp/m.cu $M
+echo "== C contract generic smem"; sed -i 's|ContractSmem \&sm = \*reinterpret_cast<ContractSmem \*>(smem_raw + .*|ContractSmem \&sm = *reinterpret_cast<ContractSmem *>(((uintptr_t)smem_raw + 127) \& ~(uintptr_t)127);|' $C; grep -n "ContractSmem &sm" $C; run
+cp /tmp/c.cu $C
