@@ -620,47 +620,43 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
         }
         r1 = __shfl_sync(0xffffffffu, r0, 1);
         r0 = __shfl_sync(0xffffffffu, r0, 0);
-        const int32_t tbase = wt * tb;  // slots: a row starting in the tile ends below tb + kWB <= 2kWB
         unsigned long long *out = a.tout + (r0 < r1 ? __ldcg(a.off + r0) : 0);
         int32_t run = 0;
         for (int32_t g0 = r0; g0 < r1; g0 += 32) {
             const int32_t c = g0 + lane;
-            int32_t ub = 0, slot = 0x7fffffff, cntc = 0;
+            int32_t ub = 0, cntc = 0;
             int4 sg = make_int4(0, 0, 0, 0);
             if (c < r1) {
                 const int32_t o0 = __ldcg(a.off + c);
-                slot = o0 - tbase;
                 ub = __ldcg(a.off + c + 1) - o0;
                 if (ub <= kWarpNet) sg = __ldcg(a.seg + c);
                 if (ub > kWB) cntc = __ldcg(a.cnt + c);  // merged by C1h
             }
-            // ---- stage the arcs of every row with ub <= 64 into its slot, coalesced: lane
-            // e of a step owns flat index idx; its row is the last lane with slot <= idx ----
+            // Positions in the warp's slot area: rows with ub <= 64 (staged) packed first, rows
+            // of 65..kWB entries after them; rows > kWB (C1h) take none.  Both sums are
+            // <= tb + kWB <= 2kWB: every such row starts inside this tile.
+            const bool srow = c < r1 && ub <= kWarpNet;
+            const bool mrow = c < r1 && ub > kWarpNet && ub <= kWB;
+            int32_t S, Mt;
+            const int32_t sp = warp_excl(srow ? ub : 0, S);
+            const int32_t sq = S + warp_excl(mrow ? ub : 0, Mt);
+            const int32_t slot = srow ? sp : sq;
+            // ---- staging, coalesced: each staged row writes its arc indices into its slots
+            // (the map), then lane e of a step owns flat slot idx: arc -> (adjncy, adjwgt)
+            // -> CM, and overwrites the slot with the key (cx << 32 | w) ----
+            if (srow) {
+                for (int32_t q = 0; q < sg.y; ++q) wb[sp + q] = (unsigned long long)(sg.x + q);
+                for (int32_t q = 0; q < sg.w; ++q) wb[sp + sg.y + q] = (unsigned long long)(sg.z + q);
+            }
+            __syncwarp();
             {
-                const int32_t lo = __shfl_sync(0xffffffffu, slot, 0);
-                int32_t hi = (c < r1 && ub <= kWarpNet) ? slot + ub : 0;  // staged rows only
-#pragma unroll
-                for (int off = 16; off > 0; off >>= 1) hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, off));
                 constexpr int kB = 8;  // steps per batch: all loads of a batch are in flight together
-                for (int32_t b0 = lo; b0 < hi; b0 += 32 * kB) {
-                    int32_t jj[kB], rc[kB], x[kB], w[kB], cx[kB];
+                for (int32_t b0 = 0; b0 < S; b0 += 32 * kB) {
+                    int32_t jj[kB], x[kB], w[kB], cx[kB];
 #pragma unroll
                     for (int k = 0; k < kB; ++k) {
                         const int32_t idx = b0 + k * 32 + lane;
-                        int r = 0;
-#pragma unroll
-                        for (int step = 16; step > 0; step >>= 1) {
-                            const int32_t sl = __shfl_sync(0xffffffffu, slot, r + step);
-                            if (sl <= idx) r += step;
-                        }
-                        const int32_t rs = __shfl_sync(0xffffffffu, slot, r);
-                        const int32_t rub = __shfl_sync(0xffffffffu, ub, r);
-                        const int32_t rsu = __shfl_sync(0xffffffffu, sg.x, r);
-                        const int32_t rdu = __shfl_sync(0xffffffffu, sg.y, r);
-                        const int32_t rsv = __shfl_sync(0xffffffffu, sg.z, r);
-                        const int32_t p = idx - rs;
-                        rc[k] = g0 + r;
-                        jj[k] = (idx < hi && p < rub && rub <= kWarpNet) ? ((p < rdu) ? rsu + p : rsv + (p - rdu)) : -1;
+                        jj[k] = idx < S ? (int32_t)wb[idx] : -1;
                     }
 #pragma unroll
                     for (int k = 0; k < kB; ++k) {
@@ -671,48 +667,26 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
                     for (int k = 0; k < kB; ++k) cx[k] = jj[k] >= 0 ? __ldcg(a.CM + x[k]) : 0;
 #pragma unroll
                     for (int k = 0; k < kB; ++k)
-                        if (jj[k] >= 0)  // collapsed edge dropped (R9)
-                            wb[b0 + k * 32 + lane] = (cx[k] != rc[k] + a.cbase) ? ckey(cx[k], w[k]) : kMaxKey;
+                        if (jj[k] >= 0) wb[b0 + k * 32 + lane] = ckey(cx[k], w[k]);
                 }
                 __syncwarp();
             }
-            if (c < r1 && ub > 0 && ub <= kNet) {
-                uint32_t kc[kNet];
-                int32_t kw[kNet];
-#pragma unroll
-                for (int i = 0; i < kNet; ++i) {
-                    const unsigned long long kv = (i < ub) ? wb[slot + i] : kMaxKey;
-                    kc[i] = (uint32_t)(kv >> 32);
-                    kw[i] = (int32_t)(uint32_t)kv;
-                }
-                cx_sort16(kc, kw);
-                uint32_t prev = 0xFFFFFFFFu;
-                int32_t acc = 0;
-#pragma unroll
-                for (int i = 0; i < kNet; ++i) {
-                    if (kc[i] == prev) {
-                        acc += kw[i];  // repeated coarse neighbour: weights summed (R8, P12.s28)
-                    } else {
-                        if (prev != 0xFFFFFFFFu) wb[slot + cntc++] = ckey((int32_t)prev, acc);
-                        prev = kc[i];
-                        acc = kw[i];
-                    }
-                }
-                if (prev != 0xFFFFFFFFu) wb[slot + cntc++] = ckey((int32_t)prev, acc);
-            }
-            // rows of 17..64 entries: the warp, registers + shuffles, keys from the slot
-            unsigned m64 = __ballot_sync(0xffffffffu, c < r1 && ub > kNet && ub <= kWarpNet);
+            const uint32_t self = (uint32_t)(c + a.cbase);  // the collapsed edge's coarse id (R9)
+            // rows of 17..64 entries: the warp, registers + shuffles, merged in place
+            unsigned m64 = __ballot_sync(0xffffffffu, srow && ub > kNet);
             nw64 += __popc(m64);
             while (m64) {
                 const int src = __ffs(m64) - 1;
                 m64 &= m64 - 1;
-                const int32_t sl = __shfl_sync(0xffffffffu, slot, src);
+                const int32_t sl = __shfl_sync(0xffffffffu, sp, src);
                 const int32_t rub = __shfl_sync(0xffffffffu, ub, src);
+                const uint32_t rself = __shfl_sync(0xffffffffu, self, src);
                 unsigned long long v[2];
 #pragma unroll
                 for (int r = 0; r < 2; ++r) {
                     const int32_t e = r * 32 + lane;
                     v[r] = (e < rub) ? wb[sl + e] : kMaxKey;
+                    if ((uint32_t)(v[r] >> 32) == rself) v[r] = kMaxKey;  // collapsed edge dropped
                 }
                 __syncwarp();
                 warp_sort64(v);
@@ -721,12 +695,12 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
                 if (lane == src) cntc = cc;
             }
             // rows of 65..kWB entries: the warp, shared-memory sort in the slot, compacted
-            unsigned mm = __ballot_sync(0xffffffffu, c < r1 && ub > kWarpNet && ub <= kWB);
+            unsigned mm = __ballot_sync(0xffffffffu, mrow);
             while (mm) {
                 const int src = __ffs(mm) - 1;
                 mm &= mm - 1;
                 const int32_t cw = __shfl_sync(0xffffffffu, c, src);
-                const int32_t sl = __shfl_sync(0xffffffffu, slot, src);
+                const int32_t sl = __shfl_sync(0xffffffffu, sq, src);
                 unsigned long long *keys = wb + sl;
                 if (lane == 0) sm.wlen[wib] = 0;
                 __syncwarp();
@@ -749,6 +723,33 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
                     __syncwarp();
                 }
                 if (lane == src) cntc = cc;
+            }
+            // rows of <= 16 entries: one thread, registers + odd-even merge network, written
+            // back compacted into the row's slots
+            if (srow && ub > 0 && ub <= kNet) {
+                uint32_t kc[kNet];
+                int32_t kw[kNet];
+#pragma unroll
+                for (int i = 0; i < kNet; ++i) {
+                    const unsigned long long kv = (i < ub) ? wb[sp + i] : kMaxKey;
+                    kc[i] = (uint32_t)(kv >> 32);
+                    kw[i] = (int32_t)(uint32_t)kv;
+                    if (kc[i] == self) kc[i] = 0xFFFFFFFFu;  // collapsed edge dropped (R9)
+                }
+                cx_sort16(kc, kw);
+                uint32_t prev = 0xFFFFFFFFu;
+                int32_t acc = 0;
+#pragma unroll
+                for (int i = 0; i < kNet; ++i) {
+                    if (kc[i] == prev) {
+                        acc += kw[i];  // repeated coarse neighbour: weights summed (R8, P12.s28)
+                    } else {
+                        if (prev != 0xFFFFFFFFu) wb[sp + cntc++] = ckey((int32_t)prev, acc);
+                        prev = kc[i];
+                        acc = kw[i];
+                    }
+                }
+                if (prev != 0xFFFFFFFFu) wb[sp + cntc++] = ckey((int32_t)prev, acc);
             }
             int32_t part;
             const int32_t ex = warp_excl(cntc, part);
