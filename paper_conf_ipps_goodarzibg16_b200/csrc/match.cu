@@ -489,6 +489,7 @@ struct FlatQ {
     };
     int32_t s[kFQ];
     int32_t off[kFQ + 2];
+    uint8_t own[32 * kFB];  // single batch: queue entry of every item (no search)
 };
 static_assert(sizeof(FlatQ) * (kNT / 32) <= sizeof(int32_t) * ((kStages - 1) * kStageArcs + kStages * kStageArcs),
               "flat rescan queues must fit the idle phase-0 buffers");
@@ -541,6 +542,14 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
             fq.k2[r] = 0ull;
         }
     }
+    if (one) {  // every queued row marks its items with its entry
+#pragma unroll
+        for (int i = 0; i < kVL; ++i)
+            if (need[i]) {
+                const int32_t o = fq.off[rpos[i]];
+                for (int32_t q = 0; q < re[i] - rs[i]; ++q) fq.own[o + q] = (uint8_t)rpos[i];
+            }
+    }
     __syncwarp();
     for (int pass = 0; pass < (one ? 1 : 2); ++pass) {
         for (int32_t b0 = 0; b0 < T; b0 += 32 * kFB) {
@@ -554,9 +563,13 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
                 w[b] = 0;
                 if (f < T) {  // entry of item f: the last row with off <= f
                     int32_t r = 0;
+                    if (one) {
+                        r = fq.own[f];
+                    } else {
 #pragma unroll
-                    for (int step = kFQ / 2; step > 0; step >>= 1)
-                        if (r + step < qn && fq.off[r + step] <= f) r += step;
+                        for (int step = kFQ / 2; step > 0; step >>= 1)
+                            if (r + step < qn && fq.off[r + step] <= f) r += step;
+                    }
                     e[b] = r;
                     const int32_t j = fq.s[r] + (f - fq.off[r]);
                     x[b] = __ldg(a.adjncy + j);
