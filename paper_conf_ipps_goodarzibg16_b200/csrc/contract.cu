@@ -1018,7 +1018,7 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
         static int tm = -1;
         if (tm < 0) {
             const char *e = getenv("GP_TB_MIN");  // tuning knob (results never depend on it)
-            tm = e ? atoi(e) : 32;
+            tm = e ? atoi(e) : 128;
             if (tm < 32) tm = 32;
             if (tm > kWB) tm = kWB;
         }

@@ -46,6 +46,8 @@ struct MatchCtl {
     // length and the rows rescanned by a thread / by a whole warp
     unsigned long long wmax[16];
     int32_t lens[16], trows[16], wrows[16];
+    // GP_PROF=1: round-k grid barrier: ~(first CTA arrival), last arrival, last release (ns)
+    unsigned long long barr[16][3];
 };
 
 constexpr int kMaxContractCtas = 1024;  // grid cap of the contraction kernel

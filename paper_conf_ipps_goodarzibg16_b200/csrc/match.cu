@@ -66,6 +66,7 @@ struct MatchArgs {
     int32_t lanes_mode;  // 1: short live lists use G lanes per vertex (phase_k_lanes)
     int32_t tail_live;   // live lists this short are finished by CTA 0 alone
     int32_t interleave;  // phase-k groups dealt to CTAs round-robin (1) or in contiguous ranges (0)
+    int32_t static_mode; // 1: small levels walk all vertices each round (no live list; GP_MATCH_STATIC=1)
     int32_t prof;        // GP_PROF=1: per-round slowest-warp times and rescan counts (MatchCtl)
     int32_t mode;  // kMatchWhole, or one launch per phase for the sharded path
     int32_t k;     // round of a kMatchRound launch
@@ -395,7 +396,8 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
         const long long idx = g * VPW + lane / G;
         int32_t u = idx < len ? ((k == 1) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
         const int32_t p = u >= 0 ? ldcg(Pk + u) : kNone;
-        const int32_t s2 = (u >= 0 && p != kNone) ? ldcg(a.S + u) : kNone;
+        const int32_t s2r = u >= 0 ? ldcg(a.S + u) : kNone;  // not predicated on p: same load level
+        const int32_t s2 = p != kNone ? s2r : kNone;
         const int32_t qq = p != kNone ? ldcg(Pk + p) : kNone;
         const int32_t ps = s2 != kNone ? ldcg(Pk + s2) : -1;
         const int32_t rr = (p != kNone && qq != u && qq >= 0) ? ldcg(Pk + qq) : -1;
@@ -636,7 +638,12 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
 
 // kVL live vertices per lane per step: their dependent loads overlap.  4 on long lists, 1 on
 // short ones (a wide step would leave most warps idle).
-template <int kVL>
+// kStatic (small levels, <= 2 vertices per thread): the round walks ALL vertices of the level
+// in place of the compacted live list; u is live iff M[u] is FREE and P_k[u] != NONE (matched
+// vertices keep their partner in P, dead ones NONE), read at the same level as P_k[u].  No list
+// load, no list append and no atomic with a return value on the round's critical path; the
+// next round's live count is a fire-and-forget reduction.
+template <int kVL, bool kStatic = false>
 __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t len, unsigned long long &scanned,
                              unsigned long long &rows, unsigned long long &visits, int32_t &made) {
     const int32_t *Pk = a.P[k & 1];
@@ -671,13 +678,17 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
             const long long idx = base + i * 32 + lane;
-            u[i] = idx < len ? ((k == 1) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
+            u[i] = idx < len ? ((kStatic || k == 1) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
         }
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
             p[i] = u[i] >= 0 ? ldcg(Pk + u[i]) : kNone;
-            s2[i] = (u[i] >= 0 && p[i] != kNone) ? ldcg(a.S + u[i]) : kNone;
+            s2[i] = u[i] >= 0 ? ldcg(a.S + u[i]) : kNone;  // not predicated on p: same load level
+            if (kStatic && u[i] >= 0 && k > 1 && ldcg(a.M + u[i]) != kFree) p[i] = kNone;  // matched: not live
         }
+#pragma unroll
+        for (int i = 0; i < kVL; ++i)
+            if (p[i] == kNone) s2[i] = kNone;
         // level 3: P_k[p] and P_k[s2] (freedom test of the cached candidate, P only)
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
@@ -716,14 +727,25 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
 #pragma unroll
         for (int i = 0; i < kVL; ++i) live[i] = u[i] >= 0 && p[i] != kNone && !need[i];
         flat_rescan<kVL>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows);
+        if (kStatic) {
 #pragma unroll
-        for (int i = 0; i < kVL; ++i) wq_push(q, qn, Ln, &next->live, live[i], u[i]);
+            for (int i = 0; i < kVL; ++i) qn += live[i] ? 1 : 0;  // live count only
+        } else {
+#pragma unroll
+            for (int i = 0; i < kVL; ++i) wq_push(q, qn, Ln, &next->live, live[i], u[i]);
+        }
     }
-    cta_flush(sm, q, qn, Ln, &next->live);
+    if (kStatic) {
+        const int32_t c = warp_sum(qn);
+        if (lane == 0 && c) atomicAdd(&next->live, c);  // result unused: a RED, no round trip
+    } else {
+        cta_flush(sm, q, qn, Ln, &next->live);
+    }
 }
 
-__device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, unsigned long long &scanned,
-                        unsigned long long &rows, unsigned long long &visits, int32_t &made) {
+__device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, bool stat,
+                        unsigned long long &scanned, unsigned long long &rows, unsigned long long &visits,
+                        int32_t &made) {
     (void)n;
     unsigned long long t0 = 0, rows0 = rows;
     if (a.prof) {
@@ -732,7 +754,10 @@ __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int
         t0 = globaltimer();
     }
     const long long threads = (long long)g_nact * kNT;
-    if ((long long)len >= 4LL * threads) phase_k_impl<4>(a, sm, k, len, scanned, rows, visits, made);
+    if (stat) {
+        if ((long long)len > threads) phase_k_impl<2, true>(a, sm, k, len, scanned, rows, visits, made);
+        else phase_k_impl<1, true>(a, sm, k, len, scanned, rows, visits, made);
+    } else if ((long long)len >= 4LL * threads) phase_k_impl<4>(a, sm, k, len, scanned, rows, visits, made);
     else if (a.lanes_mode == 0 || (long long)len * 2 > threads) phase_k_impl<1>(a, sm, k, len, scanned, rows, visits, made);
     else if ((long long)len * 8 <= threads) phase_k_lanes<8>(a, sm, k, len, scanned, rows, visits, made);
     else if ((long long)len * 4 <= threads) phase_k_lanes<4>(a, sm, k, len, scanned, rows, visits, made);
@@ -791,6 +816,8 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
     const int nact_all = g_nact;  // CTAs of this launch (g_nact drops to 1 in the tail)
     bool tail = false;            // CTA 0 alone runs the remaining (short) rounds
     int32_t known_len = -1;       // next round's live-list length, read at the end of a round
+    // small level: every round walks all vertices (kStatic), at most 2 per thread
+    const bool stat = a.mode == kMatchWhole && a.static_mode && (long long)n <= 2LL * nact_all * kNT;
     if (a.mode == kMatchWhole || a.mode == kMatchRound) {
         // kMatchWhole: the device-side round loop; kMatchRound: round a.k only (the sharded
         // driver exchanges the boundary proposals between launches and decides termination)
@@ -803,14 +830,24 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
                 z->matches = 0;
                 z->claim = 0;
             }
-            const int32_t len = (k == 1) ? n : known_len >= 0 ? known_len : *(volatile int32_t *)&ctl->slot[k & 3].live;
+            const int32_t len = (k == 1 || stat) ? n : known_len >= 0 ? known_len : *(volatile int32_t *)&ctl->slot[k & 3].live;
             int32_t made = 0;
-            phase_k(a, sm, n, k, len, scanned, rows, visits, made);
+            phase_k(a, sm, n, k, len, stat, scanned, rows, visits, made);
             // any match this round: one flag store per CTA (only "> 0" is used)
             if (__syncthreads_or(made > 0) && threadIdx.x == 0) *(volatile int32_t *)&ctl->slot[k & 3].matches = 1;
             trace_mark(ctl->trace, tr++);
+            const bool bprof = a.prof && k < 16 && !tail;
+            if (bprof) {
+                __syncthreads();
+                if (threadIdx.x == 0) {
+                    const unsigned long long t = globaltimer();
+                    atomicMax(&ctl->barr[k][0], ~t);
+                    atomicMax(&ctl->barr[k][1], t);
+                }
+            }
             if (tail) __syncthreads();  // one CTA: the block barrier orders the round
             else grid_barrier(ctl->bar, bar_epoch, nact_all);
+            if (bprof && threadIdx.x == 0) atomicMax(&ctl->barr[k][2], globaltimer());
             trace_mark(ctl->trace, tr++);
             // the next slot {live, nhub} and this round's match flag: two independent loads
             // in flight together (one L2 round trip instead of three)
@@ -834,7 +871,7 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
             if (a.max_rounds > 0 && rounds >= a.max_rounds) break;
             // short live list: the grid barriers (not the work) would dominate the remaining
             // rounds, so CTA 0 finishes them alone; the others wait at the barrier below
-            if (!tail && nact_all > 1 && live <= a.tail_live) {
+            if (!stat && !tail && nact_all > 1 && live <= a.tail_live) {
                 tail = true;
                 if (blockIdx.x != 0) break;
                 __syncthreads();
@@ -953,6 +990,12 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
             pf = (e && atoi(e) == 1) ? 1 : 0;
         }
         a.prof = pf;
+        static int sm = -1;
+        if (sm < 0) {
+            const char *e = getenv("GP_MATCH_STATIC");  // tuning knob (results never depend on it)
+            sm = (e && atoi(e) == 1) ? 1 : 0;  // measured neutral on C3 (3.41 ms both): off
+        }
+        a.static_mode = sm;
     }
     {
         // vertices per chunk: ~80 % of a stage at the average degree, a multiple of the
