@@ -41,7 +41,8 @@ constexpr int kCNT = 256;        // threads per CTA (4 co-resident CTAs per SM)
 constexpr int kCW = kCNT / 32;   // warps per CTA
 constexpr int kCItems = 8;       // vertices per lane of a C1 warp tile
 constexpr int kVW = 32 * kCItems;  // 256 vertices per C1 warp tile
-constexpr int kWB = kContractTileBudget;  // C2 warp-tile budget (upper-bound entries)
+constexpr int kWB = kContractTileBudget;  // C2: rows up to this bound merged by a warp (slot area 2*kWB)
+constexpr int kRT = 32;          // C2 warp tile: coarse rows (single GPU; 8..32, see k_contract_level)
 constexpr int kCtaRow = 4096;    // C1h: rows up to this bound are merged in shared memory
 constexpr int kNet = 16;         // one-thread merge capacity
 constexpr int kWarpNet = 64;     // one-warp register merge capacity
@@ -74,7 +75,6 @@ struct ContractArgs {
     // host takes the stop decision.  Single GPU: dist = 0, cbase = 0.
     int32_t dist, cbase, tb_fixed, nnz_ub;
     int32_t prof;    // GP_PROF=1: slowest C2a warp tile (ctl->dbg)
-    int32_t tb_min;  // smallest C2 warp-tile budget (GP_TB_MIN tuning knob; results never depend on it)
 };
 
 struct ContractSmem {
@@ -461,10 +461,8 @@ __device__ void phase_c1a(const ContractArgs &a, int32_t n, int nt1, int T1) {
 // ---------------------------------------------------------------------------------------
 // C1b: CM, cvwgt, off, seg, C2 warp-tile starts, huge rows
 // ---------------------------------------------------------------------------------------
-__device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, int nt1, int T1, int32_t ntiles2,
-                          int32_t tb) {
+__device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, int nt1, int T1) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    const int tb_log = 31 - __clz(tb);
     const int t_lo = blockIdx.x * T1, t_hi = min(nt1, t_lo + T1);
     if (t_lo >= t_hi) return;
     int32_t pc = 0, pu = 0;
@@ -503,7 +501,6 @@ __device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, in
             vw[i] = (lead ? __ldg(a.vwgt + u) : 0) + (pair ? __ldg(a.vwgt + m[i]) : 0);  // P12.s27
         }
         int32_t c = tpc[t - s_lo], o = tpu[t - s_lo];
-        if (t == 0 && lane == 0) a.tile_start[0] = 0;
         const unsigned lt = lanemask_lt();
 #pragma unroll
         for (int i = 0; i < kCItems; ++i) {
@@ -523,10 +520,6 @@ __device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, in
                 a.cvwgt[cc] = vw[i];
                 a.off[cc] = oo;
                 a.seg[cc] = make_int4(su[i], dl, sv[i], d - dl);
-                // C2 warp tile t2 starts at the first row with off >= t2*tb: row cc+1 for
-                // every t2 with oo < t2*tb <= oo + d (tb is a power of two)
-                for (int32_t t2 = (oo >> tb_log) + 1; t2 <= ((oo + d) >> tb_log) && t2 < ntiles2; ++t2)
-                    a.tile_start[t2] = cc + 1;
                 if (d > kWB) a.huge[atomicAdd(&a.ctl->n_huge, 1)] = cc;
             }
             c += __popc(bl);
@@ -535,7 +528,6 @@ __device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, in
         if (t == nt1 - 1 && lane == 0) {
             a.ctl->n_coarse = c;
             a.off[c] = o;  // = nnz
-            a.tile_start[ntiles2] = c;
         }
     }
     __syncthreads();  // the prefix arrays are rewritten by the next segment
@@ -599,7 +591,7 @@ __device__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
 // ---------------------------------------------------------------------------------------
 // C2a: warp tiles: merge every row, write the tile compacted to tout at its ub offset
 // ---------------------------------------------------------------------------------------
-__device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntiles2, int T2, int32_t tb) {
+__device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntiles2, int T2, int32_t nc, int32_t rt) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int gw = blockIdx.x * kCW + wib, nw = g_cact * kCW;
     unsigned long long *wb = sm.buf + wib * 2 * kWB;  // this warp's slots (2*kWB entries)
@@ -614,29 +606,39 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
         const unsigned long long tt0 = a.prof ? globaltimer() : 0ull;
         int32_t nw64 = 0;
         int32_t r0 = 0, r1 = 0;
-        if (lane < 2) {
-            const int32_t x = __ldcg(a.tile_start + wt + lane);
-            r0 = x;
+        if (a.dist) {  // sharded levels: tiles of <= tb upper-bound entries (dist.cu k_dc_tiles)
+            if (lane < 2) r0 = __ldcg(a.tile_start + wt + lane);
+            r1 = __shfl_sync(0xffffffffu, r0, 1);
+            r0 = __shfl_sync(0xffffffffu, r0, 0);
+        } else {  // rt (<= 32) consecutive coarse rows
+            r0 = wt * rt;
+            r1 = min(nc, r0 + rt);
         }
-        r1 = __shfl_sync(0xffffffffu, r0, 1);
-        r0 = __shfl_sync(0xffffffffu, r0, 0);
         unsigned long long *out = a.tout + (r0 < r1 ? __ldcg(a.off + r0) : 0);
         int32_t run = 0;
         for (int32_t g0 = r0; g0 < r1; g0 += 32) {
             const int32_t c = g0 + lane;
-            int32_t ub = 0, cntc = 0;
+            int32_t ub = 0, hcnt = 0;
             int4 sg = make_int4(0, 0, 0, 0);
             if (c < r1) {
                 const int32_t o0 = __ldcg(a.off + c);
                 ub = __ldcg(a.off + c + 1) - o0;
                 if (ub <= kWarpNet) sg = __ldcg(a.seg + c);
-                if (ub > kWB) cntc = __ldcg(a.cnt + c);  // merged by C1h
+                if (ub > kWB) hcnt = __ldcg(a.cnt + c);  // merged by C1h
             }
-            // Positions in the warp's slot area: rows with ub <= 64 (staged) packed first, rows
-            // of 65..kWB entries after them; rows > kWB (C1h) take none.  Both sums are
-            // <= tb + kWB <= 2kWB: every such row starts inside this tile.
-            const bool srow = c < r1 && ub <= kWarpNet;
-            const bool mrow = c < r1 && ub > kWarpNet && ub <= kWB;
+            // Passes over the 32 rows: a pass takes the next lanes whose slots (ub of rows
+            // <= kWB; C1h rows take none) fit the warp's 2kWB slot area -- one pass unless the
+            // rows are long.  The first lane of a pass always fits (ub <= kWB).
+            for (int32_t first = 0;;) {
+            const bool inr = c < r1 && lane >= first;
+            const int32_t used = warp_incl_scan((inr && ub <= kWB) ? ub : 0);  // all lanes: a shuffle scan
+            const bool act = inr && used <= 2 * kWB;
+            const unsigned pm = __ballot_sync(0xffffffffu, act);
+            int32_t cntc = (act && ub > kWB) ? hcnt : 0;
+            // Positions in the slot area: rows with ub <= 64 (staged) packed first, rows of
+            // 65..kWB entries after them.
+            const bool srow = act && ub <= kWarpNet;
+            const bool mrow = act && ub > kWarpNet && ub <= kWB;
             int32_t S, Mt;
             const int32_t sp = warp_excl(srow ? ub : 0, S);
             const int32_t sq = S + warp_excl(mrow ? ub : 0, Mt);
@@ -650,24 +652,43 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
             }
             __syncwarp();
             {
-                constexpr int kB = 8;  // steps per batch: all loads of a batch are in flight together
+                // two sweeps of up to 16 steps (512 slots: a whole pass) so that every load of
+                // a level is in flight together: (adjncy, adjwgt) -> slot as (x << 32 | w), then
+                // CM[x] replaces the slot's high word -> key (cx << 32 | w)
+                constexpr int kB = 16;
+                uint32_t *wb32 = reinterpret_cast<uint32_t *>(wb);
                 for (int32_t b0 = 0; b0 < S; b0 += 32 * kB) {
-                    int32_t jj[kB], x[kB], w[kB], cx[kB];
+                    int32_t x[kB], w[kB];
 #pragma unroll
                     for (int k = 0; k < kB; ++k) {
                         const int32_t idx = b0 + k * 32 + lane;
-                        jj[k] = idx < S ? (int32_t)wb[idx] : -1;
+                        const int32_t jj = idx < S ? (int32_t)wb32[2 * idx] : -1;
+                        x[k] = jj >= 0 ? __ldcs(a.adjncy + jj) : -1;
+                        w[k] = jj >= 0 ? __ldcs(a.adjwgt + jj) : 0;
                     }
 #pragma unroll
                     for (int k = 0; k < kB; ++k) {
-                        x[k] = jj[k] >= 0 ? __ldcs(a.adjncy + jj[k]) : 0;
-                        w[k] = jj[k] >= 0 ? __ldcs(a.adjwgt + jj[k]) : 0;
+                        const int32_t idx = b0 + k * 32 + lane;
+                        if (idx < S) {
+                            wb32[2 * idx] = (uint32_t)w[k];
+                            wb32[2 * idx + 1] = (uint32_t)x[k];
+                        }
+                    }
+                }
+                __syncwarp();
+                for (int32_t b0 = 0; b0 < S; b0 += 32 * kB) {
+                    int32_t cx[kB];
+#pragma unroll
+                    for (int k = 0; k < kB; ++k) {
+                        const int32_t idx = b0 + k * 32 + lane;
+                        const int32_t x = idx < S ? (int32_t)wb32[2 * idx + 1] : -1;
+                        cx[k] = x >= 0 ? __ldcg(a.CM + x) : 0;
                     }
 #pragma unroll
-                    for (int k = 0; k < kB; ++k) cx[k] = jj[k] >= 0 ? __ldcg(a.CM + x[k]) : 0;
-#pragma unroll
-                    for (int k = 0; k < kB; ++k)
-                        if (jj[k] >= 0) wb[b0 + k * 32 + lane] = ckey(cx[k], w[k]);
+                    for (int k = 0; k < kB; ++k) {
+                        const int32_t idx = b0 + k * 32 + lane;
+                        if (idx < S) wb32[2 * idx + 1] = (uint32_t)cx[k];
+                    }
                 }
                 __syncwarp();
             }
@@ -753,13 +774,13 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
             }
             int32_t part;
             const int32_t ex = warp_excl(cntc, part);
-            if (c < r1) {
+            if (act) {
                 a.lofs[c] = run + ex;
                 if (ub <= kWB)
                     for (int32_t j = 0; j < cntc; ++j) __stcs(out + run + ex + j, wb[slot + j]);
             }
             // rows merged by C1h: the warp copies them in
-            unsigned mh = __ballot_sync(0xffffffffu, c < r1 && ub > kWB);
+            unsigned mh = __ballot_sync(0xffffffffu, act && ub > kWB);
             while (mh) {
                 const int src = __ffs(mh) - 1;
                 mh &= mh - 1;
@@ -771,6 +792,9 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
             }
             __syncwarp();
             run += part;
+            first += __popc(pm);
+            if (first >= 32 || g0 + first >= r1) break;
+            }
         }
         if (a.prof && lane == 0) {
             const unsigned long long dt = globaltimer() - tt0;
@@ -792,7 +816,7 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
 // ---------------------------------------------------------------------------------------
 // C2b: cadjp + coalesced copy of the tiles of this CTA's chunk into the final CSR
 // ---------------------------------------------------------------------------------------
-__device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, int32_t ntiles2, int T2) {
+__device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, int32_t ntiles2, int T2, int32_t rt) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int t_lo = blockIdx.x * T2, t_hi = min(ntiles2, t_lo + T2);
     if (t_lo >= t_hi) return;
@@ -807,9 +831,14 @@ __device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, i
     for (int t = s_lo + wib; t < s_hi; t += kCW) {
         const int32_t p = tp[t - s_lo];
         int32_t r0 = 0, r1 = 0;
-        if (lane < 2) r0 = __ldcg(a.tile_start + t + lane);
-        r1 = __shfl_sync(0xffffffffu, r0, 1);
-        r0 = __shfl_sync(0xffffffffu, r0, 0);
+        if (a.dist) {
+            if (lane < 2) r0 = __ldcg(a.tile_start + t + lane);
+            r1 = __shfl_sync(0xffffffffu, r0, 1);
+            r0 = __shfl_sync(0xffffffffu, r0, 0);
+        } else {
+            r0 = t * rt;
+            r1 = min(nc, r0 + rt);
+        }
         const int32_t total = __ldcg(a.ttot + t);
         for (int32_t c = r0 + lane; c < r1; c += 32) a.cadjp[c] = p + __ldcg(a.lofs + c);
         if (r0 < r1) {
@@ -879,19 +908,13 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
     unsigned bar_epoch = 0;  // grid barriers passed (thread 0)
     const int nt1 = (n + kVW - 1) / kVW;
     const int T1 = (nt1 + g_cact - 1) / g_cact;            // C1b tiles per CTA
-    // C2 warp-tile budget: kWB, halved (down to 32) while there are < 4 tiles per warp
-    int32_t tb = kWB;
-    while (tb > a.tb_min && (long long)nnz < 4LL * tb * g_cact * kCW) tb >>= 1;
-    if (a.dist) tb = a.tb_fixed;
-    const int32_t ntiles2 = nnz > 0 ? (nnz + tb - 1) / tb : 0;
-    const int T2 = (ntiles2 + g_cact - 1) / g_cact;        // C2b tiles per CTA
     trace_mark(ctl->trace, 0);
     if (n > 0 && !a.dist) {
         phase_c1a(a, n, nt1, T1);
         trace_mark(ctl->trace, 1);
         grid_barrier(ctl->bar, bar_epoch, g_cact);
         trace_mark(ctl->trace, 2);
-        phase_c1b(a, sm, n, nt1, T1, ntiles2, tb);
+        phase_c1b(a, sm, n, nt1, T1);
         trace_mark(ctl->trace, 3);
         grid_barrier(ctl->bar, bar_epoch, g_cact);
     }
@@ -903,12 +926,19 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
         grid_barrier(ctl->bar, bar_epoch, g_cact);
     }
     trace_mark(ctl->trace, 5);
+    // C2 warp tiles: 32 consecutive coarse rows each (single GPU); sharded levels get tiles of
+    // <= tb_fixed upper-bound entries from dist.cu
+    // rows per single-GPU tile: 32 (full lanes in the row merges).  Halving it on small levels
+    // (more, shorter tiles) measured slower: the per-tile latency chain dominates there.
+    const int32_t rt = kRT;
+    const int32_t ntiles2 = nnz <= 0 ? 0 : a.dist ? (nnz + a.tb_fixed - 1) / a.tb_fixed : (nc + rt - 1) / rt;
+    const int T2 = (ntiles2 + g_cact - 1) / g_cact;  // C2b tiles (and chunk sums) per CTA
     if (ntiles2 > 0) {
-        phase_c2a(a, sm, ntiles2, T2, tb);
+        phase_c2a(a, sm, ntiles2, T2, nc, rt);
         trace_mark(ctl->trace, 6);
         grid_barrier(ctl->bar, bar_epoch, g_cact);
         trace_mark(ctl->trace, 7);
-        phase_c2b(a, sm, nc, ntiles2, T2);
+        phase_c2b(a, sm, nc, ntiles2, T2, rt);
     } else {  // no arcs: every coarse row is empty
         for (long long c = (long long)blockIdx.x * kCNT + threadIdx.x; c <= nc; c += (long long)g_cact * kCNT)
             a.cadjp[c] = 0;
@@ -974,7 +1004,8 @@ int contract_grid(Ctx *ctx) {
 }
 
 size_t contract_tiles(int32_t n, int32_t nnz) {
-    return (size_t)(nnz + 31) / 32 + 2 * ((size_t)(n + kVW - 1) / kVW) + 8;  // smallest budget: 32
+    // sharded tiles of >= 32 upper-bound entries, single-GPU tiles of kRT rows, C1 warp tiles
+    return (size_t)(nnz + 31) / 32 + (size_t)(n + 7) / 8 + 2 * ((size_t)(n + kVW - 1) / kVW) + 8;
 }
 
 gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *CM, Graph *cg, ContractCtl *ctl,
@@ -1015,14 +1046,6 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
     a.tb_fixed = prm.tb;
     a.nnz_ub = prm.nnz_ub;
     {
-        static int tm = -1;
-        if (tm < 0) {
-            const char *e = getenv("GP_TB_MIN");  // tuning knob (results never depend on it)
-            tm = e ? atoi(e) : 128;
-            if (tm < 32) tm = 32;
-            if (tm > kWB) tm = kWB;
-        }
-        a.tb_min = tm;
         static int pf = -1;
         if (pf < 0) {
             const char *e = getenv("GP_PROF");
