@@ -500,18 +500,11 @@ template <int kVL>
 __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, const int32_t *Pk, int32_t *Pn,
                                             int32_t *Pkw, RoundSlot *next, const int32_t (&u)[kVL],
                                             bool (&need)[kVL], bool (&live)[kVL], unsigned long long &scanned,
-                                            unsigned long long &rows) {
+                                            unsigned long long &rows, const int32_t (&rs)[kVL],
+                                            const int32_t (&re)[kVL]) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     FlatQ &fq = *(reinterpret_cast<FlatQ *>(&sm.adj[1][0]) + wib);
-    int32_t rs[kVL], re[kVL], rpos[kVL];
-#pragma unroll
-    for (int i = 0; i < kVL; ++i) {  // row bounds of every vertex to rescan: one load level
-        rs[i] = re[i] = 0;
-        if (need[i]) {
-            rs[i] = __ldg(a.adjp + (u[i] - a.vbase));
-            re[i] = __ldg(a.adjp + (u[i] - a.vbase) + 1);
-        }
-    }
+    int32_t rpos[kVL];
     int32_t qn = 0, T = 0;
 #pragma unroll
     for (int i = 0; i < kVL; ++i) {
@@ -680,10 +673,14 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
             const long long idx = base + i * 32 + lane;
             u[i] = idx < len ? ((kStatic || k == 1) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
         }
+        int32_t rs[kVL], re[kVL];  // row bounds, loaded speculatively with P_k[u]: a rescan
+                                   // then starts one dependent level earlier
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
             p[i] = u[i] >= 0 ? ldcg(Pk + u[i]) : kNone;
             s2[i] = u[i] >= 0 ? ldcg(a.S + u[i]) : kNone;  // not predicated on p: same load level
+            rs[i] = u[i] >= 0 ? __ldg(a.adjp + (u[i] - a.vbase)) : 0;
+            re[i] = u[i] >= 0 ? __ldg(a.adjp + (u[i] - a.vbase) + 1) : 0;
             if (kStatic && u[i] >= 0 && k > 1 && ldcg(a.M + u[i]) != kFree) p[i] = kNone;  // matched: not live
         }
 #pragma unroll
@@ -726,7 +723,7 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
         bool live[kVL];
 #pragma unroll
         for (int i = 0; i < kVL; ++i) live[i] = u[i] >= 0 && p[i] != kNone && !need[i];
-        flat_rescan<kVL>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows);
+        flat_rescan<kVL>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re);
         if (kStatic) {
 #pragma unroll
             for (int i = 0; i < kVL; ++i) qn += live[i] ? 1 : 0;  // live count only
