@@ -595,12 +595,11 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int gw = blockIdx.x * kCW + wib, nw = g_cact * kCW;
     unsigned long long *wb = sm.buf + wib * 2 * kWB;  // this warp's slots (2*kWB entries)
-    (void)gw;
-    (void)nw;
     // warp tiles are claimed dynamically from one global counter: the merge cost of a tile
     // varies (row mix, C1h copies), and a static split per CTA leaves barrier tails
     // (measured: +30 % on the phase at small levels)
-    for (int wt = (lane == 0) ? (int)atomicAdd(&a.ctl->tile_ctr, 1u) : 0;;) {
+    // (the first tile of a warp is static -- tile gw -- so no claim round trip precedes it)
+    for (int wt = gw;;) {
         wt = __shfl_sync(0xffffffffu, wt, 0);
         if (wt >= ntiles2) break;
         const unsigned long long tt0 = a.prof ? globaltimer() : 0ull;
@@ -808,7 +807,7 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
         if (lane == 0) {
             a.ttot[wt] = run;
             atomicAdd(&a.ctl->chunk2[wt / T2], run);
-            wt = (int)atomicAdd(&a.ctl->tile_ctr, 1u);
+            wt = nw + (int)atomicAdd(&a.ctl->tile_ctr, 1u);
         }
     }
 }

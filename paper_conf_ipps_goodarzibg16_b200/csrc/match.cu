@@ -215,16 +215,21 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
     if (t == 0) {
         for (int q = 0; q < kStages; ++q) mbar_init(&sm.bar[q], 1);
         fence_mbar_init();
+        // the first kStages chunks of a CTA are static (b, b + nact, b + 2 nact): their bounds
+        // load in parallel and no claim atomic precedes the first TMA (a chain of 3 claims +
+        // bounds held the first copies back by ~8 us, the whole phase on small levels);
+        // later chunks are claimed dynamically beyond 3 nact -- per CTA still in increasing order
+        int32_t cs[kStages], ce[kStages];
+#pragma unroll
+        for (int q = 0; q < kStages; ++q)
+            load_bounds(a, n, nchunks, (long long)blockIdx.x + (long long)q * g_nact, cs[q], ce[q]);
+#pragma unroll
         for (int q = 0; q < kStages; ++q) {
-            const long long c = atomicAdd(&a.ctl->chunk_ctr, 1u);
+            const long long c = (long long)blockIdx.x + (long long)q * g_nact;
             sm.cid[q] = c;
-            if (c < nchunks) {
-                int32_t cs, ce;
-                load_bounds(a, n, nchunks, c, cs, ce);
-                stage_chunk(a, sm, n, c, cs, ce, q);
-            }
+            if (c < nchunks) stage_chunk(a, sm, n, c, cs[q], ce[q], q);
         }
-        nxt = atomicAdd(&a.ctl->chunk_ctr, 1u);
+        nxt = (long long)kStages * g_nact + atomicAdd(&a.ctl->chunk_ctr, 1u);
         load_bounds(a, n, nchunks, nxt, nb_s, nb_e);
     }
     __syncthreads();
@@ -289,7 +294,7 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
             sm.cid[st] = nxt;
             if (nxt < nchunks) {
                 stage_chunk(a, sm, n, nxt, nb_s, nb_e, st);
-                nxt = atomicAdd(&a.ctl->chunk_ctr, 1u);
+                nxt = (long long)kStages * g_nact + atomicAdd(&a.ctl->chunk_ctr, 1u);
                 load_bounds(a, n, nchunks, nxt, nb_s, nb_e);  // in flight during the next chunk
             }
         }
@@ -397,6 +402,8 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
         int32_t u = idx < len ? ((k == 1) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
         const int32_t p = u >= 0 ? ldcg(Pk + u) : kNone;
         const int32_t s2r = u >= 0 ? ldcg(a.S + u) : kNone;  // not predicated on p: same load level
+        const int32_t rs0 = u >= 0 ? __ldg(a.adjp + (u - a.vbase)) : 0;  // speculative row bounds
+        const int32_t re0 = u >= 0 ? __ldg(a.adjp + (u - a.vbase) + 1) : 0;
         const int32_t s2 = p != kNone ? s2r : kNone;
         const int32_t qq = p != kNone ? ldcg(Pk + p) : kNone;
         const int32_t ps = s2 != kNone ? ldcg(Pk + s2) : -1;
@@ -426,8 +433,8 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
         }
         int32_t s = 0, e = 0;
         if (need) {
-            s = __ldg(a.adjp + (u - a.vbase));
-            e = __ldg(a.adjp + (u - a.vbase) + 1);
+            s = rs0;
+            e = re0;
             if (e - s > kHubDeg) {
                 if (gl == 0) a.H[atomicAdd(&next->nhub, 1)] = u;
                 need = false;
