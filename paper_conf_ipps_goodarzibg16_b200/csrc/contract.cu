@@ -375,6 +375,87 @@ __device__ __forceinline__ int32_t warp_runmerge64(const unsigned long long (&v)
     return __popc(b0) + __popc(b1);
 }
 
+// Half-warp (16-lane segment) version for rows of 17..32 entries: two rows per warp step.
+// Element e = r*16 + l of a segment lives in v[r] of segment lane l; same flip-bitonic
+// network (15 stages instead of 21) and segmented run merge.  `out` is this segment's row.
+__device__ __forceinline__ void seg_sort32(unsigned long long (&v)[2]) {
+    const int l = threadIdx.x & 15;
+#pragma unroll
+    for (int size = 2; size <= 32; size <<= 1) {
+        if (size == 32) {  // mirrored step across the two registers
+            const unsigned long long o0 = __shfl_xor_sync(0xffffffffu, v[1], 15, 16);
+            const unsigned long long o1 = __shfl_xor_sync(0xffffffffu, v[0], 15, 16);
+            v[0] = v[0] < o0 ? v[0] : o0;
+            v[1] = v[1] > o1 ? v[1] : o1;
+        } else {
+            const bool lower = (l & (size >> 1)) == 0;
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const unsigned long long o = __shfl_xor_sync(0xffffffffu, v[r], size - 1, 16);
+                v[r] = lower ? (v[r] < o ? v[r] : o) : (v[r] > o ? v[r] : o);
+            }
+        }
+#pragma unroll
+        for (int j = size / 4; j > 0; j >>= 1) {
+            const bool lower = (l & j) == 0;
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const unsigned long long o = __shfl_xor_sync(0xffffffffu, v[r], j, 16);
+                v[r] = lower ? (v[r] < o ? v[r] : o) : (v[r] > o ? v[r] : o);
+            }
+        }
+    }
+}
+
+__device__ __forceinline__ int32_t seg_runmerge32(const unsigned long long (&v)[2], unsigned long long *out) {
+    const int lane = threadIdx.x & 31, l = lane & 15;
+    const unsigned seg = (lane & 16) ? 0xFFFF0000u : 0x0000FFFFu;
+    uint32_t cx[2], w[2];
+    bool head[2], tail[2];
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {
+        cx[r] = (uint32_t)(v[r] >> 32);
+        w[r] = (uint32_t)v[r];
+    }
+    const uint32_t prev0 = __shfl_up_sync(0xffffffffu, cx[0], 1, 16);
+    const uint32_t prev1 = __shfl_up_sync(0xffffffffu, cx[1], 1, 16);
+    const uint32_t last0 = __shfl_sync(0xffffffffu, cx[0], 15, 16);
+    const uint32_t next0 = __shfl_down_sync(0xffffffffu, cx[0], 1, 16);
+    const uint32_t next1 = __shfl_down_sync(0xffffffffu, cx[1], 1, 16);
+    const uint32_t first1 = __shfl_sync(0xffffffffu, cx[1], 0, 16);
+    head[0] = l == 0 || prev0 != cx[0];
+    head[1] = (l == 0) ? (last0 != cx[1]) : (prev1 != cx[1]);
+    tail[0] = (l == 15) ? (first1 != cx[0]) : (next0 != cx[0]);
+    tail[1] = l == 15 || next1 != cx[1];
+    uint32_t sum[2];
+    bool seen[2];
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {
+        uint32_t val = w[r];
+        bool f = head[r];
+#pragma unroll
+        for (int off = 1; off < 16; off <<= 1) {
+            const uint32_t tv = __shfl_up_sync(0xffffffffu, val, off, 16);
+            const bool tf = __shfl_up_sync(0xffffffffu, f ? 1 : 0, off, 16);
+            if (l >= off) {
+                if (!f) val += tv;
+                f = f || tf;
+            }
+        }
+        sum[r] = val;
+        seen[r] = f;
+    }
+    const uint32_t carry = __shfl_sync(0xffffffffu, sum[0], 15, 16);
+    if (!seen[1]) sum[1] += carry;
+    const bool e0 = tail[0] && cx[0] != 0xFFFFFFFFu;
+    const bool e1 = tail[1] && cx[1] != 0xFFFFFFFFu;
+    const unsigned b0 = __ballot_sync(0xffffffffu, e0) & seg, b1 = __ballot_sync(0xffffffffu, e1) & seg;
+    const unsigned lt = lanemask_lt();
+    if (e0) out[__popc(b0 & lt)] = ((unsigned long long)cx[0] << 32) | sum[0];
+    if (e1) out[__popc(b0) + __popc(b1 & lt)] = ((unsigned long long)cx[1] << 32) | sum[1];
+    return __popc(b0) + __popc(b1);
+}
+
 // ---------------------------------------------------------------------------------------
 // block-wide helpers (all threads call)
 // ---------------------------------------------------------------------------------------
@@ -692,8 +773,38 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
                 __syncwarp();
             }
             const uint32_t self = (uint32_t)(c + a.cbase);  // the collapsed edge's coarse id (R9)
-            // rows of 17..64 entries: the warp, registers + shuffles, merged in place
-            unsigned m64 = __ballot_sync(0xffffffffu, srow && ub > kNet);
+            // rows of 17..32 entries: two at a time, one per half-warp, merged in place
+            unsigned m32 = __ballot_sync(0xffffffffu, srow && ub > kNet && ub <= 2 * kNet);
+            nw64 += __popc(m32);
+            while (m32) {
+                const int sa = __ffs(m32) - 1;
+                m32 &= m32 - 1;
+                const int sb = m32 ? __ffs(m32) - 1 : -1;
+                if (sb >= 0) m32 &= m32 - 1;
+                const int src = (lane & 16) ? sb : sa;  // this half-warp's row (-1: idle)
+                const int s0 = src < 0 ? sa : src;
+                const int32_t sl = __shfl_sync(0xffffffffu, sp, s0);
+                const int32_t rub0 = __shfl_sync(0xffffffffu, ub, s0);  // all lanes shuffle
+                const int32_t rub = src < 0 ? 0 : rub0;
+                const uint32_t rself = __shfl_sync(0xffffffffu, self, s0);
+                unsigned long long v[2];
+#pragma unroll
+                for (int r = 0; r < 2; ++r) {
+                    const int32_t e = r * 16 + (lane & 15);
+                    v[r] = (e < rub) ? wb[sl + e] : kMaxKey;
+                    if ((uint32_t)(v[r] >> 32) == rself) v[r] = kMaxKey;  // collapsed edge dropped
+                }
+                __syncwarp();
+                seg_sort32(v);
+                unsigned long long dummy[1];
+                const int32_t cc = seg_runmerge32(v, src < 0 ? dummy : wb + sl);  // idle half: all padding
+                __syncwarp();
+                const int32_t cca = __shfl_sync(0xffffffffu, cc, 0), ccb = __shfl_sync(0xffffffffu, cc, 16);
+                if (lane == sa) cntc = cca;  // the owners may sit in either half
+                if (lane == sb) cntc = ccb;
+            }
+            // rows of 33..64 entries: the warp, registers + shuffles, merged in place
+            unsigned m64 = __ballot_sync(0xffffffffu, srow && ub > 2 * kNet);
             nw64 += __popc(m64);
             while (m64) {
                 const int src = __ffs(m64) - 1;
