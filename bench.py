@@ -35,8 +35,8 @@ WORKLOADS = {
     "C1": ("grid64x64_unit", 100),
     "C2": ("rgg_n2^20_deg13_w1-100", 100),
     "C3": ("delaunay_like_n2^22_w1-100", 100),
-    "C4": ("rmat_s24_ef16_w1-100", 100),
-    "C5": ("road_like_n2^26_deg2.5_w1-100", 100),
+    "C4": ("rmat_s24_ef16_w1-4", 100),
+    "C5": ("road_like_n2^26_deg2.5_w1-10", 100),
 }
 METRIC = "fine edges coarsened/sec (sum of |E| over levels / full coarsen-to-threshold time)"
 UNIT = "edges/s"

@@ -632,21 +632,129 @@ __device__ __forceinline__ void gather_row(const ContractArgs &a, int32_t c, int
 }
 
 // ---------------------------------------------------------------------------------------
+// Long rows (> kCtaRow keys, R-MAT hubs): runs of kCtaRow keys are sorted in shared memory,
+// then merged pairwise through global memory (merge path, windows of kMW outputs staged in
+// shared memory; the window split points of a batch are searched by all threads at once).
+// A bitonic network over global memory (the earlier design) paid ~log^2 dependent passes.
+// ---------------------------------------------------------------------------------------
+constexpr int kMW = kBuf / 2;  // outputs per merge window (A and B pieces staged side by side)
+
+// number of A elements among the first d outputs of merge(A, B) (A first on ties)
+__device__ __forceinline__ int32_t merge_path(const unsigned long long *A, int32_t la, const unsigned long long *B,
+                                              int32_t lb, int32_t d) {
+    int32_t lo = max(0, d - lb), hi = min(d, la);
+    while (lo < hi) {
+        const int32_t mid = (lo + hi) >> 1;
+        if (A[mid] <= B[d - mid - 1]) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+// CTA merge of sorted A[0, la) and B[0, lb) into O (all global); all threads call
+__device__ void cta_merge(ContractSmem &sm, const unsigned long long *A, int32_t la, const unsigned long long *B,
+                          int32_t lb, unsigned long long *O) {
+    const int tid = threadIdx.x;
+    const int32_t m = la + lb;
+    int32_t *split = sm.lead;  // lead[] and has[] are adjacent: kCNT + 1 split points fit
+    const int32_t nwin = (m + kMW - 1) / kMW;
+    for (int32_t wb0 = 0; wb0 < nwin; wb0 += kCNT) {
+        const int32_t nbw = min(kCNT, nwin - wb0);
+        for (int t = tid; t <= nbw; t += kCNT) split[t] = merge_path(A, la, B, lb, min(m, (wb0 + t) * kMW));
+        __syncthreads();
+        for (int32_t w = 0; w < nbw; ++w) {
+            const int32_t d0 = (wb0 + w) * kMW, d1 = min(m, d0 + kMW);
+            const int32_t i0 = split[w], i1 = split[w + 1], j0 = d0 - i0, j1 = d1 - i1;
+            const int32_t na = i1 - i0, nb = j1 - j0;
+            for (int32_t t = tid; t < na; t += kCNT) sm.buf[t] = A[i0 + t];
+            for (int32_t t = tid; t < nb; t += kCNT) sm.buf[kMW + t] = B[j0 + t];
+            __syncthreads();
+            constexpr int kPer = kMW / kCNT;
+            const int32_t dl = tid * kPer;
+            if (dl < na + nb) {
+                const unsigned long long *sa = sm.buf, *sb = sm.buf + kMW;
+                int32_t i = merge_path(sa, na, sb, nb, dl), j = dl - i;
+#pragma unroll
+                for (int k = 0; k < kPer; ++k) {
+                    if (dl + k < na + nb) {
+                        const bool ta = j >= nb || (i < na && sa[i] <= sb[j]);
+                        O[d0 + dl + k] = ta ? sa[i] : sb[j];
+                        i += ta ? 1 : 0;
+                        j += ta ? 0 : 1;
+                    }
+                }
+            }
+            __syncthreads();
+        }
+    }
+}
+
+// sort keys[0, len) (global) in place; tmp: len entries of global scratch
+__device__ __noinline__ void cta_sort_long(ContractSmem &sm, unsigned long long *keys, unsigned long long *tmp, int32_t len) {
+    const int tid = threadIdx.x;
+    for (int32_t r0 = 0; r0 < len; r0 += kCtaRow) {  // sorted runs of kCtaRow keys
+        const int32_t rl = min(kCtaRow, len - r0);
+        for (int32_t t = tid; t < rl; t += kCNT) sm.buf[t] = keys[r0 + t];
+        __syncthreads();
+        coop_sort(sm.buf, rl, tid, kCNT, []() { __syncthreads(); });
+        for (int32_t t = tid; t < rl; t += kCNT) keys[r0 + t] = sm.buf[t];
+        __syncthreads();
+    }
+    unsigned long long *src = keys, *dst = tmp;
+    for (int32_t run = kCtaRow; run < len; run *= 2) {
+        for (int32_t a0 = 0; a0 < len; a0 += 2 * run) {
+            const int32_t la = min(run, len - a0), lb = max(0, min(run, len - a0 - la));
+            cta_merge(sm, src + a0, la, src + a0 + la, lb, dst + a0);
+        }
+        unsigned long long *x = src;
+        src = dst;
+        dst = x;
+    }
+    if (src != keys) {
+        for (int32_t t = tid; t < len; t += kCNT) keys[t] = src[t];
+    }
+    __syncthreads();
+}
+
+// ---------------------------------------------------------------------------------------
 // C1h: rows with ub > kWB, one CTA each; result compacted at gkeys[off[c]], count cnt[c]
 // ---------------------------------------------------------------------------------------
-__device__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
+__device__ __noinline__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
     for (int i = blockIdx.x; i < nh; i += g_cact) {
         const int32_t c = a.huge[i];
         const int32_t o0 = __ldcg(a.off + c);
         const int32_t ub = __ldcg(a.off + c + 1) - o0;
         unsigned long long *dst = a.gkeys + o0;
         unsigned long long *keys = (ub <= kCtaRow) ? sm.buf : dst;
-        if (threadIdx.x == 0) sm.len = 0;
-        __syncthreads();
-        gather_row(a, c, threadIdx.x, kCNT, keys, [&]() { return atomicAdd(&sm.len, 1); });
-        __syncthreads();
-        const int len = sm.len;
-        coop_sort(keys, len, threadIdx.x, kCNT, []() { __syncthreads(); });
+        // gather at fixed positions (leader's arcs, then the partner's; 4 per thread in flight);
+        // the collapsed edge becomes kMaxKey, sorts last and is cut off (no claim atomics)
+        const int4 sg = __ldcg(a.seg + c);
+        int32_t nself = 0, dummy = 0;
+        for (int32_t p0 = threadIdx.x; p0 < ub; p0 += 4 * kCNT) {
+            int32_t x[4], w[4], cx[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int32_t p = p0 + q * kCNT;
+                const int32_t j = p < sg.y ? sg.x + p : sg.z + (p - sg.y);
+                x[q] = p < ub ? __ldcs(a.adjncy + j) : -1;
+                w[q] = p < ub ? __ldcs(a.adjwgt + j) : 0;
+            }
+#pragma unroll
+            for (int q = 0; q < 4; ++q) cx[q] = x[q] >= 0 ? __ldcg(a.CM + x[q]) : 0;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int32_t p = p0 + q * kCNT;
+                if (p < ub) {
+                    const bool self = cx[q] == c + a.cbase;  // collapsed edge dropped (R9)
+                    keys[p] = self ? kMaxKey : ckey(cx[q], w[q]);
+                    nself += self ? 1 : 0;
+                }
+            }
+        }
+        block_sum2(sm, nself, dummy);  // (syncs: the keys are complete)
+        const int len = ub - nself;
+        if (ub <= kCtaRow) coop_sort(keys, ub, threadIdx.x, kCNT, []() { __syncthreads(); });
+        else cta_sort_long(sm, keys, a.tout + o0, ub);  // tout is idle until C2a
         const int32_t cnt = coop_runsum(
             keys, len, threadIdx.x, kCNT, sm.lead, sm.has,
             [&](int32_t v, int32_t &tot) { return block_excl_scan<kCNT>(v, sm.scan, tot); },

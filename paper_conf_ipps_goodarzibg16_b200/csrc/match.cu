@@ -38,7 +38,7 @@ constexpr int kNT = 512;            // threads per CTA of the persistent kernels
 constexpr int kStageArcs = 4096;    // arcs per TMA stage (adjncy + adjwgt = 32 KB)
 constexpr int kStages = 3;          // TMA pipeline depth of phase 0
 constexpr int kMaxVch = 1024;       // vertices per phase-0 chunk (adjp slice staged too)
-constexpr int kHubDeg = 4096;       // rows longer than this: one CTA each (hub phase)
+constexpr int kHubDeg = 1024;       // rows longer than this: hub phase (chunks over all CTAs)
 
 // CTAs taking part in this launch: min(grid, ceil(n / vpc)).  The host launches the full
 // persistent grid before the level's size is known; the level's kernel retires the CTAs a
@@ -53,6 +53,7 @@ struct MatchArgs {
     int32_t *L[2];
     int32_t *H;  // hub list of the pending hub phase
     int32_t *S;  // second-heaviest neighbour of the last full scan (NONE = none cached)
+    unsigned long long *hk;  // multi-CTA hub phase: best key per listed hub (the contraction's idle gkeys)
     MatchCtl *ctl;
     int32_t max_rounds;
     int32_t leftover;
@@ -268,9 +269,19 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
             } else if (valid) {
                 if (e - s > kHubDeg) {
                     hub = true;
-                } else {
-                    for (int32_t j = s + gl; j < e; j += G)
-                        top2_add(key, key2, pack_key(__ldg(a.adjwgt + j), __ldg(a.adjncy + j)));
+                } else {  // 8 arcs per lane per batch, all loads in flight together
+                    for (int32_t j0 = s + gl; j0 < e; j0 += 8 * G) {
+                        int32_t xv[8], wv[8];
+#pragma unroll
+                        for (int q = 0; q < 8; ++q) {
+                            const int32_t j = j0 + q * G;
+                            xv[q] = j < e ? __ldg(a.adjncy + j) : -1;
+                            wv[q] = j < e ? __ldg(a.adjwgt + j) : 0;
+                        }
+#pragma unroll
+                        for (int q = 0; q < 8; ++q)
+                            if (xv[q] >= 0) top2_add(key, key2, pack_key(wv[q], xv[q]));
+                    }
                 }
             }
             group_top2_rt(key, key2, G);
@@ -278,7 +289,9 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
                 const int32_t x = a.vbase + (int32_t)v;  // row v is vertex vbase + v
                 a.M[x] = kFree;
                 if (hub) {
-                    a.H[atomicAdd(&a.ctl->slot[1].nhub, 1)] = x;
+                    const int32_t h = atomicAdd(&a.ctl->slot[1].nhub, 1);
+                    a.H[h] = x;
+                    if (a.hk) a.hk[h] = 0ull;  // (sharded launches: per-CTA hub_phase, no hk)
                     a.S[x] = kNone;
                 } else {
                     const int32_t p = key_vertex(key);
@@ -306,7 +319,7 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
 // hub phase: every listed row (deg > kHubDeg) is scanned by a whole CTA
 // kCheck = false in round 1 (every vertex free), true for rescans after round k.
 // ---------------------------------------------------------------------------------------
-__device__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool check, const int32_t *Pk,
+__device__ __noinline__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool check, const int32_t *Pk,
                           int32_t *Pn, int32_t *Lnext, int32_t *live_next, unsigned long long &scanned) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     for (int i = blockIdx.x; i < nhub; i += g_nact) {
@@ -335,6 +348,96 @@ __device__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool 
             scanned += (unsigned long long)(e - s);
         }
         __syncthreads();
+    }
+}
+
+// Multi-CTA hub phase (kMatchWhole): the listed rows are cut into chunks of kHC arcs and the
+// chunks are dealt round-robin to all CTAs, so a 400 K-arc R-MAT hub is scanned by ~100 CTAs
+// at once instead of one (each thread: 8 arcs, all loads of a level in flight).  Each chunk's
+// best key goes to hk[hub] by a 64-bit global atomicMax; after a grid barrier the hubs'
+// proposals are written (top-1 only: S = NONE for hubs, as in hub_phase).  Every CTA walks the
+// hub list in segments of kNT hubs with a block scan of the chunk counts.
+constexpr int kHC = kNT * 8;  // arcs per hub chunk
+__device__ __noinline__ void hub_phase_mc(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool check, const int32_t *Pk,
+                             int32_t *Pn, int32_t *Lnext, int32_t *live_next, unsigned long long &scanned,
+                             unsigned *bar, unsigned &bar_epoch, int nact) {
+    const int t = threadIdx.x, lane = t & 31, wib = t >> 5;
+    int32_t *hs = reinterpret_cast<int32_t *>(&sm.adj[0][0]);  // per segment: row start, end, chunk base
+    int32_t *he = hs + kNT, *hb = he + kNT;
+    long long carry = 0;  // chunks of earlier segments
+    for (int32_t seg = 0; seg < nhub; seg += kNT) {
+        const int32_t i = seg + t;
+        int32_t rs = 0, re = 0, ch = 0;
+        if (i < nhub) {
+            const int32_t u = a.H[i];
+            rs = __ldg(a.adjp + (u - a.vbase));
+            re = __ldg(a.adjp + (u - a.vbase) + 1);
+            ch = (re - rs + kHC - 1) / kHC;
+            if (blockIdx.x == 0) scanned += (unsigned long long)(re - rs);
+        }
+        int32_t tot;
+        const int32_t ex = block_excl_scan<kNT>(ch, sm.scratch, tot);
+        hs[t] = rs;
+        he[t] = re;
+        hb[t] = ex;
+        __syncthreads();
+        const int32_t nseg = min(kNT, nhub - seg);
+        // global chunk g = carry + local; this CTA takes g = b (mod nact)
+        long long g0 = carry + (((long long)blockIdx.x - carry) % nact + nact) % nact;
+        for (long long g = g0; g < carry + tot; g += nact) {
+            const int32_t loc = (int32_t)(g - carry);
+            int32_t r = 0;  // hub of chunk loc: the last with hb <= loc
+            for (int step = kNT / 2; step > 0; step >>= 1)
+                if (r + step < nseg && hb[r + step] <= loc) r += step;
+            const int32_t c0 = hs[r] + (loc - hb[r]) * kHC, c1 = min(he[r], c0 + kHC);
+            int32_t x[8], w[8], px[8];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const int32_t j = c0 + q * kNT + t;
+                x[q] = j < c1 ? __ldg(a.adjncy + j) : -1;
+                w[q] = j < c1 ? __ldg(a.adjwgt + j) : 0;
+            }
+            unsigned long long key = 0;
+            if (check) {
+#pragma unroll
+                for (int q = 0; q < 8; ++q) px[q] = x[q] >= 0 ? ldcg(Pk + x[q]) : -1;
+#pragma unroll
+                for (int q = 0; q < 8; ++q) {
+                    const int32_t pp = px[q] >= 0 ? ldcg(Pk + px[q]) : -1;
+                    if (x[q] >= 0 && pp != x[q]) key = umax64(key, pack_key(w[q], x[q]));  // x free after round k
+                }
+            } else {
+#pragma unroll
+                for (int q = 0; q < 8; ++q)
+                    if (x[q] >= 0) key = umax64(key, pack_key(w[q], x[q]));
+            }
+            key = group_max64<32>(key);
+            if (lane == 0) sm.red[wib] = key;
+            __syncthreads();
+            if (t == 0) {
+                unsigned long long k = 0;
+                for (int q = 0; q < kNT / 32; ++q) k = umax64(k, sm.red[q]);
+                if (k) atomicMax(&a.hk[seg + r], k);
+            }
+            __syncthreads();
+        }
+        carry += tot;
+        __syncthreads();  // hs/he/hb are rewritten by the next segment
+    }
+    grid_barrier(bar, bar_epoch, nact);
+    // finalize: one thread per hub
+    for (long long i = (long long)blockIdx.x * kNT + t; i < nhub; i += (long long)nact * kNT) {
+        const int32_t u = a.H[i];
+        const unsigned long long k = __ldcg(a.hk + i);
+        const int32_t p = key_vertex(k);
+        Pn[u] = p;
+        a.S[u] = kNone;
+        if (p == kNone) {
+            a.P[0][u] = kNone;
+            a.P[1][u] = kNone;
+        } else if (Lnext) {
+            Lnext[atomicAdd(live_next, 1)] = u;
+        }
     }
 }
 
@@ -436,7 +539,11 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
             s = rs0;
             e = re0;
             if (e - s > kHubDeg) {
-                if (gl == 0) a.H[atomicAdd(&next->nhub, 1)] = u;
+                if (gl == 0) {
+                    const int32_t h = atomicAdd(&next->nhub, 1);
+                    a.H[h] = u;
+                    if (a.hk) a.hk[h] = 0ull;  // (sharded launches: per-CTA hub_phase, no hk)
+                }
                 need = false;
                 e = s;
             } else if (gl == 0) {
@@ -518,7 +625,9 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
         int32_t d = need[i] ? re[i] - rs[i] : 0;
         if (need[i]) ++rows;
         if (need[i] && d > kHubDeg) {
-            a.H[atomicAdd(&next->nhub, 1)] = u[i];
+            const int32_t h = atomicAdd(&next->nhub, 1);
+            a.H[h] = u[i];
+            if (a.hk) a.hk[h] = 0ull;  // (sharded launches: per-CTA hub_phase, no hk)
             need[i] = false;
             d = 0;
         }
@@ -812,8 +921,12 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
         trace_mark(ctl->trace, tr++);
         const int32_t nh = *(volatile int32_t *)&ctl->slot[1].nhub;
         if (nh > 0) {
-            hub_phase(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned);
-            if (a.mode == kMatchWhole) grid_barrier(ctl->bar, bar_epoch, g_nact);
+            if (a.mode == kMatchWhole) {
+                hub_phase_mc(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned, ctl->bar, bar_epoch, g_nact);
+                grid_barrier(ctl->bar, bar_epoch, g_nact);
+            } else {
+                hub_phase(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned);
+            }
         }
     }
     int32_t rounds = 0, maximal = 0;
@@ -859,8 +972,12 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
             const int32_t made_any = *(volatile int32_t *)&ctl->slot[k & 3].matches;
             int32_t live = nxt.x;
             if (nxt.y > 0) {
-                hub_phase(a, sm, nxt.y, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1],
-                          &ctl->slot[(k + 1) & 3].live, scanned);
+                if (a.mode == kMatchWhole && !tail)
+                    hub_phase_mc(a, sm, nxt.y, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1],
+                                 &ctl->slot[(k + 1) & 3].live, scanned, ctl->bar, bar_epoch, nact_all);
+                else
+                    hub_phase(a, sm, nxt.y, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1],
+                              &ctl->slot[(k + 1) & 3].live, scanned);
                 if (tail) __syncthreads();
                 else grid_barrier(ctl->bar, bar_epoch, nact_all);
                 live = *(volatile int32_t *)&ctl->slot[(k + 1) & 3].live;  // hub rows may stay live
@@ -964,6 +1081,7 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     a.L[1] = lb.L[1];
     a.H = lb.H;
     a.S = lb.S;
+    a.hk = lb.gkeys;  // idle while a level matches (the contraction's hub-row scratch, >= nnz keys)
     a.ctl = ctl;
     a.max_rounds = max_rounds;
     a.leftover = leftover ? 1 : 0;
