@@ -716,6 +716,57 @@ __device__ __noinline__ void cta_sort_long(ContractSmem &sm, unsigned long long 
     __syncthreads();
 }
 
+// Run-sum + compaction of a sorted long row keys[0, len) (global) in place, window by window
+// through shared memory: each window's runs are summed and compacted in smem, the window's
+// last run is held back (it may continue into the next window) and the rest is written at
+// the row's compacted position (always <= the window start: no unread key is overwritten).
+__device__ int32_t long_runsum_compact(ContractSmem &sm, unsigned long long *keys, int32_t len) {
+    const int tid = threadIdx.x;
+    int32_t wr = 0;
+    unsigned long long pend = 0;
+    bool has_pend = false;  // uniform
+    for (int32_t w0 = 0; w0 < len; w0 += kBuf) {
+        const int32_t wl = min(kBuf, len - w0);
+        for (int32_t t = tid; t < wl; t += kCNT) sm.buf[t] = keys[w0 + t];
+        __syncthreads();
+        const int32_t cntw = coop_runsum(
+            sm.buf, wl, tid, kCNT, sm.lead, sm.has,
+            [&](int32_t v, int32_t &tot) { return block_excl_scan<kCNT>(v, sm.scan, tot); },
+            []() { __syncthreads(); });
+        int32_t hw = 0;  // compact the window's heads to sm.buf[0, cntw) (in place, as in C1h)
+        for (int32_t b0 = 0; b0 < wl; b0 += kCNT) {
+            const int32_t j = b0 + tid;
+            const unsigned long long kv = j < wl ? sm.buf[j] : 0ull;
+            const bool h = j < wl && is_head(sm.buf, j);
+            int32_t tot;
+            const int32_t ex = block_excl_scan<kCNT>(h ? 1 : 0, sm.scan, tot);
+            if (h) sm.buf[hw + ex] = kv;
+            hw += tot;
+            __syncthreads();
+        }
+        // the pending run of the previous window: continued by this window's first run, or done
+        const bool cont = has_pend && (uint32_t)(sm.buf[0] >> 32) == (uint32_t)(pend >> 32);
+        __syncthreads();
+        if (tid == 0) {
+            if (cont) sm.buf[0] = (pend & 0xFFFFFFFF00000000ull) | (uint32_t)((uint32_t)pend + (uint32_t)sm.buf[0]);
+            else if (has_pend) keys[wr] = pend;
+        }
+        if (has_pend && !cont) ++wr;
+        __syncthreads();
+        for (int32_t t = tid; t < cntw - 1; t += kCNT) keys[wr + t] = sm.buf[t];
+        wr += cntw - 1;
+        pend = sm.buf[cntw - 1];
+        has_pend = true;
+        __syncthreads();
+    }
+    if (has_pend) {
+        if (tid == 0) keys[wr] = pend;
+        ++wr;
+    }
+    __syncthreads();
+    return wr;
+}
+
 // ---------------------------------------------------------------------------------------
 // C1h: rows with ub > kWB, one CTA each; result compacted at gkeys[off[c]], count cnt[c]
 // ---------------------------------------------------------------------------------------
@@ -755,22 +806,26 @@ __device__ __noinline__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, 
         const int len = ub - nself;
         if (ub <= kCtaRow) coop_sort(keys, ub, threadIdx.x, kCNT, []() { __syncthreads(); });
         else cta_sort_long(sm, keys, a.tout + o0, ub);  // tout is idle until C2a
-        const int32_t cnt = coop_runsum(
-            keys, len, threadIdx.x, kCNT, sm.lead, sm.has,
-            [&](int32_t v, int32_t &tot) { return block_excl_scan<kCNT>(v, sm.scan, tot); },
-            []() { __syncthreads(); });
-        // compact the run heads into dst (in place when keys == dst: a chunk's writes land
-        // below its reads, and every read of a chunk precedes its writes)
-        int32_t wr = 0;
-        for (int32_t b0 = 0; b0 < len; b0 += kCNT) {
-            const int32_t j = b0 + threadIdx.x;
-            const unsigned long long kv = j < len ? keys[j] : 0ull;
-            const bool h = j < len && is_head(keys, j);
-            int32_t tot;
-            const int32_t ex = block_excl_scan<kCNT>(h ? 1 : 0, sm.scan, tot);
-            if (h) dst[wr + ex] = kv;
-            wr += tot;
-            __syncthreads();
+        int32_t cnt;
+        if (ub > kCtaRow) {
+            cnt = long_runsum_compact(sm, dst, len);
+        } else {
+            cnt = coop_runsum(
+                keys, len, threadIdx.x, kCNT, sm.lead, sm.has,
+                [&](int32_t v, int32_t &tot) { return block_excl_scan<kCNT>(v, sm.scan, tot); },
+                []() { __syncthreads(); });
+            // compact the run heads into dst
+            int32_t wr = 0;
+            for (int32_t b0 = 0; b0 < len; b0 += kCNT) {
+                const int32_t j = b0 + threadIdx.x;
+                const unsigned long long kv = j < len ? keys[j] : 0ull;
+                const bool h = j < len && is_head(keys, j);
+                int32_t tot;
+                const int32_t ex = block_excl_scan<kCNT>(h ? 1 : 0, sm.scan, tot);
+                if (h) dst[wr + ex] = kv;
+                wr += tot;
+                __syncthreads();
+            }
         }
         if (threadIdx.x == 0) a.cnt[c] = cnt;
         __syncthreads();
