@@ -637,6 +637,7 @@ __device__ __forceinline__ void gather_row(const ContractArgs &a, int32_t c, int
 // shared memory; the window split points of a batch are searched by all threads at once).
 // A bitonic network over global memory (the earlier design) paid ~log^2 dependent passes.
 // ---------------------------------------------------------------------------------------
+constexpr int kBigTile = 4096;  // C2b: tiles with more merged keys are copied by the whole CTA
 constexpr int kMW = kBuf / 2;  // outputs per merge window (A and B pieces staged side by side)
 
 // number of A elements among the first d outputs of merge(A, B) (A first on ties)
@@ -771,7 +772,9 @@ __device__ int32_t long_runsum_compact(ContractSmem &sm, unsigned long long *key
 // C1h: rows with ub > kWB, one CTA each; result compacted at gkeys[off[c]], count cnt[c]
 // ---------------------------------------------------------------------------------------
 __device__ __noinline__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
-    for (int i = blockIdx.x; i < nh; i += g_cact) {
+    // rows are claimed dynamically (first one static): a CTA busy with a 400 K-key hub row
+    // takes no further rows, instead of a fixed 1/nact share of them
+    for (int i = blockIdx.x; i < nh;) {
         const int32_t c = a.huge[i];
         const int32_t o0 = __ldcg(a.off + c);
         const int32_t ub = __ldcg(a.off + c + 1) - o0;
@@ -827,7 +830,12 @@ __device__ __noinline__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, 
                 __syncthreads();
             }
         }
-        if (threadIdx.x == 0) a.cnt[c] = cnt;
+        if (threadIdx.x == 0) {
+            a.cnt[c] = cnt;
+            sm.last = g_cact + (int)atomicAdd(&a.ctl->hub_ctr, 1u);
+        }
+        __syncthreads();
+        i = sm.last;
         __syncthreads();
     }
 }
@@ -1061,7 +1069,19 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
                 const int32_t k = __shfl_sync(0xffffffffu, cntc, src);
                 const int32_t pos = run + __shfl_sync(0xffffffffu, ex, src);
                 const unsigned long long *src_keys = a.gkeys + __ldcg(a.off + cw);
-                for (int32_t j = lane; j < k; j += 32) out[pos + j] = __ldcg(src_keys + j);
+                for (int32_t j0 = 0; j0 < k; j0 += 32 * 8) {  // 8 keys per lane in flight
+                    unsigned long long kk[8];
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) {
+                        const int32_t j = j0 + q * 32 + lane;
+                        kk[q] = j < k ? __ldcg(src_keys + j) : 0ull;
+                    }
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) {
+                        const int32_t j = j0 + q * 32 + lane;
+                        if (j < k) out[pos + j] = kk[q];
+                    }
+                }
             }
             __syncwarp();
             run += part;
@@ -1101,6 +1121,8 @@ __device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, i
     for (int s_lo = t_lo; s_lo < t_hi; s_lo += kCap) {
     const int s_hi = min(t_hi, s_lo + kCap);
     pre += block_scan_list(sm, a.ttot + s_lo, 1, 0, s_hi - s_lo, pre, tp);
+    if (threadIdx.x == 0) sm.len = 0;  // tiles too big for one warp (R-MAT hub rows): CTA copies
+    __syncthreads();
     for (int t = s_lo + wib; t < s_hi; t += kCW) {
         const int32_t p = tp[t - s_lo];
         int32_t r0 = 0, r1 = 0;
@@ -1114,7 +1136,17 @@ __device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, i
         }
         const int32_t total = __ldcg(a.ttot + t);
         for (int32_t c = r0 + lane; c < r1; c += 32) a.cadjp[c] = p + __ldcg(a.lofs + c);
-        if (r0 < r1) {
+        bool big = false;
+        if (r0 < r1 && total > kBigTile) {
+            int slot = 0;
+            if (lane == 0) slot = atomicAdd(&sm.len, 1);
+            slot = __shfl_sync(0xffffffffu, slot, 0);
+            if (slot < kCNT) {
+                big = true;
+                if (lane == 0) sm.lead[slot] = t;
+            }
+        }
+        if (r0 < r1 && !big) {
             const unsigned long long *src = a.tout + __ldcg(a.off + r0);
             constexpr int kB = 8;
             for (int32_t j0 = 0; j0 < total; j0 += 32 * kB) {
@@ -1137,6 +1169,32 @@ __device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, i
         if (t == ntiles2 - 1 && lane == 0) {
             a.cadjp[nc] = p + total;
             a.ctl->cnnz = p + total;
+        }
+    }
+    __syncthreads();
+    const int nbig = min(sm.len, kCNT);
+    for (int b = 0; b < nbig; ++b) {  // whole-CTA copies, 8 keys per thread in flight
+        const int t = sm.lead[b];
+        const int32_t p = tp[t - s_lo];
+        const int32_t r0 = a.dist ? __ldcg(a.tile_start + t) : t * rt;
+        const int32_t total = __ldcg(a.ttot + t);
+        const unsigned long long *src = a.tout + __ldcg(a.off + r0);
+        constexpr int kB = 8;
+        for (int32_t j0 = 0; j0 < total; j0 += kCNT * kB) {
+            unsigned long long k[kB];
+#pragma unroll
+            for (int q = 0; q < kB; ++q) {
+                const int32_t j = j0 + q * kCNT + threadIdx.x;
+                k[q] = j < total ? __ldcs(src + j) : 0ull;
+            }
+#pragma unroll
+            for (int q = 0; q < kB; ++q) {
+                const int32_t j = j0 + q * kCNT + threadIdx.x;
+                if (j < total) {
+                    a.cadjncy[p + j] = (int32_t)(k[q] >> 32);
+                    a.cadjwgt[p + j] = (int32_t)(uint32_t)k[q];
+                }
+            }
         }
     }
     __syncthreads();

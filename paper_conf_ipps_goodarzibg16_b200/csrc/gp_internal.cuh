@@ -58,7 +58,7 @@ struct ContractCtl {
     int32_t n_coarse, cnnz, n_huge;
     unsigned blocks_done;
     unsigned tile_ctr;  // dynamic C2a warp-tile claims
-    unsigned pad0;
+    unsigned hub_ctr;   // dynamic C1h row claims
     int32_t chunk1[2 * kMaxContractCtas];  // C1 chunk sums {#leaders, sum ub} per owner CTA
     int32_t chunk2[kMaxContractCtas];      // C2 chunk sums of merged entries per owner CTA
     unsigned long long dbg[8];             // debug: slowest C2a warp tile (ns<<32 | tile), paths
