@@ -615,13 +615,14 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
                                             int32_t *Pkw, RoundSlot *next, const int32_t (&u)[kVL],
                                             bool (&need)[kVL], bool (&live)[kVL], unsigned long long &scanned,
                                             unsigned long long &rows, const int32_t (&rs)[kVL],
-                                            const int32_t (&re)[kVL]) {
+                                            const int32_t (&re)[kVL], int i0 = 0, int i1 = kVL) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     FlatQ &fq = *(reinterpret_cast<FlatQ *>(&sm.adj[1][0]) + wib);
     int32_t rpos[kVL];
     int32_t qn = 0, T = 0;
 #pragma unroll
     for (int i = 0; i < kVL; ++i) {
+        if (i < i0 || i >= i1) continue;  // (warp-uniform)
         int32_t d = need[i] ? re[i] - rs[i] : 0;
         if (need[i]) ++rows;
         if (need[i] && d > kHubDeg) {
@@ -656,7 +657,7 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
     if (one) {  // every queued row marks its items with its entry
 #pragma unroll
         for (int i = 0; i < kVL; ++i)
-            if (need[i]) {
+            if (i >= i0 && i < i1 && need[i]) {
                 const int32_t o = fq.off[rpos[i]];
                 for (int32_t q = 0; q < re[i] - rs[i]; ++q) fq.own[o + q] = (uint8_t)rpos[i];
             }
@@ -731,7 +732,7 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
     }
 #pragma unroll
     for (int i = 0; i < kVL; ++i) {
-        if (need[i]) {
+        if (i >= i0 && i < i1 && need[i]) {
             const int32_t r = rpos[i];
             const unsigned long long k1 = one ? (((unsigned long long)fq.w1[r] << 32) | fq.n1[r]) : fq.k1[r];
             const unsigned long long k2 = one ? (((unsigned long long)fq.w2[r] << 32) | fq.n2[r]) : fq.k2[r];
@@ -839,7 +840,20 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
         bool live[kVL];
 #pragma unroll
         for (int i = 0; i < kVL; ++i) live[i] = u[i] >= 0 && p[i] != kNone && !need[i];
-        flat_rescan<kVL>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re);
+        {
+            // > 32*kFB items would take the two-pass CAS path: split the group's rescans in two
+            // single-batch halves instead (two dependent chains, no CAS)
+            int32_t dsum = 0;
+#pragma unroll
+            for (int i = 0; i < kVL; ++i)
+                if (need[i] && re[i] - rs[i] <= kHubDeg) dsum += re[i] - rs[i];
+            if (kVL >= 2 && warp_sum(dsum) > 32 * kFB) {
+                flat_rescan<kVL>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re, 0, kVL / 2);
+                flat_rescan<kVL>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re, kVL / 2, kVL);
+            } else {
+                flat_rescan<kVL>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re);
+            }
+        }
         if (kStatic) {
 #pragma unroll
             for (int i = 0; i < kVL; ++i) qn += live[i] ? 1 : 0;  // live count only
