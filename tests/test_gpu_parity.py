@@ -82,6 +82,9 @@ SMALL = {
     "C3_256": lambda: G.delaunay_like(256),
     "C3_300": lambda: G.delaunay_like(300),
     "C4_s14": lambda: G.rmat(14),
+    # weights [1,4] as C4: 785 rows > 1024 arcs (multi-CTA hub phase), 18 > 4096, max 15.8 K
+    # (C1h long rows: smem-sorted runs + merge-path merges + windowed run sums)
+    "C4_s17_w4": lambda: G.rmat(17, wmax=4),
     "C4_s12_unit": lambda: G.rmat(12, unit=True),
     "C5_256": lambda: G.road_like(256),
     "grid_unit_128": lambda: G.grid2d(128, 128),
