@@ -48,6 +48,9 @@ struct MatchCtl {
     int32_t lens[16], trows[16], wrows[16];
     // GP_PROF=1: round-k grid barrier: ~(first CTA arrival), last arrival, last release (ns)
     unsigned long long barr[16][3];
+    // parking: per round (ring k & 3) the wake tasks (matched vertices with parked neighbours)
+    // and the woken vertices to resolve within the round
+    int32_t nwake[4], nres[4];
 };
 
 constexpr int kMaxContractCtas = 1024;  // grid cap of the contraction kernel

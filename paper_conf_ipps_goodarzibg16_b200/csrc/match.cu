@@ -54,6 +54,11 @@ struct MatchArgs {
     int32_t *H;  // hub list of the pending hub phase
     int32_t *S;  // second-heaviest neighbour of the last full scan (NONE = none cached)
     unsigned long long *hk;  // multi-CTA hub phase: best key per listed hub (the contraction's idle gkeys)
+    // parking (single-GPU whole-level launches; null: off).  parked[u] = 1 while u, whose
+    // target is still free, is off the live list; pcnt[v] counts vertices that parked on v;
+    // W: wake tasks (matched vertices with parked neighbours), R: woken vertices.  All live in
+    // the contraction's scratch, idle while a level matches (cnt, lofs, huge, seg).
+    int32_t *parked, *pcnt, *W, *R;
     MatchCtl *ctl;
     int32_t max_rounds;
     int32_t leftover;
@@ -288,6 +293,10 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
             if (valid && gl == 0) {
                 const int32_t x = a.vbase + (int32_t)v;  // row v is vertex vbase + v
                 a.M[x] = kFree;
+                if (a.parked) {
+                    a.parked[x] = 0;
+                    a.pcnt[x] = 0;
+                }
                 if (hub) {
                     const int32_t h = atomicAdd(&a.ctl->slot[1].nhub, 1);
                     a.H[h] = x;
@@ -471,18 +480,96 @@ __device__ __forceinline__ void cta_flush(MatchSmem &sm, const int32_t *q, int32
     for (int i = lane; i < qn; i += 32) list[base + i] = q[i];
 }
 
+// Parking.  Under the rule a free vertex u keeps proposing its target p while
+// p is free, so a "keep p" vertex leaves the live list (parked) until p matches; a handshake
+// with p is then detected from p's side (a vertex whose proposal changed is always live in the
+// next round).  When v matches in round k it becomes a wake task; after the round barrier the
+// wake phase finds the vertices parked on v (P_k[x] == v and parked) and the resolve pass
+// gives them their round-(k+1) proposals exactly as the live-list protocol would have (their
+// target matched in round k: cached second choice or rescan), all within round k -- so the
+// proposals, handshakes and round counts are the rule's.  Each x is parked on one vertex and
+// each matched vertex is listed once (by itself, or by its live partner if it was parked).
+__device__ __forceinline__ void park_match(const MatchArgs &a, int32_t *Pn, RoundSlot *, int k, int32_t u,
+                                           int32_t p) {
+    int32_t *nw = &a.ctl->nwake[k & 3];
+    if (ldcg(a.parked + p)) {  // p is off the list: u also writes p's side (P_k[p] == u already)
+        a.M[p] = u;
+        Pn[p] = u;
+        a.parked[p] = 0;
+        if (ldcg(a.pcnt + p)) a.W[atomicAdd(nw, 1)] = p;
+    }
+    if (ldcg(a.pcnt + u)) a.W[atomicAdd(nw, 1)] = u;
+}
+__device__ __forceinline__ void park_keep(const MatchArgs &a, int32_t u, int32_t p) {
+    a.parked[u] = 1;
+    atomicAdd(&a.pcnt[p], 1);
+}
+
+// wake phase: the rows of the wake tasks in chunks of kHC arcs over all CTAs (as the hub phase)
+constexpr int kWC = kNT * 8;
+__device__ __noinline__ void wake_phase(const MatchArgs &a, MatchSmem &sm, int32_t nw, const int32_t *Pk,
+                                        int32_t *nres, int nact) {
+    const int t = threadIdx.x;
+    int32_t *hs = reinterpret_cast<int32_t *>(&sm.adj[0][0]);
+    int32_t *he = hs + kNT, *hb = he + kNT, *hv = hb + kNT;
+    long long carry = 0;
+    for (int32_t seg = 0; seg < nw; seg += kNT) {
+        const int32_t i = seg + t;
+        int32_t rs = 0, re = 0, ch = 0, v = -1;
+        if (i < nw) {
+            v = a.W[i];
+            rs = __ldg(a.adjp + (v - a.vbase));
+            re = __ldg(a.adjp + (v - a.vbase) + 1);
+            ch = (re - rs + kWC - 1) / kWC;
+        }
+        int32_t tot;
+        const int32_t ex = block_excl_scan<kNT>(ch, sm.scratch, tot);
+        hs[t] = rs;
+        he[t] = re;
+        hb[t] = ex;
+        hv[t] = v;
+        __syncthreads();
+        const int32_t nseg = min(kNT, nw - seg);
+        const long long g0 = carry + (((long long)blockIdx.x - carry) % nact + nact) % nact;
+        for (long long g = g0; g < carry + tot; g += nact) {
+            const int32_t loc = (int32_t)(g - carry);
+            int32_t r = 0;
+            for (int step = kNT / 2; step > 0; step >>= 1)
+                if (r + step < nseg && hb[r + step] <= loc) r += step;
+            const int32_t c0 = hs[r] + (loc - hb[r]) * kWC, c1 = min(he[r], c0 + kWC), vv = hv[r];
+            int32_t x[8], px[8];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const int32_t j = c0 + q * kNT + t;
+                x[q] = j < c1 ? __ldg(a.adjncy + j) : -1;
+            }
+#pragma unroll
+            for (int q = 0; q < 8; ++q) px[q] = x[q] >= 0 ? ldcg(Pk + x[q]) : -1;
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+                if (px[q] == vv && ldcg(a.parked + x[q])) {  // parked on the matched vv: resolve it
+                    a.parked[x[q]] = 0;
+                    a.R[atomicAdd(nres, 1)] = x[q];
+                }
+        }
+        carry += tot;
+        __syncthreads();
+    }
+}
+
 // Short live lists (small levels, late rounds): G lanes per live vertex, so a warp covers
 // 32/G vertices and a rescan reads G*4 arcs per dependent step instead of 8 per thread.
 // The round's critical path is then ~8 dependent loads whatever the row length (<= kHubDeg).
 // Same decisions as phase_k_impl (commit / keep p / cached second choice / rescan).
 template <int G>
-__device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t len, unsigned long long &scanned,
-                              unsigned long long &rows, unsigned long long &visits, int32_t &made) {
+__device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t len, bool park, const int32_t *Lover,
+                              unsigned long long &scanned, unsigned long long &rows, unsigned long long &visits,
+                              int32_t &made) {
     constexpr int VPW = 32 / G;  // live vertices per warp step
     const int32_t *Pk = a.P[k & 1];
     int32_t *Pn = a.P[(k + 1) & 1];
     int32_t *Pkw = a.P[k & 1];
-    const int32_t *Lk = a.L[k & 1];
+    const int32_t *Lk = Lover ? Lover : a.L[k & 1];
     int32_t *Ln = a.L[(k + 1) & 1];
     RoundSlot *next = &a.ctl->slot[(k + 1) & 3];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5, gl = lane % G;
@@ -502,7 +589,7 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
     };
     for (long long g = claim_next(); g < (a.interleave ? ngroups : g_hi); g = claim_next()) {
         const long long idx = g * VPW + lane / G;
-        int32_t u = idx < len ? ((k == 1) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
+        int32_t u = idx < len ? ((k == 1 && !Lover) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
         const int32_t p = u >= 0 ? ldcg(Pk + u) : kNone;
         const int32_t s2r = u >= 0 ? ldcg(a.S + u) : kNone;  // not predicated on p: same load level
         const int32_t rs0 = u >= 0 ? __ldg(a.adjp + (u - a.vbase)) : 0;  // speculative row bounds
@@ -519,11 +606,15 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
                 if (gl == 0) {
                     a.M[u] = p;  // handshake
                     Pn[u] = p;
+                    if (park) park_match(a, Pn, next, k, u, p);
                     ++made;
                 }
             } else if (rr != p) {
-                if (gl == 0) Pn[u] = p;  // p still free: still the heaviest free neighbour
-                live = true;
+                if (gl == 0) {
+                    Pn[u] = p;  // p still free: still the heaviest free neighbour
+                    if (park) park_keep(a, u, p);
+                }
+                live = !park;
             } else if (s2 != kNone && pps != s2) {
                 if (gl == 0) {
                     Pn[u] = s2;  // cached second choice still free
@@ -754,12 +845,13 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
 // load, no list append and no atomic with a return value on the round's critical path; the
 // next round's live count is a fire-and-forget reduction.
 template <int kVL, bool kStatic = false>
-__device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t len, unsigned long long &scanned,
-                             unsigned long long &rows, unsigned long long &visits, int32_t &made) {
+__device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t len, bool park, const int32_t *Lover,
+                             unsigned long long &scanned, unsigned long long &rows, unsigned long long &visits,
+                             int32_t &made) {
     const int32_t *Pk = a.P[k & 1];
     int32_t *Pn = a.P[(k + 1) & 1];
     int32_t *Pkw = a.P[k & 1];
-    const int32_t *Lk = a.L[k & 1];
+    const int32_t *Lk = Lover ? Lover : a.L[k & 1];
     int32_t *Ln = a.L[(k + 1) & 1];
     RoundSlot *next = &a.ctl->slot[(k + 1) & 3];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -788,7 +880,7 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
             const long long idx = base + i * 32 + lane;
-            u[i] = idx < len ? ((kStatic || k == 1) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
+            u[i] = idx < len ? ((kStatic || (k == 1 && !Lover)) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
         }
         int32_t rs[kVL], re[kVL];  // row bounds, loaded speculatively with P_k[u]: a rescan
                                    // then starts one dependent level earlier
@@ -815,19 +907,25 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
             rr[i] = (p[i] != kNone && qq[i] != u[i] && qq[i] >= 0) ? ldcg(Pk + qq[i]) : -1;
             pps[i] = ps[i] >= 0 ? ldcg(Pk + ps[i]) : -1;
         }
-        bool need[kVL];
+        bool need[kVL], parked_now[kVL];
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
             need[i] = false;
+            parked_now[i] = false;
             if (p[i] == kNone) continue;
             ++visits;
             if (qq[i] == u[i]) {
                 a.M[u[i]] = p[i];  // handshake: u and p propose each other
                 Pn[u[i]] = p[i];
+                if (park) park_match(a, Pn, next, k, u[i], p[i]);
                 ++made;
                 u[i] = -1;  // done
             } else if (rr[i] != p[i]) {
                 Pn[u[i]] = p[i];  // p is still free: still the heaviest free neighbour
+                if (park) {
+                    park_keep(a, u[i], p[i]);
+                    parked_now[i] = true;
+                }
             } else if (s2[i] != kNone && pps[i] != s2[i]) {
                 // the cached second-heaviest neighbour of u's last scan is still free: it is
                 // now u's heaviest free neighbour (the free set only shrinks)
@@ -839,7 +937,7 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
         }
         bool live[kVL];
 #pragma unroll
-        for (int i = 0; i < kVL; ++i) live[i] = u[i] >= 0 && p[i] != kNone && !need[i];
+        for (int i = 0; i < kVL; ++i) live[i] = u[i] >= 0 && p[i] != kNone && !need[i] && !parked_now[i];
         {
             // > 32*kFB items would take the two-pass CAS path: split the group's rescans in two
             // single-batch halves instead (two dependent chains, no CAS)
@@ -870,9 +968,9 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
     }
 }
 
-__device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, bool stat,
-                        unsigned long long &scanned, unsigned long long &rows, unsigned long long &visits,
-                        int32_t &made) {
+__device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, bool stat, bool park,
+                        const int32_t *Lover, unsigned long long &scanned, unsigned long long &rows,
+                        unsigned long long &visits, int32_t &made) {
     (void)n;
     unsigned long long t0 = 0, rows0 = rows;
     if (a.prof) {
@@ -882,13 +980,13 @@ __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int
     }
     const long long threads = (long long)g_nact * kNT;
     if (stat) {
-        if ((long long)len > threads) phase_k_impl<2, true>(a, sm, k, len, scanned, rows, visits, made);
-        else phase_k_impl<1, true>(a, sm, k, len, scanned, rows, visits, made);
-    } else if ((long long)len >= 4LL * threads) phase_k_impl<4>(a, sm, k, len, scanned, rows, visits, made);
-    else if (a.lanes_mode == 0 || (long long)len * 2 > threads) phase_k_impl<1>(a, sm, k, len, scanned, rows, visits, made);
-    else if ((long long)len * 8 <= threads) phase_k_lanes<8>(a, sm, k, len, scanned, rows, visits, made);
-    else if ((long long)len * 4 <= threads) phase_k_lanes<4>(a, sm, k, len, scanned, rows, visits, made);
-    else phase_k_lanes<2>(a, sm, k, len, scanned, rows, visits, made);
+        if ((long long)len > threads) phase_k_impl<2, true>(a, sm, k, len, false, nullptr, scanned, rows, visits, made);
+        else phase_k_impl<1, true>(a, sm, k, len, false, nullptr, scanned, rows, visits, made);
+    } else if ((long long)len >= 4LL * threads) phase_k_impl<4>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
+    else if (a.lanes_mode == 0 || (long long)len * 2 > threads) phase_k_impl<1>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
+    else if ((long long)len * 8 <= threads) phase_k_lanes<8>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
+    else if ((long long)len * 4 <= threads) phase_k_lanes<4>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
+    else phase_k_lanes<2>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
     if (a.prof && k < 16) {  // one shared atomic per warp, one global atomic per CTA
         const unsigned long long dt = globaltimer() - t0;
         const int32_t dr = warp_sum((int32_t)(rows - rows0));
@@ -949,6 +1047,7 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
     int32_t known_len = -1;       // next round's live-list length, read at the end of a round
     // small level: every round walks all vertices (kStatic), at most 2 per thread
     const bool stat = a.mode == kMatchWhole && a.static_mode && (long long)n <= 2LL * nact_all * kNT;
+    const bool park = a.mode == kMatchWhole && !stat && a.parked != nullptr;
     if (a.mode == kMatchWhole || a.mode == kMatchRound) {
         // kMatchWhole: the device-side round loop; kMatchRound: round a.k only (the sharded
         // driver exchanges the boundary proposals between launches and decides termination)
@@ -960,10 +1059,12 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
                 z->nhub = 0;
                 z->matches = 0;
                 z->claim = 0;
+                ctl->nwake[(k + 2) & 3] = 0;
+                ctl->nres[(k + 2) & 3] = 0;
             }
             const int32_t len = (k == 1 || stat) ? n : known_len >= 0 ? known_len : *(volatile int32_t *)&ctl->slot[k & 3].live;
             int32_t made = 0;
-            phase_k(a, sm, n, k, len, stat, scanned, rows, visits, made);
+            phase_k(a, sm, n, k, len, stat, park, nullptr, scanned, rows, visits, made);
             // any match this round: one flag store per CTA (only "> 0" is used)
             if (__syncthreads_or(made > 0) && threadIdx.x == 0) *(volatile int32_t *)&ctl->slot[k & 3].matches = 1;
             trace_mark(ctl->trace, tr++);
@@ -982,8 +1083,24 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
             trace_mark(ctl->trace, tr++);
             // the next slot {live, nhub} and this round's match flag: two independent loads
             // in flight together (one L2 round trip instead of three)
-            const int4 nxt = ld_volatile_v4(reinterpret_cast<const int4 *>(&ctl->slot[(k + 1) & 3]));
+            int4 nxt = ld_volatile_v4(reinterpret_cast<const int4 *>(&ctl->slot[(k + 1) & 3]));
             const int32_t made_any = *(volatile int32_t *)&ctl->slot[k & 3].matches;
+            if (park) {
+                const int32_t nw = *(volatile int32_t *)&ctl->nwake[k & 3];
+                if (nw > 0) {  // wake phase + resolve pass, still round k (see park_match)
+                    wake_phase(a, sm, nw, a.P[k & 1], &ctl->nres[k & 3], g_nact);
+                    if (tail) __syncthreads();
+                    else grid_barrier(ctl->bar, bar_epoch, nact_all);
+                    const int32_t nr = *(volatile int32_t *)&ctl->nres[k & 3];
+                    if (nr > 0) {
+                        int32_t made2 = 0;
+                        phase_k(a, sm, n, k, nr, false, true, a.R, scanned, rows, visits, made2);
+                        if (tail) __syncthreads();
+                        else grid_barrier(ctl->bar, bar_epoch, nact_all);
+                    }
+                    nxt = ld_volatile_v4(reinterpret_cast<const int4 *>(&ctl->slot[(k + 1) & 3]));
+                }
+            }
             int32_t live = nxt.x;
             if (nxt.y > 0) {
                 if (a.mode == kMatchWhole && !tail)
@@ -1096,6 +1213,18 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     a.H = lb.H;
     a.S = lb.S;
     a.hk = lb.gkeys;  // idle while a level matches (the contraction's hub-row scratch, >= nnz keys)
+    {
+        static int pk = -1;
+        if (pk < 0) {
+            const char *e = getenv("GP_MATCH_PARK");  // tuning knob (results never depend on it)
+            pk = (e && atoi(e) == 1) ? 1 : 0;
+        }
+        const bool on = pk && mode == kMatchWhole && lb.cnt && lb.lofs && lb.huge && lb.seg;
+        a.parked = on ? lb.cnt : nullptr;  // contraction scratch, idle while matching
+        a.pcnt = on ? lb.lofs : nullptr;
+        a.W = on ? lb.huge : nullptr;
+        a.R = on ? reinterpret_cast<int32_t *>(lb.seg) : nullptr;
+    }
     a.ctl = ctl;
     a.max_rounds = max_rounds;
     a.leftover = leftover ? 1 : 0;
