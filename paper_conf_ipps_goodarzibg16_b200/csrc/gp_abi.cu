@@ -685,6 +685,10 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
                         fprintf(stderr, " [%d %.1f %d/%d]", hd[l].match.lens[k], hd[l].match.wmax[k] * 1e-3,
                                 hd[l].match.trows[k], hd[l].match.wrows[k]);
                     fprintf(stderr, "\n");
+                    fprintf(stderr, "[gp]   per round (matched / kept target / second choice, impl path):");
+                    for (int k = 1; k < 16 && hd[l].match.lens[k]; ++k)
+                        fprintf(stderr, " [%d %d %d]", hd[l].match.nmatch[k], hd[l].match.nkeep[k], hd[l].match.nsec[k]);
+                    fprintf(stderr, "\n");
                     fprintf(stderr, "[gp]   round barriers (arrival spread | last arrival -> last release, us):");
                     for (int k = 1; k < 16 && hd[l].match.barr[k][1]; ++k)
                         fprintf(stderr, " [%.1f %.1f]", (hd[l].match.barr[k][1] - ~hd[l].match.barr[k][0]) * 1e-3,

@@ -51,6 +51,9 @@ struct MatchCtl {
     // parking: per round (ring k & 3) the wake tasks (matched vertices with parked neighbours)
     // and the woken vertices to resolve within the round
     int32_t nwake[4], nres[4];
+    // GP_PROF=1: per round k < 16, how the live vertices ended: kept their target / took the
+    // cached second choice / matched (rescans: trows)
+    int32_t nkeep[16], nsec[16], nmatch[16];
 };
 
 constexpr int kMaxContractCtas = 1024;  // grid cap of the contraction kernel

@@ -1123,7 +1123,9 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
             if (a.max_rounds > 0 && rounds >= a.max_rounds) break;
             // short live list: the grid barriers (not the work) would dominate the remaining
             // rounds, so CTA 0 finishes them alone; the others wait at the barrier below
-            if (!stat && !tail && nact_all > 1 && live <= a.tail_live) {
+            // (not with parking: the list then holds only the changed vertices while many may
+            // still be parked, and their wake/resolve passes need the whole grid)
+            if (!stat && !park && !tail && nact_all > 1 && live <= a.tail_live) {
                 tail = true;
                 if (blockIdx.x != 0) break;
                 __syncthreads();
