@@ -149,18 +149,18 @@ class ClockSampler:
 # ------------------------------------------------------------------------------------------
 # oracle timing (cpu_baseline and --impl reference)
 # ------------------------------------------------------------------------------------------
-def oracle_run(g, threshold):
+def oracle_run(g, threshold, tie_seed=0):
     import oracle
     t0 = time.perf_counter()
-    levels = oracle.coarsen_to(g, threshold)
+    levels = oracle.coarsen_to(g, threshold, tie_seed=tie_seed)
     dt = time.perf_counter() - t0
     return dt, sum(l["nnz"] // 2 for l in levels), len(levels)
 
 
-def cpu_baseline(g, threshold, budget_s=12.0):
+def cpu_baseline(g, threshold, budget_s=12.0, tie_seed=0):
     runs, tot_t, tot_e, nlev = 0, 0.0, 0, 0
     while runs == 0 or tot_t < budget_s:
-        dt, e, nlev = oracle_run(g, threshold)
+        dt, e, nlev = oracle_run(g, threshold, tie_seed)
         runs += 1
         tot_t += dt
         tot_e += e
@@ -212,7 +212,7 @@ def run_ours(args, rank, world, local_rank):
     stream = ctx.stream
 
     def step():
-        return graph.coarsen_to(threshold)
+        return graph.coarsen_to(threshold, tie_seed=args.tie_seed)
 
     # warm-up
     hier = None
@@ -318,7 +318,7 @@ def run_ours(args, rank, world, local_rank):
             gh = gp.Graph.create_dist(ctx, n, vb, host["adjp"], host["adjncy"], host["adjwgt"], host["vwgt"])
         else:
             gh = gp.Graph.create(ctx, host["adjp"], host["adjncy"], host["adjwgt"], host["vwgt"])
-        hh = gh.coarsen_to(threshold)
+        hh = gh.coarsen_to(threshold, tie_seed=args.tie_seed)
         nb = 0
         for i in range(len(hh)):
             _, c = hh.download_level(i, cmap=cm_bufs[i], want_match=False)
@@ -338,7 +338,7 @@ def run_ours(args, rank, world, local_rank):
         "metric": METRIC, "value": edges_per_step / (ms_step / 1e3), "unit": UNIT, "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
         "scaling": "strong" if sharded else "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-        "config": {"workload": f"{args.config}:{name}", "n": n, "edges": nnz // 2, "threshold": threshold,
+        "config": {"workload": f"{args.config}:{name}" + (f":rm_seed{args.tie_seed:#x}" if args.tie_seed else ""), "n": n, "edges": nnz // 2, "threshold": threshold,
                    "levels": len(levels), "edges_all_levels": edges_per_step,
                    "level0_edges_per_s": (nnz // 2) / (ms_step / 1e3),
                    "t_full_ms": ms_step, "rounds": [l["rounds"] for l in levels],
@@ -363,7 +363,7 @@ def run_ours(args, rank, world, local_rank):
     }
     if rank == 0 and not args.no_cpu_baseline:
         gh = {k: g[k].cpu() for k in ("adjp", "adjncy", "adjwgt", "vwgt")}
-        line["cpu_baseline"] = cpu_baseline(gh, threshold)
+        line["cpu_baseline"] = cpu_baseline(gh, threshold, tie_seed=args.tie_seed)
         line["cpu_baseline"].update(host_info())
     graph.close()
     ctx.close()
@@ -376,18 +376,18 @@ def run_reference(args, rank, world):
         return None
     g, _ = make_graph(args.config, "cpu")
     for _ in range(args.warmup):
-        oracle_run(g, threshold)
+        oracle_run(g, threshold, args.tie_seed)
     t = 0.0
     e = 0
     for _ in range(args.steps):
-        dt, e, nlev = oracle_run(g, threshold)
+        dt, e, nlev = oracle_run(g, threshold, args.tie_seed)
         t += dt
     ms = t / args.steps * 1e3
     value = e / (ms / 1e3)
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-            "config": {"workload": f"{args.config}:{name}", "n": g["n"], "edges": g["nnz"] // 2,
+            "config": {"workload": f"{args.config}:{name}" + (f":rm_seed{args.tie_seed:#x}" if args.tie_seed else ""), "n": g["n"], "edges": g["nnz"] // 2,
                        "threshold": threshold, "edges_all_levels": e},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
                              "sample": f"full coarsen-to-{threshold} per step, single-threaded C oracle"},
@@ -406,6 +406,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--loopback", type=int, default=0,
                     help="run the sharded protocol with this many simulated ranks on one GPU")
+    ap.add_argument("--tie-seed", type=lambda x: int(x, 0), default=0,
+                    help="0: lower id wins equal-weight ties (north_star); else the RM tie priority "
+                         "lowbias32(v ^ seed) (DESIGN R17, P18.s8)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3) if args.impl == "ours" else args.warmup
 

@@ -15,7 +15,7 @@
  *     weights >= 1, equal in both directions), vwgt[n] (vertex weights >= 1).  All ids,
  *     offsets and weights are int32 (R14): n < 2^31, nnz < 2^31, sum(vwgt) and
  *     sum(adjwgt) <= INT32_MAX (checked by gp_graph_create; then no coarse level can
- *     overflow).  No self-loops, no duplicate arcs; neighbour order is arbitrary (R15).
+ *     overflow).  No self-loops, no duplicate arcs; neighbour order is arbitrary (R17).
  *   * "d_" pointers are device pointers on the context's device; "h_" pointers are host.
  *   * Everything is enqueued on the context's CUDA stream.  Calls documented as
  *     "synchronous" block the calling thread until the stream has drained their work.
@@ -115,6 +115,17 @@ gp_status gp_graph_download(gp_graph g, gp_vid *h_adjp, gp_vid *h_adjncy, gp_wgt
  *               that created at least one match (R4). */
 gp_status gp_match_level(gp_graph g, gp_vid *d_match, int32_t max_rounds, int32_t *rounds_out);
 
+/* gp_match_level with a tie priority (R17 of DESIGN.md §2; P18.s8: "If all the edges have the
+ * same weight, a random matching (RM) ... where each vertex chooses one of its unmatched
+ * vertices randomly").  Among neighbours of equal edge weight the proposal goes to the lower
+ * h_s(v) = lowbias32(v ^ tie_seed) instead of the lower id (lowbias32: x ^= x>>16;
+ * x *= 0x7feb352d; x ^= x>>15; x *= 0x846ca68b; x ^= x>>16, all mod 2^32).  tie_seed = 0 is
+ * exactly gp_match_level.  The result is deterministic for a given seed; heavier edges still
+ * win, so only ties (all of them on unit-weight graphs) are decided "randomly".  The rule is
+ * the default rule on the vertices relabeled by h_s, so it is maximal and terminates alike. */
+gp_status gp_match_level_ex(gp_graph g, gp_vid *d_match, int32_t max_rounds, uint32_t tie_seed,
+                            int32_t *rounds_out);
+
 /* Contraction of one level (P18.s16-27 cmap; P12.s26-28, P20.s0-26 contraction):
  *   d_match     a valid matching of g (output of gp_match_level), device int32[n]
  *   d_cmap      caller-owned device int32[n]; receives CM: leaders (u <= M[u]) get
@@ -132,6 +143,8 @@ typedef struct {
     int32_t stall_ratio_pct; /* stop after a level with 100*n_c > pct*n; 0 => 95            */
     int32_t max_levels;      /* 0 => 64                                                     */
     int32_t max_rounds;      /* per level; 0 => fixpoint (maximal matchings)               */
+    uint32_t tie_seed;       /* 0 => lower id wins ties (north_star); else the RM tie
+                                priority of gp_match_level_ex at every level (R17)          */
 } gp_coarsen_opts;
 
 #define GP_STOP_NONE 0      /* more levels follow                                          */

@@ -44,6 +44,11 @@ def _load():
         lib.oracle_match_level.restype = ctypes.c_int
         lib.oracle_match_level.argtypes = [ctypes.c_int32, _i32p, _i32p, _i32p, ctypes.c_int32,
                                            _i32p, _i32p, _i32p]
+        lib.oracle_match_level_seeded.restype = ctypes.c_int
+        lib.oracle_match_level_seeded.argtypes = [ctypes.c_int32, _i32p, _i32p, _i32p, ctypes.c_int32,
+                                                  ctypes.c_uint32, _i32p, _i32p, _i32p]
+        lib.oracle_tie_hash.restype = ctypes.c_uint32
+        lib.oracle_tie_hash.argtypes = [ctypes.c_uint32, ctypes.c_uint32]
         lib.oracle_cmap.restype = ctypes.c_int32
         lib.oracle_cmap.argtypes = [ctypes.c_int32, _i32p, _i32p]
         lib.oracle_contract.restype = ctypes.c_int64
@@ -71,8 +76,15 @@ def as_numpy_graph(g: Dict) -> Dict[str, np.ndarray]:
     return out
 
 
-def match_level(g: Dict, max_rounds: int = 0):
-    """Heavy-edge handshake matching of one level (oracle.c: oracle_match_level).
+def tie_hash(v: int, seed: int) -> int:
+    """RM tie priority h_s(v) of oracle.c (reading R17, P18.s8)."""
+    return int(_load().oracle_tie_hash(v & 0xFFFFFFFF, seed & 0xFFFFFFFF))
+
+
+def match_level(g: Dict, max_rounds: int = 0, tie_seed: int = 0):
+    """Heavy-edge handshake matching of one level (oracle.c: oracle_match_level_seeded).
+    tie_seed = 0: equal weights go to the lower id (north_star); else to the lower
+    h_s(v) (RM reading R17 of P18.s8).
 
     Returns (match int32[n], rounds, maximal)."""
     lib = _load()
@@ -81,9 +93,9 @@ def match_level(g: Dict, max_rounds: int = 0):
     match = np.empty(max(n, 1), dtype=np.int32)
     rounds = ctypes.c_int32(0)
     maximal = ctypes.c_int32(0)
-    st = lib.oracle_match_level(n, _p(g["adjp"]), _p(g["adjncy"]), _p(g["adjwgt"]),
-                                int(max_rounds), _p(match), ctypes.byref(rounds),
-                                ctypes.byref(maximal))
+    st = lib.oracle_match_level_seeded(n, _p(g["adjp"]), _p(g["adjncy"]), _p(g["adjwgt"]),
+                                       int(max_rounds), int(tie_seed) & 0xFFFFFFFF, _p(match),
+                                       ctypes.byref(rounds), ctypes.byref(maximal))
     if st != 0:
         raise RuntimeError("oracle_match_level: a round with proposals made no match")
     return match[:n], int(rounds.value), bool(maximal.value)
@@ -125,7 +137,7 @@ STOP_MAX_LEVELS = 3  # max_levels reached
 
 
 def coarsen_to(g: Dict, threshold: int, stall_ratio_pct: int = 95, max_levels: int = 64,
-               max_rounds: int = 0) -> List[Dict]:
+               max_rounds: int = 0, tie_seed: int = 0) -> List[Dict]:
     """Level loop (P10.s16, P20.s27-31, P12.s30; readings R12, R13).
 
     while n > threshold and levels < max_levels:
@@ -139,7 +151,7 @@ def coarsen_to(g: Dict, threshold: int, stall_ratio_pct: int = 95, max_levels: i
     levels: List[Dict] = []
     cur = as_numpy_graph(g)
     while cur["n"] > threshold and len(levels) < max_levels:
-        m, rounds, maximal = match_level(cur, max_rounds)
+        m, rounds, maximal = match_level(cur, max_rounds, tie_seed)
         cm, n_c = cmap(m)
         coarse = contract(cur, m, cm, n_c)
         stall = 100 * n_c > stall_ratio_pct * cur["n"]

@@ -43,6 +43,36 @@ static int oracle_prefers(int32_t w1, int32_t v1, int32_t w2, int32_t v2)
 }
 
 /*
+ * RM tie priority (reading R17 of DESIGN.md §2 for P18.s8: "If all the edges have the same
+ * weight, a random matching (RM) ... where each vertex chooses one of its unmatched
+ * vertices randomly").  The random choice is made deterministic by a seeded counter-based
+ * priority: h_s(v) = lowbias32(v XOR s), all arithmetic mod 2^32:
+ *   x ^= x >> 16;  x *= 0x7feb352d;  x ^= x >> 15;  x *= 0x846ca68b;  x ^= x >> 16.
+ * Exported so that the tests can pin it against an independent Python transcription.
+ */
+uint32_t oracle_tie_hash(uint32_t v, uint32_t s)
+{
+    uint32_t x = v ^ s;
+    x ^= x >> 16;
+    x *= 0x7feb352du;
+    x ^= x >> 15;
+    x *= 0x846ca68bu;
+    x ^= x >> 16;
+    return x;
+}
+
+/*
+ * Preference under a tie seed s != 0: the heavier edge wins; on equal weight the lower
+ * h_s(v) wins.  s == 0 is oracle_prefers (north_star rule).
+ */
+static int oracle_prefers_seeded(int32_t w1, int32_t v1, int32_t w2, int32_t v2, uint32_t s)
+{
+    if (s == 0) return oracle_prefers(w1, v1, w2, v2);
+    if (w1 != w2) return w1 > w2;
+    return oracle_tie_hash((uint32_t)v1, s) < oracle_tie_hash((uint32_t)v2, s);
+}
+
+/*
  * One matching level (P16.s23-25, P18.s6-13 and north_star's pinned rule, R1-R4):
  *
  *   M[u] = FREE for all u; rounds = 0
@@ -64,9 +94,9 @@ static int oracle_prefers(int32_t w1, int32_t v1, int32_t w2, int32_t v2)
  * Returns 0 on success, -1 if a round with a proposing vertex created no match (the
  * termination lemma of DESIGN.md §2 says this cannot happen; the tests assert it).
  */
-int oracle_match_level(int32_t n, const int32_t *adjp, const int32_t *adjncy,
-                       const int32_t *adjwgt, int32_t max_rounds,
-                       int32_t *match, int32_t *rounds_out, int32_t *maximal_out)
+int oracle_match_level_seeded(int32_t n, const int32_t *adjp, const int32_t *adjncy,
+                              const int32_t *adjwgt, int32_t max_rounds, uint32_t tie_seed,
+                              int32_t *match, int32_t *rounds_out, int32_t *maximal_out)
 {
     int32_t *P = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
     int32_t *Mn = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
@@ -91,7 +121,7 @@ int oracle_match_level(int32_t n, const int32_t *adjp, const int32_t *adjncy,
                 int32_t v = adjncy[j];
                 int32_t w = adjwgt[j];
                 if (match[v] != ORACLE_FREE) continue;
-                if (best_v == ORACLE_NONE || oracle_prefers(w, v, best_w, best_v)) {
+                if (best_v == ORACLE_NONE || oracle_prefers_seeded(w, v, best_w, best_v, tie_seed)) {
                     best_v = v;
                     best_w = w;
                 }
@@ -122,6 +152,15 @@ int oracle_match_level(int32_t n, const int32_t *adjp, const int32_t *adjncy,
     free(P);
     free(Mn);
     return status;
+}
+
+/* The north_star rule: lower id wins ties (tie seed 0). */
+int oracle_match_level(int32_t n, const int32_t *adjp, const int32_t *adjncy,
+                       const int32_t *adjwgt, int32_t max_rounds,
+                       int32_t *match, int32_t *rounds_out, int32_t *maximal_out)
+{
+    return oracle_match_level_seeded(n, adjp, adjncy, adjwgt, max_rounds, 0u,
+                                     match, rounds_out, maximal_out);
 }
 
 /*

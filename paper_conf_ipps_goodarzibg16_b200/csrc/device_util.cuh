@@ -33,13 +33,32 @@ __device__ __forceinline__ unsigned lanemask_lt() {
     return m;
 }
 
-// Proposal key of neighbour v over edge weight w (P12.s23, R3): heavier first, then the
-// lower id.  key > 0 for every valid (w >= 1) arc; 0 means "no candidate".
-__device__ __forceinline__ unsigned long long pack_key(int32_t w, int32_t v) {
-    return ((unsigned long long)(uint32_t)w << 32) | (unsigned long long)(~(uint32_t)v);
+// Tie priority of neighbour v (R17): seed 0 is the north_star rule (the lower
+// id wins among equal weights); a nonzero seed is the deterministic reading of the paper's
+// random matching for equal weights (P18.s8): the lower h_s(v) = lowbias32(v ^ seed) wins.
+// lowbias32 is a bijection of uint32, so keys stay distinct per row and the termination
+// lemma (§2.1) holds unchanged (it is the default rule on the vertices relabeled by h_s).
+__device__ __forceinline__ uint32_t tie_hash(uint32_t v, uint32_t s) {
+    uint32_t x = v ^ s;
+    x ^= x >> 16; x *= 0x7feb352du; x ^= x >> 15; x *= 0x846ca68bu; x ^= x >> 16;
+    return x;
 }
-__device__ __forceinline__ int32_t key_vertex(unsigned long long k) {
-    return k ? (int32_t)(~(uint32_t)k) : kNone;
+__device__ __forceinline__ uint32_t tie_unhash(uint32_t x, uint32_t s) {
+    x ^= x >> 16; x *= 0x43021123u; x ^= x >> 15; x ^= x >> 30; x *= 0x1d69e2a5u; x ^= x >> 16;
+    return x ^ s;
+}
+
+// Proposal key of neighbour v over edge weight w (P12.s23, R3): heavier first, then the
+// tie priority (lower id, or lower h_s(v) under a tie seed).  key > 0 for every valid
+// (w >= 1) arc; 0 means "no candidate".
+__device__ __forceinline__ unsigned long long pack_key(uint32_t s, int32_t w, int32_t v) {
+    const uint32_t t = s ? tie_hash((uint32_t)v, s) : (uint32_t)v;
+    return ((unsigned long long)(uint32_t)w << 32) | (unsigned long long)(~t);
+}
+__device__ __forceinline__ int32_t key_vertex(uint32_t s, unsigned long long k) {
+    if (!k) return kNone;
+    const uint32_t t = ~(uint32_t)k;
+    return (int32_t)(s ? tie_unhash(t, s) : t);
 }
 
 __device__ __forceinline__ unsigned long long umax64(unsigned long long a, unsigned long long b) {

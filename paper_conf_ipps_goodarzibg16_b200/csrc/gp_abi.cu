@@ -421,12 +421,18 @@ static gp_status fresh_sizes(Ctx *ctx, const Graph *g, SizeRec *dst) {
 static double avg_degree(int32_t n, int32_t nnz) { return n > 0 ? (double)nnz / n : 0.0; }
 
 gp_status gp_match_level(gp_graph g, gp_vid *d_match, int32_t max_rounds, int32_t *rounds_out) {
+    return gp_match_level_ex(g, d_match, max_rounds, 0u, rounds_out);
+}
+
+gp_status gp_match_level_ex(gp_graph g, gp_vid *d_match, int32_t max_rounds, uint32_t tie_seed,
+                            int32_t *rounds_out) {
     if (!tagged<Graph>(g, kTagGraph) || (!d_match && g->n > 0) || max_rounds < 0) {
         set_error("gp_match_level: bad graph, match buffer or max_rounds");
         return GP_ERR_INVALID_ARG;
     }
     GP_TRY_BEGIN
     Ctx *ctx = g->ctx;
+    ctx->tie_seed = tie_seed;
     if (ctx->comm) {
         set_error("gp_match_level: per-level calls are single-GPU; sharded graphs use gp_coarsen_to");
         return GP_ERR_INVALID_ARG;
@@ -550,6 +556,7 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
     }
     GP_TRY_BEGIN
     Ctx *ctx = g->ctx;
+    ctx->tie_seed = opts->tie_seed;
     if (ctx->comm) return dist_coarsen_to(g, opts, out);  // sharded path (dist.cu)
     const int32_t pct = opts->stall_ratio_pct ? opts->stall_ratio_pct : 95;
     int32_t max_levels = opts->max_levels ? opts->max_levels : 64;

@@ -183,6 +183,9 @@ struct gp_ctx_s {
     unsigned long long *status = nullptr;  // look-back tile status words
     size_t status_words = 0;
     uint32_t epoch = 1;  // look-back epoch (no memset between scans)
+    // tie priority of the matching launches of the current call (R17): set by the ABI entry
+    // (gp_match_level_ex / gp_coarsen_to from its opts) before it enqueues any match launch
+    uint32_t tie_seed = 0;
 
     // sharded path: NCCL (one local rank) or loopback (all ranks simulated); null = 1 GPU
     gp::DistComm *comm = nullptr;

@@ -48,7 +48,8 @@ class GPError(RuntimeError):
 
 
 class CoarsenOpts(ctypes.Structure):
-    _fields_ = [("threshold", _i32), ("stall_ratio_pct", _i32), ("max_levels", _i32), ("max_rounds", _i32)]
+    _fields_ = [("threshold", _i32), ("stall_ratio_pct", _i32), ("max_levels", _i32), ("max_rounds", _i32),
+                ("tie_seed", ctypes.c_uint32)]
 
 
 class Level(ctypes.Structure):
@@ -79,6 +80,7 @@ _sig("gp_graph_view", ctypes.c_int, [_vp, _i32p, _i32p, ctypes.POINTER(_vp), cty
                                      ctypes.POINTER(_vp), ctypes.POINTER(_vp)])
 _sig("gp_graph_download", ctypes.c_int, [_vp, _vp, _vp, _vp, _vp])
 _sig("gp_match_level", ctypes.c_int, [_vp, _vp, _i32, _i32p])
+_sig("gp_match_level_ex", ctypes.c_int, [_vp, _vp, _i32, ctypes.c_uint32, _i32p])
 _sig("gp_contract_level", ctypes.c_int, [_vp, _vp, _vp, ctypes.POINTER(_vp)])
 _sig("gp_coarsen_to", ctypes.c_int, [_vp, ctypes.POINTER(CoarsenOpts), ctypes.POINTER(_vp)])
 _sig("gp_hier_num_levels", ctypes.c_int, [_vp, _i32p])
@@ -261,11 +263,13 @@ class Graph:
         out["n"], out["nnz"] = n, nnz
         return out
 
-    def match_level(self, match: torch.Tensor, max_rounds: int = 0, sync_rounds: bool = True) -> Optional[int]:
-        """gp_match_level into a caller-owned device int32[n] tensor; returns rounds."""
+    def match_level(self, match: torch.Tensor, max_rounds: int = 0, sync_rounds: bool = True,
+                    tie_seed: int = 0) -> Optional[int]:
+        """gp_match_level_ex into a caller-owned device int32[n] tensor; returns rounds.
+        tie_seed != 0: equal-weight ties go to the lower lowbias32(v ^ seed) (RM, P18.s8)."""
         r = _i32()
-        _check(_lib.gp_match_level(self.handle, _ptr(match), max_rounds, ctypes.byref(r) if sync_rounds else None),
-               "gp_match_level")
+        _check(_lib.gp_match_level_ex(self.handle, _ptr(match), max_rounds, tie_seed & 0xFFFFFFFF,
+                                      ctypes.byref(r) if sync_rounds else None), "gp_match_level_ex")
         return r.value if sync_rounds else None
 
     def contract_level(self, match: torch.Tensor, cmap: torch.Tensor) -> "Graph":
@@ -275,8 +279,8 @@ class Graph:
         return Graph(self.ctx, h)
 
     def coarsen_to(self, threshold: int, stall_ratio_pct: int = 95, max_levels: int = 64,
-                   max_rounds: int = 0) -> "Hierarchy":
-        opts = CoarsenOpts(threshold, stall_ratio_pct, max_levels, max_rounds)
+                   max_rounds: int = 0, tie_seed: int = 0) -> "Hierarchy":
+        opts = CoarsenOpts(threshold, stall_ratio_pct, max_levels, max_rounds, tie_seed & 0xFFFFFFFF)
         h = _vp()
         _check(_lib.gp_coarsen_to(self.handle, ctypes.byref(opts), ctypes.byref(h)), "gp_coarsen_to")
         return Hierarchy(self.ctx, h)
