@@ -67,8 +67,27 @@ def _exchange(send: Dict[int, np.ndarray], width: int) -> Dict[int, np.ndarray]:
     return {s: t.numpy() for s, t in recv.items()}
 
 
+TIE_SEED = 0  # RM tie priority (DESIGN R17); set by coarsen_to
+
+
+def _tie(v):
+    """Tie priority of v: its id (seed 0) or lowbias32(v ^ seed)."""
+    if TIE_SEED == 0:
+        return int(v)
+    x = (int(v) ^ TIE_SEED) & 0xFFFFFFFF
+    x ^= x >> 16
+    x = (x * 0x7FEB352D) & 0xFFFFFFFF
+    x ^= x >> 15
+    x = (x * 0x846CA68B) & 0xFFFFFFFF
+    return x ^ (x >> 16)
+
+
 def _key(w, v):
-    return (int(w) << 32) | (0xFFFFFFFF - int(v))
+    return ((int(w) << 32) | (0xFFFFFFFF - _tie(v)), int(v))
+
+
+def _key_vertex(k):
+    return NONE if k == 0 else k[1]
 
 
 class Shard:
@@ -127,7 +146,7 @@ def match_level(sh: Shard, max_rounds: int = 0):
     for u in loc:
         keys = [_key(sh.adjwgt[j], sh.adjncy[j]) for j in sh.row(u)]
         k = max(keys) if keys else 0
-        P[1][u] = NONE if k == 0 else 0xFFFFFFFF - (k & 0xFFFFFFFF)
+        P[1][u] = _key_vertex(k)
         if P[1][u] == NONE:
             P[0][u] = NONE
     live = [u for u in loc if P[1][u] != NONE]
@@ -155,7 +174,7 @@ def match_level(sh: Shard, max_rounds: int = 0):
                 continue
             keys = [_key(sh.adjwgt[j], sh.adjncy[j]) for j in sh.row(u) if free_after(int(sh.adjncy[j]))]
             kk = max(keys) if keys else 0
-            b = NONE if kk == 0 else 0xFFFFFFFF - (kk & 0xFFFFFFFF)
+            b = _key_vertex(kk)
             Pn[u] = b
             if b == NONE:
                 Pk[u] = NONE  # dead: NONE in both buffers (after everyone read P_k[u]? see note)
@@ -259,8 +278,11 @@ def contract_level(sh: Shard, M: np.ndarray):
     return CM, coarse
 
 
-def coarsen_to(sh: Shard, threshold: int, stall_ratio_pct: int = 95, max_levels: int = 64, max_rounds: int = 0):
+def coarsen_to(sh: Shard, threshold: int, stall_ratio_pct: int = 95, max_levels: int = 64, max_rounds: int = 0,
+               tie_seed: int = 0):
     """Levels of this rank: list of dicts with the rank's slices of M / CM and coarse piece."""
+    global TIE_SEED
+    TIE_SEED = tie_seed & 0xFFFFFFFF
     levels = []
     while sh.N > threshold and len(levels) < max_levels:
         M, rounds, maximal = match_level(sh, max_rounds)
