@@ -76,7 +76,7 @@ struct MatchArgs {
     int32_t prof;        // GP_PROF=1: per-round slowest-warp times and rescan counts (MatchCtl)
     int32_t mode;  // kMatchWhole, or one launch per phase for the sharded path
     int32_t k;     // round of a kMatchRound launch
-    uint32_t tie_seed;  // 0: lower id wins ties (north_star); else RM tie priority (R17, P18.s8)
+    TieHash tie;  // tie priority: seed 0 = lower id wins (north_star); else RM (R17, P18.s8)
 };
 
 
@@ -271,7 +271,7 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
             bool hub = false;
             if (fits) {
                 const int32_t *sa = sm.adj[st], *sw = sm.wgt[st];
-                for (int32_t j = s - A0 + gl; j < e - A0; j += G) top2_add(key, key2, pack_key(a.tie_seed, sw[j], sa[j]));
+                for (int32_t j = s - A0 + gl; j < e - A0; j += G) top2_add(key, key2, pack_key(a.tie, sw[j], sa[j]));
             } else if (valid) {
                 if (e - s > kHubDeg) {
                     hub = true;
@@ -286,7 +286,7 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
                         }
 #pragma unroll
                         for (int q = 0; q < 8; ++q)
-                            if (xv[q] >= 0) top2_add(key, key2, pack_key(a.tie_seed, wv[q], xv[q]));
+                            if (xv[q] >= 0) top2_add(key, key2, pack_key(a.tie, wv[q], xv[q]));
                     }
                 }
             }
@@ -304,9 +304,9 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
                     if (a.hk) a.hk[h] = 0ull;  // (sharded launches: per-CTA hub_phase, no hk)
                     a.S[x] = kNone;
                 } else {
-                    const int32_t p = key_vertex(a.tie_seed, key);
+                    const int32_t p = key_vertex(a.tie, key);
                     P1[x] = p;
-                    a.S[x] = key_vertex(a.tie_seed, key2);  // cached second-heaviest neighbour
+                    a.S[x] = key_vertex(a.tie, key2);  // cached second-heaviest neighbour
                     if (p == kNone) P0[x] = kNone;  // dead vertices: NONE in both buffers
                     scanned += (unsigned long long)(e - s);
                 }
@@ -338,7 +338,7 @@ __device__ __noinline__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_
         unsigned long long key = 0;
         for (int32_t j = s + threadIdx.x; j < e; j += kNT) {
             const int32_t x = __ldg(a.adjncy + j);
-            if (!check || free_after(x, Pk)) key = umax64(key, pack_key(a.tie_seed, __ldg(a.adjwgt + j), x));
+            if (!check || free_after(x, Pk)) key = umax64(key, pack_key(a.tie, __ldg(a.adjwgt + j), x));
         }
         key = group_max64<32>(key);
         if (lane == 0) sm.red[wib] = key;
@@ -346,7 +346,7 @@ __device__ __noinline__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_
         if (threadIdx.x == 0) {
             unsigned long long k = 0;
             for (int q = 0; q < kNT / 32; ++q) k = umax64(k, sm.red[q]);
-            const int32_t p = key_vertex(a.tie_seed, k);
+            const int32_t p = key_vertex(a.tie, k);
             Pn[u] = p;
             a.S[u] = kNone;
             if (p == kNone) {
@@ -414,12 +414,12 @@ __device__ __noinline__ void hub_phase_mc(const MatchArgs &a, MatchSmem &sm, int
 #pragma unroll
                 for (int q = 0; q < 8; ++q) {
                     const int32_t pp = px[q] >= 0 ? ldcg(Pk + px[q]) : -1;
-                    if (x[q] >= 0 && pp != x[q]) key = umax64(key, pack_key(a.tie_seed, w[q], x[q]));  // x free after round k
+                    if (x[q] >= 0 && pp != x[q]) key = umax64(key, pack_key(a.tie, w[q], x[q]));  // x free after round k
                 }
             } else {
 #pragma unroll
                 for (int q = 0; q < 8; ++q)
-                    if (x[q] >= 0) key = umax64(key, pack_key(a.tie_seed, w[q], x[q]));
+                    if (x[q] >= 0) key = umax64(key, pack_key(a.tie, w[q], x[q]));
             }
             key = group_max64<32>(key);
             if (lane == 0) sm.red[wib] = key;
@@ -439,7 +439,7 @@ __device__ __noinline__ void hub_phase_mc(const MatchArgs &a, MatchSmem &sm, int
     for (long long i = (long long)blockIdx.x * kNT + t; i < nhub; i += (long long)nact * kNT) {
         const int32_t u = a.H[i];
         const unsigned long long k = __ldcg(a.hk + i);
-        const int32_t p = key_vertex(a.tie_seed, k);
+        const int32_t p = key_vertex(a.tie, k);
         Pn[u] = p;
         a.S[u] = kNone;
         if (p == kNone) {
@@ -662,13 +662,13 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
             for (int b = 0; b < 4; ++b) pp[b] = px[b] >= 0 ? ldcg(Pk + px[b]) : -1;
 #pragma unroll
             for (int b = 0; b < 4; ++b)
-                if (x[b] >= 0 && pp[b] != x[b]) top2_add(key, key2, pack_key(a.tie_seed, w[b], x[b]));  // x free after round k
+                if (x[b] >= 0 && pp[b] != x[b]) top2_add(key, key2, pack_key(a.tie, w[b], x[b]));  // x free after round k
         }
         if (trips > 0) group_top2<G>(key, key2);
         if (need && gl == 0) {
-            const int32_t b = key_vertex(a.tie_seed, key);
+            const int32_t b = key_vertex(a.tie, key);
             Pn[u] = b;
-            a.S[u] = key_vertex(a.tie_seed, key2);
+            a.S[u] = key_vertex(a.tie, key2);
             if (b == kNone) Pkw[u] = kNone;  // dead: NONE in both buffers
             live = b != kNone;
         }
@@ -785,7 +785,7 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
 #pragma unroll
             for (int b = 0; b < kFB; ++b) {
                 const int32_t pp = px[b] >= 0 ? ldcg(Pk + px[b]) : -1;
-                key[b] = (x[b] >= 0 && pp != x[b]) ? pack_key(a.tie_seed, w[b], x[b]) : 0ull;  // x free after round k
+                key[b] = (x[b] >= 0 && pp != x[b]) ? pack_key(a.tie, w[b], x[b]) : 0ull;  // x free after round k
             }
             if (one) {
                 // top-2 of (w, ~x) per row with native 32-bit shared atomics, field by field
@@ -828,9 +828,9 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
             const int32_t r = rpos[i];
             const unsigned long long k1 = one ? (((unsigned long long)fq.w1[r] << 32) | fq.n1[r]) : fq.k1[r];
             const unsigned long long k2 = one ? (((unsigned long long)fq.w2[r] << 32) | fq.n2[r]) : fq.k2[r];
-            const int32_t bv = key_vertex(a.tie_seed, fq.w1[r] || !one ? k1 : 0ull);
+            const int32_t bv = key_vertex(a.tie, fq.w1[r] || !one ? k1 : 0ull);
             Pn[u[i]] = bv;
-            a.S[u[i]] = key_vertex(a.tie_seed, !one || fq.w2[r] ? k2 : 0ull);
+            a.S[u[i]] = key_vertex(a.tie, !one || fq.w2[r] ? k2 : 0ull);
             if (bv == kNone) Pkw[u[i]] = kNone;  // dead: NONE in both buffers
             live[i] = bv != kNone;
         }
@@ -1230,7 +1230,7 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     }
     a.ctl = ctl;
     a.max_rounds = max_rounds;
-    a.tie_seed = ctx->tie_seed;
+    a.tie = make_tie_hash(ctx->tie_seed);
     a.leftover = leftover ? 1 : 0;
     a.G = choose_group(avg_deg_hint);
     a.vpc = match_vpc();
