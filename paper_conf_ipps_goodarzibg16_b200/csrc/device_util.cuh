@@ -38,44 +38,32 @@ __device__ __forceinline__ unsigned lanemask_lt() {
 // random matching for equal weights (P18.s8): the lower h_s(v) = lowbias32(v ^ seed) wins.
 // lowbias32 is a bijection of uint32, so keys stay distinct per row and the termination
 // lemma (§2.1) holds unchanged (it is the default rule on the vertices relabeled by h_s).
-// Branch-free in the arc loops: with seed 0 the masks are 0 and the multipliers 1, so the
-// same instructions compute the identity (a per-arc branch split the unrolled gathers).
-struct TieHash {
-    uint32_t s, k;       // seed; k = ~0 if seed != 0 else 0 (masks the xorshifts)
-    uint32_t m1, m2;     // 0x7feb352d, 0x846ca68b (1, 1 for seed 0)
-    uint32_t i1, i2;     // their inverses mod 2^32: 0x1d69e2a5, 0x43021123 (1, 1)
-};
-inline TieHash make_tie_hash(uint32_t seed) {
-    const bool on = seed != 0;
-    return TieHash{seed, on ? 0xFFFFFFFFu : 0u, on ? 0x7feb352du : 1u, on ? 0x846ca68bu : 1u,
-                   on ? 0x1d69e2a5u : 1u, on ? 0x43021123u : 1u};
-}
-__device__ __forceinline__ uint32_t tie_hash(const TieHash &h, uint32_t v) {
-    uint32_t x = v ^ h.s;
-    x ^= (x >> 16) & h.k;
-    x *= h.m1;
-    x ^= (x >> 15) & h.k;
-    x *= h.m2;
-    x ^= (x >> 16) & h.k;
+// The level kernel is instantiated for H = (seed != 0), so the default rule keeps its
+// one-instruction tie word (a runtime test per arc, branched or masked, cost C3's match
+// kernel 4-7 %).
+__device__ __forceinline__ uint32_t tie_hash(uint32_t v, uint32_t s) {
+    uint32_t x = v ^ s;
+    x ^= x >> 16; x *= 0x7feb352du; x ^= x >> 15; x *= 0x846ca68bu; x ^= x >> 16;
     return x;
 }
-__device__ __forceinline__ uint32_t tie_unhash(const TieHash &h, uint32_t x) {
-    x ^= (x >> 16) & h.k;
-    x *= h.i2;
-    x ^= ((x >> 15) ^ (x >> 30)) & h.k;
-    x *= h.i1;
-    x ^= (x >> 16) & h.k;
-    return x ^ h.s;
+__device__ __forceinline__ uint32_t tie_unhash(uint32_t x, uint32_t s) {
+    x ^= x >> 16; x *= 0x43021123u; x ^= x >> 15; x ^= x >> 30; x *= 0x1d69e2a5u; x ^= x >> 16;
+    return x ^ s;
 }
 
 // Proposal key of neighbour v over edge weight w (P12.s23, R3): heavier first, then the
-// tie priority (lower id, or lower h_s(v) under a tie seed).  key > 0 for every valid
-// (w >= 1) arc; 0 means "no candidate".
-__device__ __forceinline__ unsigned long long pack_key(const TieHash &h, int32_t w, int32_t v) {
-    return ((unsigned long long)(uint32_t)w << 32) | (unsigned long long)(~tie_hash(h, (uint32_t)v));
+// tie priority (lower id, or lower h_s(v) when H).  key > 0 for every valid (w >= 1) arc;
+// 0 means "no candidate".
+template <bool H>
+__device__ __forceinline__ unsigned long long pack_key(uint32_t s, int32_t w, int32_t v) {
+    const uint32_t t = H ? tie_hash((uint32_t)v, s) : (uint32_t)v;
+    return ((unsigned long long)(uint32_t)w << 32) | (unsigned long long)(~t);
 }
-__device__ __forceinline__ int32_t key_vertex(const TieHash &h, unsigned long long k) {
-    return k ? (int32_t)tie_unhash(h, ~(uint32_t)k) : kNone;
+template <bool H>
+__device__ __forceinline__ int32_t key_vertex(uint32_t s, unsigned long long k) {
+    if (!k) return kNone;
+    const uint32_t t = ~(uint32_t)k;
+    return (int32_t)(H ? tie_unhash(t, s) : t);
 }
 
 __device__ __forceinline__ unsigned long long umax64(unsigned long long a, unsigned long long b) {

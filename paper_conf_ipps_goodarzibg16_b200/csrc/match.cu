@@ -76,7 +76,7 @@ struct MatchArgs {
     int32_t prof;        // GP_PROF=1: per-round slowest-warp times and rescan counts (MatchCtl)
     int32_t mode;  // kMatchWhole, or one launch per phase for the sharded path
     int32_t k;     // round of a kMatchRound launch
-    TieHash tie;  // tie priority: seed 0 = lower id wins (north_star); else RM (R17, P18.s8)
+    uint32_t tie_seed;  // 0: lower id wins ties (north_star); else RM tie priority (R17, P18.s8)
 };
 
 
@@ -210,6 +210,7 @@ __device__ __forceinline__ void load_bounds(const MatchArgs &a, int32_t n, long 
     }
 }
 
+template <bool H>
 __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned long long &scanned) {
     const int G = a.G;
     const int ngroups = kNT / G;
@@ -271,7 +272,7 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
             bool hub = false;
             if (fits) {
                 const int32_t *sa = sm.adj[st], *sw = sm.wgt[st];
-                for (int32_t j = s - A0 + gl; j < e - A0; j += G) top2_add(key, key2, pack_key(a.tie, sw[j], sa[j]));
+                for (int32_t j = s - A0 + gl; j < e - A0; j += G) top2_add(key, key2, pack_key<H>(a.tie_seed, sw[j], sa[j]));
             } else if (valid) {
                 if (e - s > kHubDeg) {
                     hub = true;
@@ -286,7 +287,7 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
                         }
 #pragma unroll
                         for (int q = 0; q < 8; ++q)
-                            if (xv[q] >= 0) top2_add(key, key2, pack_key(a.tie, wv[q], xv[q]));
+                            if (xv[q] >= 0) top2_add(key, key2, pack_key<H>(a.tie_seed, wv[q], xv[q]));
                     }
                 }
             }
@@ -304,9 +305,9 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
                     if (a.hk) a.hk[h] = 0ull;  // (sharded launches: per-CTA hub_phase, no hk)
                     a.S[x] = kNone;
                 } else {
-                    const int32_t p = key_vertex(a.tie, key);
+                    const int32_t p = key_vertex<H>(a.tie_seed, key);
                     P1[x] = p;
-                    a.S[x] = key_vertex(a.tie, key2);  // cached second-heaviest neighbour
+                    a.S[x] = key_vertex<H>(a.tie_seed, key2);  // cached second-heaviest neighbour
                     if (p == kNone) P0[x] = kNone;  // dead vertices: NONE in both buffers
                     scanned += (unsigned long long)(e - s);
                 }
@@ -329,6 +330,7 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
 // hub phase: every listed row (deg > kHubDeg) is scanned by a whole CTA
 // kCheck = false in round 1 (every vertex free), true for rescans after round k.
 // ---------------------------------------------------------------------------------------
+template <bool H>
 __device__ __noinline__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool check, const int32_t *Pk,
                           int32_t *Pn, int32_t *Lnext, int32_t *live_next, unsigned long long &scanned) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -338,7 +340,7 @@ __device__ __noinline__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_
         unsigned long long key = 0;
         for (int32_t j = s + threadIdx.x; j < e; j += kNT) {
             const int32_t x = __ldg(a.adjncy + j);
-            if (!check || free_after(x, Pk)) key = umax64(key, pack_key(a.tie, __ldg(a.adjwgt + j), x));
+            if (!check || free_after(x, Pk)) key = umax64(key, pack_key<H>(a.tie_seed, __ldg(a.adjwgt + j), x));
         }
         key = group_max64<32>(key);
         if (lane == 0) sm.red[wib] = key;
@@ -346,7 +348,7 @@ __device__ __noinline__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_
         if (threadIdx.x == 0) {
             unsigned long long k = 0;
             for (int q = 0; q < kNT / 32; ++q) k = umax64(k, sm.red[q]);
-            const int32_t p = key_vertex(a.tie, k);
+            const int32_t p = key_vertex<H>(a.tie_seed, k);
             Pn[u] = p;
             a.S[u] = kNone;
             if (p == kNone) {
@@ -368,6 +370,7 @@ __device__ __noinline__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_
 // proposals are written (top-1 only: S = NONE for hubs, as in hub_phase).  Every CTA walks the
 // hub list in segments of kNT hubs with a block scan of the chunk counts.
 constexpr int kHC = kNT * 8;  // arcs per hub chunk
+template <bool H>
 __device__ __noinline__ void hub_phase_mc(const MatchArgs &a, MatchSmem &sm, int32_t nhub, bool check, const int32_t *Pk,
                              int32_t *Pn, int32_t *Lnext, int32_t *live_next, unsigned long long &scanned,
                              unsigned *bar, unsigned &bar_epoch, int nact) {
@@ -414,12 +417,12 @@ __device__ __noinline__ void hub_phase_mc(const MatchArgs &a, MatchSmem &sm, int
 #pragma unroll
                 for (int q = 0; q < 8; ++q) {
                     const int32_t pp = px[q] >= 0 ? ldcg(Pk + px[q]) : -1;
-                    if (x[q] >= 0 && pp != x[q]) key = umax64(key, pack_key(a.tie, w[q], x[q]));  // x free after round k
+                    if (x[q] >= 0 && pp != x[q]) key = umax64(key, pack_key<H>(a.tie_seed, w[q], x[q]));  // x free after round k
                 }
             } else {
 #pragma unroll
                 for (int q = 0; q < 8; ++q)
-                    if (x[q] >= 0) key = umax64(key, pack_key(a.tie, w[q], x[q]));
+                    if (x[q] >= 0) key = umax64(key, pack_key<H>(a.tie_seed, w[q], x[q]));
             }
             key = group_max64<32>(key);
             if (lane == 0) sm.red[wib] = key;
@@ -439,7 +442,7 @@ __device__ __noinline__ void hub_phase_mc(const MatchArgs &a, MatchSmem &sm, int
     for (long long i = (long long)blockIdx.x * kNT + t; i < nhub; i += (long long)nact * kNT) {
         const int32_t u = a.H[i];
         const unsigned long long k = __ldcg(a.hk + i);
-        const int32_t p = key_vertex(a.tie, k);
+        const int32_t p = key_vertex<H>(a.tie_seed, k);
         Pn[u] = p;
         a.S[u] = kNone;
         if (p == kNone) {
@@ -562,7 +565,7 @@ __device__ __noinline__ void wake_phase(const MatchArgs &a, MatchSmem &sm, int32
 // 32/G vertices and a rescan reads G*4 arcs per dependent step instead of 8 per thread.
 // The round's critical path is then ~8 dependent loads whatever the row length (<= kHubDeg).
 // Same decisions as phase_k_impl (commit / keep p / cached second choice / rescan).
-template <int G>
+template <int G, bool H>
 __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t len, bool park, const int32_t *Lover,
                               unsigned long long &scanned, unsigned long long &rows, unsigned long long &visits,
                               int32_t &made) {
@@ -662,13 +665,13 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
             for (int b = 0; b < 4; ++b) pp[b] = px[b] >= 0 ? ldcg(Pk + px[b]) : -1;
 #pragma unroll
             for (int b = 0; b < 4; ++b)
-                if (x[b] >= 0 && pp[b] != x[b]) top2_add(key, key2, pack_key(a.tie, w[b], x[b]));  // x free after round k
+                if (x[b] >= 0 && pp[b] != x[b]) top2_add(key, key2, pack_key<H>(a.tie_seed, w[b], x[b]));  // x free after round k
         }
         if (trips > 0) group_top2<G>(key, key2);
         if (need && gl == 0) {
-            const int32_t b = key_vertex(a.tie, key);
+            const int32_t b = key_vertex<H>(a.tie_seed, key);
             Pn[u] = b;
-            a.S[u] = key_vertex(a.tie, key2);
+            a.S[u] = key_vertex<H>(a.tie_seed, key2);
             if (b == kNone) Pkw[u] = kNone;  // dead: NONE in both buffers
             live = b != kNone;
         }
@@ -702,7 +705,7 @@ struct FlatQ {
 static_assert(sizeof(FlatQ) * (kNT / 32) <= sizeof(int32_t) * ((kStages - 1) * kStageArcs + kStages * kStageArcs),
               "flat rescan queues must fit the idle phase-0 buffers");
 
-template <int kVL>
+template <int kVL, bool H>
 __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, const int32_t *Pk, int32_t *Pn,
                                             int32_t *Pkw, RoundSlot *next, const int32_t (&u)[kVL],
                                             bool (&need)[kVL], bool (&live)[kVL], unsigned long long &scanned,
@@ -785,7 +788,7 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
 #pragma unroll
             for (int b = 0; b < kFB; ++b) {
                 const int32_t pp = px[b] >= 0 ? ldcg(Pk + px[b]) : -1;
-                key[b] = (x[b] >= 0 && pp != x[b]) ? pack_key(a.tie, w[b], x[b]) : 0ull;  // x free after round k
+                key[b] = (x[b] >= 0 && pp != x[b]) ? pack_key<H>(a.tie_seed, w[b], x[b]) : 0ull;  // x free after round k
             }
             if (one) {
                 // top-2 of (w, ~x) per row with native 32-bit shared atomics, field by field
@@ -828,9 +831,9 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
             const int32_t r = rpos[i];
             const unsigned long long k1 = one ? (((unsigned long long)fq.w1[r] << 32) | fq.n1[r]) : fq.k1[r];
             const unsigned long long k2 = one ? (((unsigned long long)fq.w2[r] << 32) | fq.n2[r]) : fq.k2[r];
-            const int32_t bv = key_vertex(a.tie, fq.w1[r] || !one ? k1 : 0ull);
+            const int32_t bv = key_vertex<H>(a.tie_seed, fq.w1[r] || !one ? k1 : 0ull);
             Pn[u[i]] = bv;
-            a.S[u[i]] = key_vertex(a.tie, !one || fq.w2[r] ? k2 : 0ull);
+            a.S[u[i]] = key_vertex<H>(a.tie_seed, !one || fq.w2[r] ? k2 : 0ull);
             if (bv == kNone) Pkw[u[i]] = kNone;  // dead: NONE in both buffers
             live[i] = bv != kNone;
         }
@@ -845,7 +848,7 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
 // vertices keep their partner in P, dead ones NONE), read at the same level as P_k[u].  No list
 // load, no list append and no atomic with a return value on the round's critical path; the
 // next round's live count is a fire-and-forget reduction.
-template <int kVL, bool kStatic = false>
+template <bool H, int kVL, bool kStatic = false>
 __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t len, bool park, const int32_t *Lover,
                              unsigned long long &scanned, unsigned long long &rows, unsigned long long &visits,
                              int32_t &made) {
@@ -947,10 +950,10 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
             for (int i = 0; i < kVL; ++i)
                 if (need[i] && re[i] - rs[i] <= kHubDeg) dsum += re[i] - rs[i];
             if (kVL >= 2 && warp_sum(dsum) > 32 * kFB) {
-                flat_rescan<kVL>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re, 0, kVL / 2);
-                flat_rescan<kVL>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re, kVL / 2, kVL);
+                flat_rescan<kVL, H>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re, 0, kVL / 2);
+                flat_rescan<kVL, H>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re, kVL / 2, kVL);
             } else {
-                flat_rescan<kVL>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re);
+                flat_rescan<kVL, H>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re);
             }
         }
         if (kStatic) {
@@ -969,6 +972,7 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
     }
 }
 
+template <bool H>
 __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, bool stat, bool park,
                         const int32_t *Lover, unsigned long long &scanned, unsigned long long &rows,
                         unsigned long long &visits, int32_t &made) {
@@ -981,13 +985,13 @@ __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int
     }
     const long long threads = (long long)g_nact * kNT;
     if (stat) {
-        if ((long long)len > threads) phase_k_impl<2, true>(a, sm, k, len, false, nullptr, scanned, rows, visits, made);
-        else phase_k_impl<1, true>(a, sm, k, len, false, nullptr, scanned, rows, visits, made);
-    } else if ((long long)len >= 4LL * threads) phase_k_impl<4>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
-    else if (a.lanes_mode == 0 || (long long)len * 2 > threads) phase_k_impl<1>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
-    else if ((long long)len * 8 <= threads) phase_k_lanes<8>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
-    else if ((long long)len * 4 <= threads) phase_k_lanes<4>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
-    else phase_k_lanes<2>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
+        if ((long long)len > threads) phase_k_impl<H, 2, true>(a, sm, k, len, false, nullptr, scanned, rows, visits, made);
+        else phase_k_impl<H, 1, true>(a, sm, k, len, false, nullptr, scanned, rows, visits, made);
+    } else if ((long long)len >= 4LL * threads) phase_k_impl<H, 4>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
+    else if (a.lanes_mode == 0 || (long long)len * 2 > threads) phase_k_impl<H, 1>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
+    else if ((long long)len * 8 <= threads) phase_k_lanes<8, H>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
+    else if ((long long)len * 4 <= threads) phase_k_lanes<4, H>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
+    else phase_k_lanes<2, H>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
     if (a.prof && k < 16) {  // one shared atomic per warp, one global atomic per CTA
         const unsigned long long dt = globaltimer() - t0;
         const int32_t dr = warp_sum((int32_t)(rows - rows0));
@@ -1005,6 +1009,7 @@ __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int
     }
 }
 
+template <bool H>
 __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ MatchArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     // 128-byte alignment by POINTER arithmetic on the __shared__ symbol: the compiler keeps the
@@ -1028,17 +1033,17 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
     int tr = 0;
     if (a.mode == kMatchWhole || a.mode == kMatchPhase0) {
         trace_mark(ctl->trace, tr++);
-        phase0(a, sm, n, scanned);
+        phase0<H>(a, sm, n, scanned);
         trace_mark(ctl->trace, tr++);
         grid_barrier(ctl->bar, bar_epoch, g_nact);
         trace_mark(ctl->trace, tr++);
         const int32_t nh = *(volatile int32_t *)&ctl->slot[1].nhub;
         if (nh > 0) {
             if (a.mode == kMatchWhole) {
-                hub_phase_mc(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned, ctl->bar, bar_epoch, g_nact);
+                hub_phase_mc<H>(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned, ctl->bar, bar_epoch, g_nact);
                 grid_barrier(ctl->bar, bar_epoch, g_nact);
             } else {
-                hub_phase(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned);
+                hub_phase<H>(a, sm, nh, false, a.P[0], a.P[1], nullptr, nullptr, scanned);
             }
         }
     }
@@ -1065,7 +1070,7 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
             }
             const int32_t len = (k == 1 || stat) ? n : known_len >= 0 ? known_len : *(volatile int32_t *)&ctl->slot[k & 3].live;
             int32_t made = 0;
-            phase_k(a, sm, n, k, len, stat, park, nullptr, scanned, rows, visits, made);
+            phase_k<H>(a, sm, n, k, len, stat, park, nullptr, scanned, rows, visits, made);
             // any match this round: one flag store per CTA (only "> 0" is used)
             if (__syncthreads_or(made > 0) && threadIdx.x == 0) *(volatile int32_t *)&ctl->slot[k & 3].matches = 1;
             trace_mark(ctl->trace, tr++);
@@ -1095,7 +1100,7 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
                     const int32_t nr = *(volatile int32_t *)&ctl->nres[k & 3];
                     if (nr > 0) {
                         int32_t made2 = 0;
-                        phase_k(a, sm, n, k, nr, false, true, a.R, scanned, rows, visits, made2);
+                        phase_k<H>(a, sm, n, k, nr, false, true, a.R, scanned, rows, visits, made2);
                         if (tail) __syncthreads();
                         else grid_barrier(ctl->bar, bar_epoch, nact_all);
                     }
@@ -1105,10 +1110,10 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
             int32_t live = nxt.x;
             if (nxt.y > 0) {
                 if (a.mode == kMatchWhole && !tail)
-                    hub_phase_mc(a, sm, nxt.y, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1],
+                    hub_phase_mc<H>(a, sm, nxt.y, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1],
                                  &ctl->slot[(k + 1) & 3].live, scanned, ctl->bar, bar_epoch, nact_all);
                 else
-                    hub_phase(a, sm, nxt.y, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1],
+                    hub_phase<H>(a, sm, nxt.y, true, a.P[k & 1], a.P[(k + 1) & 1], a.L[(k + 1) & 1],
                               &ctl->slot[(k + 1) & 3].live, scanned);
                 if (tail) __syncthreads();
                 else grid_barrier(ctl->bar, bar_epoch, nact_all);
@@ -1191,8 +1196,12 @@ int match_grid(Ctx *ctx) {
     static int per_sm = -1;
     if (per_sm < 0) {
         int b = 0;
-        cudaFuncSetAttribute(k_match_level, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(MatchSmem) + 128);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_match_level, kNT, sizeof(MatchSmem) + 128);
+        cudaFuncSetAttribute(k_match_level<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(MatchSmem) + 128);
+        cudaFuncSetAttribute(k_match_level<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(MatchSmem) + 128);
+        int b1 = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_match_level<false>, kNT, sizeof(MatchSmem) + 128);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b1, k_match_level<true>, kNT, sizeof(MatchSmem) + 128);
+        if (b1 < b) b = b1;  // one persistent grid size for both instantiations
         per_sm = b > 0 ? (b > 2 ? 2 : b) : 1;
     }
     return ctx->num_sms * per_sm;
@@ -1230,7 +1239,7 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     }
     a.ctl = ctl;
     a.max_rounds = max_rounds;
-    a.tie = make_tie_hash(ctx->tie_seed);
+    a.tie_seed = ctx->tie_seed;
     a.leftover = leftover ? 1 : 0;
     a.G = choose_group(avg_deg_hint);
     a.vpc = match_vpc();
@@ -1277,7 +1286,7 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     }
     void *args[] = {&a};
     LaunchScope ls(ctx, GP_K_PROPOSE);
-    GP_CUDA(cudaLaunchCooperativeKernel((const void *)k_match_level, dim3(match_grid(ctx)), dim3(kNT), args,
+    GP_CUDA(cudaLaunchCooperativeKernel(a.tie_seed ? (const void *)k_match_level<true> : (const void *)k_match_level<false>, dim3(match_grid(ctx)), dim3(kNT), args,
                                         sizeof(MatchSmem) + 128, ctx->stream));
     ++ctx->launches;
     return GP_OK;

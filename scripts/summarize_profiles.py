@@ -39,7 +39,7 @@ def launch_table(path):
                            h.index("Metric Unit"), h.index("ID"))
     per = collections.OrderedDict()
     for r in rows[hi + 1:]:
-        key = (int(r[idi]), r[ki].split("(")[0].replace("void ", "").replace("gp::", ""))
+        key = (int(r[idi]), r[ki].split("(")[0].split("<")[0].replace("void ", "").replace("gp::", ""))
         v = float(r[vi].replace(",", ""))
         scale = {"ns": 1e-3, "nsecond": 1e-3, "us": 1.0, "usecond": 1.0, "ms": 1e3, "msecond": 1e3,
                  "byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(r[ui], 1.0)
