@@ -118,6 +118,28 @@ def test_rm_breaks_unit_wavefront():
         assert lv[-1]["coarse"]["vwgt"].sum() == 4096
 
 
+def star(leaves: int, w: int = 1):
+    return G.from_edge_list(leaves + 1, [(0, i, w) for i in range(1, leaves + 1)])
+
+
+@pytest.mark.parametrize("s", SEEDS)
+def test_seeded_star_closed_form(s):
+    # every leaf proposes to the hub; the hub proposes to the leaf of lowest h_s, which is
+    # its partner; every other leaf is then dead (its only neighbour is matched)
+    n = 3001
+    m, rounds, maximal = oracle.match_level(star(n - 1), tie_seed=s)
+    best = min(range(1, n), key=lambda v: lowbias32(v, s))
+    assert m[0] == best and m[best] == 0 and rounds == 1 and maximal
+    assert all(m[v] == v for v in range(1, n) if v != best)
+
+
+def test_seeded_max_rounds_cap():
+    g = G.grid2d(16, 16)
+    m, r, maximal = oracle.match_level(g, max_rounds=1, tie_seed=SEEDS[1])
+    assert r == 1 and not maximal
+    check_matching(g, m, maximal=False)
+
+
 # ----------------------------------------------------------------------------- GPU parity
 
 GPU_GRAPHS = {
@@ -129,6 +151,9 @@ GPU_GRAPHS = {
     "rmat13_unit": lambda: G.rmat(13, 8, unit=True),
     "rmat14_w4": lambda: G.rmat(14, 16, wmax=4),
     "random_w1": lambda: G.random_graph(5000, 20000, seed=3, wmax=1),
+    "star3000": lambda: star(3000),                      # hub row > 1024 arcs: hub phases
+    "star50000": lambda: star(50000),                    # multi-CTA hub phase
+    "isolated": lambda: G.from_edge_list(50, [(3, 7, 1), (7, 9, 1)]),
 }
 
 
@@ -177,3 +202,13 @@ def test_gpu_seeded_loopback_equals_oracle(gp, name, nranks):
     ref = oracle.coarsen_to(g, threshold=20, tie_seed=SEEDS[1])
     got = gpu_coarsen(gp, gp.Context(0, loopback=nranks), g, threshold=20, tie_seed=SEEDS[1])
     assert_levels_equal(got, ref, f"{name} G={nranks}")
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("name", ["grid96_unit", "rmat13_unit"])
+def test_gpu_seeded_max_rounds_cap(gp, name):
+    from gpu_helpers import assert_levels_equal, gpu_coarsen
+    g = _host(GPU_GRAPHS[name]())
+    ref = oracle.coarsen_to(g, threshold=20, max_rounds=2, tie_seed=SEEDS[2])
+    got = gpu_coarsen(gp, gp.Context(0), g, threshold=20, max_rounds=2, tie_seed=SEEDS[2])
+    assert_levels_equal(got, ref, f"{name} cap")
