@@ -8,7 +8,9 @@ cmap, contraction and CSR assembly) of the BASELINE.json workload, input residen
   value   whole-job aggregate over all ranks
   e2e     the same metric through the C ABI with HOST buffers: pinned H2D of the CSR,
           gp_graph_create + gp_coarsen_to, D2H of every level's cmap + the coarsest graph
-  roofline  dominant kernel family, algorithmic bytes (DESIGN.md §5) / CUDA-event time
+  roofline  dominant kernel family, algorithmic bytes (SURVEY §8(d), DESIGN.md §5) / CUDA-event time
+  levels    per level: n, nnz, rounds, match / contract us, edges/s, §8(d) bytes, GB/s, fraction
+  level0    the level-0 match / contract roofline fractions (north_star's target)
   cpu_baseline  the oracle (oracle/, single thread) on the box's host, bounded sample
 
 --impl reference times the oracle (the reference arm of this tier) on the same config.
@@ -53,42 +55,43 @@ def peaks():
 
 
 # ------------------------------------------------------------------------------------------
-# algorithmic byte model per kernel family; int32 everywhere
+# algorithmic byte model per kernel family: SURVEY.md §8(d), int32 everywhere
 # ------------------------------------------------------------------------------------------
 def level_bytes(l) -> dict:
-    """Algorithmic HBM bytes of one level per kernel family.
+    """Compulsory HBM bytes of one level, from the device counters the level
+    reports: S = arcs scanned by the proposals (all rounds, round 1 included), V_s = rows
+    scanned, L = live vertex visits of the commits, R = rounds.
 
-    match    (k_match_level: A1-A4, every round)
-      phase 0   adjp 4(n+1) + adjncy/adjwgt 8*nnz + P and M writes 8n
-      rounds    per live visit: list entry, P[u], P[p], P[q], one write, one append (24 B)
-      rescans   8 B per rescanned arc + adjp pair and P write per rescanned row (12 B)
-                + M gathers, each M entry counted at most once per round
-    contract (k_contract_level: A4 leftover + A5-A8)
-      C1        M 4n, CM 4n, adjp of leader+partner 8n, vwgt 4n, leaders/cvwgt/off 12 n_c
-      C2        off/leaders/M/cnt per coarse row 24 n_c, adjp 8n, adjncy+adjwgt 8 nnz,
-                CM gathers (each entry once) 4n, cadjp 4 n_c, cadjncy+cadjwgt 8 cnnz
+      A1 degree binning        12 n
+      A2 propose               8 S + 12 V_s + min(4 (S - nnz), 4 n (R - 1))
+      A3 commit                12 L
+      A5 cmap                  12 n + 4 n_c
+      A6-A8 contraction        12 n + 8 nnz + 4 n + 8 cnnz + 12 n_c   (single-pass assembly)
+
+    match = A1 + A2 + A3 (k_match_level), contract = A5 + A6-A8 (k_contract_level).
     """
     n, nnz, nc, cnnz = l["n"], l["nnz"], l["n_coarse"], l["cnnz"]
     S, Vs, R, L = l["arcs_scanned"], l["rows_scanned"], max(l["rounds"], 1), l["live_visits"]
-    rescan_arcs = max(S - nnz, 0)
-    rescan_rows = max(Vs - n, 0)
-    match = (4 * (n + 1) + 8 * nnz + 8 * n) + 24 * L + 8 * rescan_arcs + 12 * rescan_rows \
-        + min(4 * rescan_arcs, 4 * n * (R - 1))
-    contract = (20 * n + 12 * nc) + (24 * nc + 8 * n + 8 * nnz + 4 * n + 4 * nc + 8 * cnnz)
-    return {"match": match, "contract": contract}
+    a1 = 12 * n
+    a2 = 8 * S + 12 * Vs + min(4 * max(S - nnz, 0), 4 * n * (R - 1))
+    a3 = 12 * L
+    a5 = 12 * n + 4 * nc
+    a678 = 12 * n + 8 * nnz + 4 * n + 8 * cnnz + 12 * nc
+    return {"match": a1 + a2 + a3, "contract": a5 + a678}
 
 
 def ncu_traffic(config: str, kernel: str):
     """DRAM bytes (read + write) per step of `kernel` from the committed ncu launch list
     (profiles/r1/ncu_traffic_<config>.json, written by scripts/summarize_profiles.py from one
     profiled gp_coarsen_to), or None when no capture of this config is committed."""
-    path = os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "r1",
-                        f"ncu_traffic_{config}.json")
-    try:
-        j = json.load(open(path))
-        return float(j["kernels"][kernel]["dram_bytes"]), "profiles/r1/" + os.path.basename(path)
-    except Exception:
-        return None
+    for rnd in ("r2", "r1"):
+        path = os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", rnd, f"ncu_traffic_{config}.json")
+        try:
+            j = json.load(open(path))
+            return float(j["kernels"][kernel]["dram_bytes"]), f"profiles/{rnd}/" + os.path.basename(path)
+        except Exception:
+            continue
+    return None
 
 
 # ------------------------------------------------------------------------------------------
@@ -110,6 +113,12 @@ class ClockSampler:
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.thread = threading.Thread(target=self._read, daemon=True)
             self.thread.start()
+            # the timed region starts only once the sampler is producing samples (nvidia-smi
+            # takes ~0.1-0.5 s to start; a short region would otherwise see none)
+            t0 = time.time()
+            while not self.lines and time.time() - t0 < 5.0:
+                time.sleep(0.01)
+            self.skip = len(self.lines)  # samples taken before the region are not counted
         except Exception:
             self.proc = None
         return self
@@ -129,7 +138,7 @@ class ClockSampler:
     def summary(self):
         sm, mx, reasons = [], 0, set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
+        for ln in self.lines[getattr(self, "skip", 0):]:
             parts = [p.strip() for p in ln.split(",")]
             if len(parts) < 6:
                 continue
@@ -149,18 +158,18 @@ class ClockSampler:
 # ------------------------------------------------------------------------------------------
 # oracle timing (cpu_baseline and --impl reference)
 # ------------------------------------------------------------------------------------------
-def oracle_run(g, threshold, tie_seed=0):
+def oracle_run(g, threshold, tie_seed=0, max_rounds=0):
     import oracle
     t0 = time.perf_counter()
-    levels = oracle.coarsen_to(g, threshold, tie_seed=tie_seed)
+    levels = oracle.coarsen_to(g, threshold, tie_seed=tie_seed, max_rounds=max_rounds)
     dt = time.perf_counter() - t0
     return dt, sum(l["nnz"] // 2 for l in levels), len(levels)
 
 
-def cpu_baseline(g, threshold, budget_s=12.0, tie_seed=0):
+def cpu_baseline(g, threshold, budget_s=12.0, tie_seed=0, max_rounds=0):
     runs, tot_t, tot_e, nlev = 0, 0.0, 0, 0
     while runs == 0 or tot_t < budget_s:
-        dt, e, nlev = oracle_run(g, threshold, tie_seed)
+        dt, e, nlev = oracle_run(g, threshold, tie_seed, max_rounds)
         runs += 1
         tot_t += dt
         tot_e += e
@@ -212,7 +221,7 @@ def run_ours(args, rank, world, local_rank):
     stream = ctx.stream
 
     def step():
-        return graph.coarsen_to(threshold, tie_seed=args.tie_seed)
+        return graph.coarsen_to(threshold, tie_seed=args.tie_seed, max_rounds=args.max_rounds)
 
     # warm-up
     hier = None
@@ -241,6 +250,7 @@ def run_ours(args, rank, world, local_rank):
     ms = ev0.elapsed_time(ev1)
     launches = ctx.launch_count() - launches0
     kstats = ctx.kernel_stats()
+    ltimes = ctx.launch_times()   # (kind, ms) of every launch of the timed steps, in order
     ctx.set_timing(False)
     # untimed-instrumentation check: the same steps without event brackets
     torch.cuda.synchronize()
@@ -273,6 +283,29 @@ def run_ours(args, rank, world, local_rank):
     achieved = fam_bytes[dom] / (fam_ms[dom] / 1e3) / 1e9 if fam_ms[dom] > 0 else 0.0
     step_bytes = sum(fam_bytes.values())
     traffic = ncu_traffic(args.config, {"match": "k_match_level", "contract": "k_contract_level"}[dom])
+
+    # per-level rows (BASELINE metric "fine edges coarsened/sec per level"): each step enqueues
+    # level l's matching then its contraction (speculative levels after the stop come last);
+    # the median over the timed steps of each launch's CUDA-event time
+    per_step = len(ltimes) // args.steps if args.steps else 0
+    level_rows = []
+    if not sharded and args.loopback <= 1 and per_step >= 2 * len(levels):
+        for i, l in enumerate(levels):
+            t = {}
+            for fam, kind, off in (("match", "propose", 0), ("contract", "contract", 1)):
+                xs = [ltimes[st * per_step + 2 * i + off] for st in range(args.steps)]
+                assert all(k == kind for k, _ in xs), "launch order does not map to levels"
+                t[fam] = statistics.median(m for _, m in xs)
+            b = level_bytes(l)
+            tl = t["match"] + t["contract"]
+            level_rows.append({
+                "level": i, "n": l["n"], "nnz": l["nnz"], "n_coarse": l["n_coarse"], "cnnz": l["cnnz"],
+                "rounds": l["rounds"], "match_us": round(1e3 * t["match"], 2), "contract_us": round(1e3 * t["contract"], 2),
+                "edges_per_s": (l["nnz"] // 2) / (tl / 1e3),
+                "bytes_match": b["match"], "bytes_contract": b["contract"],
+                "GBps_match": b["match"] / (t["match"] / 1e3) / 1e9, "GBps_contract": b["contract"] / (t["contract"] / 1e3) / 1e9,
+                "frac_match": b["match"] / (t["match"] / 1e3) / 1e9 / peak,
+                "frac_contract": b["contract"] / (t["contract"] / 1e3) / 1e9 / peak})
 
     # projection: a synthetic labelling of the coarsest graph (c mod 64)
     # carried down to level 0 in one launch; algorithmic bytes = CM_0 read + labels written +
@@ -318,7 +351,7 @@ def run_ours(args, rank, world, local_rank):
             gh = gp.Graph.create_dist(ctx, n, vb, host["adjp"], host["adjncy"], host["adjwgt"], host["vwgt"])
         else:
             gh = gp.Graph.create(ctx, host["adjp"], host["adjncy"], host["adjwgt"], host["vwgt"])
-        hh = gh.coarsen_to(threshold, tie_seed=args.tie_seed)
+        hh = gh.coarsen_to(threshold, tie_seed=args.tie_seed, max_rounds=args.max_rounds)
         nb = 0
         for i in range(len(hh)):
             _, c = hh.download_level(i, cmap=cm_bufs[i], want_match=False)
@@ -338,16 +371,26 @@ def run_ours(args, rank, world, local_rank):
         "metric": METRIC, "value": edges_per_step / (ms_step / 1e3), "unit": UNIT, "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
         "scaling": "strong" if sharded else "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-        "config": {"workload": f"{args.config}:{name}" + (f":rm_seed{args.tie_seed:#x}" if args.tie_seed else ""), "n": n, "edges": nnz // 2, "threshold": threshold,
+        "config": {"workload": f"{args.config}:{name}" + (f":rm_seed{args.tie_seed:#x}" if args.tie_seed else "")
+                   + (f":max_rounds{args.max_rounds}" if args.max_rounds else ""), "n": n, "edges": nnz // 2, "threshold": threshold,
                    "levels": len(levels), "edges_all_levels": edges_per_step,
-                   "level0_edges_per_s": (nnz // 2) / (ms_step / 1e3),
+                   "level0_edges_per_s": level_rows[0]["edges_per_s"] if level_rows else None,
                    "t_full_ms": ms_step, "rounds": [l["rounds"] for l in levels],
+                   "n_final": levels[-1]["n_coarse"], "stop_reason": levels[-1]["stop_reason"],
+                   "shrink_per_level": [round(l["n_coarse"] / l["n"], 4) for l in levels],
                    "l2": f"L0 input {(4 * (2 * nnz + 2 * n)) / 2**20:.0f} MiB > L2 126 MiB (no flush)",
                    "parallelism": (f"sharded x{world}: vertex ranges, NCCL all-gather per handshake round"
                                    if sharded else f"loopback x{args.loopback} on 1 GPU (sharded protocol simulated)"
                                    if args.loopback > 1 else "single GPU"),
                    "gen_s": round(gen_s, 2)},
         "hbm_gbs_step": step_bytes / (ms_step / 1e3) / 1e9,
+        # north_star's target: >= 50 % of HBM roofline on the matching and contraction kernels of
+        # the 2^22 mesh -- their level-0 launches, SURVEY §8(d) bytes / CUDA-event time
+        "level0": ({"match_frac": level_rows[0]["frac_match"], "contract_frac": level_rows[0]["frac_contract"],
+                    "match_us": level_rows[0]["match_us"], "contract_us": level_rows[0]["contract_us"],
+                    "edges_per_s": level_rows[0]["edges_per_s"], "peak_GBps": peak, "peak_kind": peak_kind}
+                   if level_rows else None),
+        "levels": level_rows,
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "peak_kind": peak_kind,
                      "unit": "GB/s", "frac": achieved / peak,
                      "traffic": traffic[0] if traffic else None,
@@ -363,7 +406,7 @@ def run_ours(args, rank, world, local_rank):
     }
     if rank == 0 and not args.no_cpu_baseline:
         gh = {k: g[k].cpu() for k in ("adjp", "adjncy", "adjwgt", "vwgt")}
-        line["cpu_baseline"] = cpu_baseline(gh, threshold, tie_seed=args.tie_seed)
+        line["cpu_baseline"] = cpu_baseline(gh, threshold, tie_seed=args.tie_seed, max_rounds=args.max_rounds)
         line["cpu_baseline"].update(host_info())
     graph.close()
     ctx.close()
@@ -376,18 +419,19 @@ def run_reference(args, rank, world):
         return None
     g, _ = make_graph(args.config, "cpu")
     for _ in range(args.warmup):
-        oracle_run(g, threshold, args.tie_seed)
+        oracle_run(g, threshold, args.tie_seed, args.max_rounds)
     t = 0.0
     e = 0
     for _ in range(args.steps):
-        dt, e, nlev = oracle_run(g, threshold, args.tie_seed)
+        dt, e, nlev = oracle_run(g, threshold, args.tie_seed, args.max_rounds)
         t += dt
     ms = t / args.steps * 1e3
     value = e / (ms / 1e3)
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-            "config": {"workload": f"{args.config}:{name}" + (f":rm_seed{args.tie_seed:#x}" if args.tie_seed else ""), "n": g["n"], "edges": g["nnz"] // 2,
+            "config": {"workload": f"{args.config}:{name}" + (f":rm_seed{args.tie_seed:#x}" if args.tie_seed else "")
+                       + (f":max_rounds{args.max_rounds}" if args.max_rounds else ""), "n": g["n"], "edges": g["nnz"] // 2,
                        "threshold": threshold, "edges_all_levels": e},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
                              "sample": f"full coarsen-to-{threshold} per step, single-threaded C oracle"},
@@ -399,11 +443,13 @@ def run_reference(args, rank, world):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--config", choices=sorted(WORKLOADS), default="C3")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--max-rounds", type=int, default=0,
+                    help="cap the handshake rounds per level (1 = the paper's one-shot HEM + conflict pass, P18.s7-13)")
     ap.add_argument("--loopback", type=int, default=0,
                     help="run the sharded protocol with this many simulated ranks on one GPU")
     ap.add_argument("--tie-seed", type=lambda x: int(x, 0), default=0,

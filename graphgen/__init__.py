@@ -106,6 +106,34 @@ def csr_from_edges(n: int, u: torch.Tensor, v: torch.Tensor, w: torch.Tensor,
     }
 
 
+def shuffle_rows(g: Dict[str, object], seed: int) -> Dict[str, object]:
+    """The same graph with every row's neighbours in a seeded pseudo-random order (input
+    contract R15: any neighbour order is valid).  Arcs are permuted inside their row by the
+    key (row, h(seed, arc index)); weights move with their arcs."""
+    adjp = g["adjp"]
+    dev = adjp.device
+    n = adjp.numel() - 1
+    nnz = int(adjp[-1]) if n >= 0 else 0
+    out = dict(g)
+    if nnz == 0:
+        return out
+    row = torch.repeat_interleave(torch.arange(n, device=dev, dtype=torch.int64), torch.diff(adjp).to(torch.int64))
+    r = _srl(h(7000 + seed, torch.arange(nnz, device=dev, dtype=torch.int64)), 33)  # 31 random bits
+    perm = torch.argsort((row << 31) | r)
+    out["adjncy"] = g["adjncy"][perm].contiguous()
+    out["adjwgt"] = g["adjwgt"][perm].contiguous()
+    out["name"] = f"{g.get('name', '')}_shuf{seed}"
+    return out
+
+
+def varied_vwgt(g: Dict[str, object], period: int = 7) -> Dict[str, object]:
+    """The same graph with non-unit vertex weights vwgt[u] = 1 + u mod period."""
+    n = g["adjp"].numel() - 1
+    out = dict(g)
+    out["vwgt"] = (1 + torch.arange(n, device=g["adjp"].device, dtype=torch.int64) % period).to(torch.int32)
+    return out
+
+
 def _unique_pairs(u: torch.Tensor, v: torch.Tensor) -> (torch.Tensor, torch.Tensor):
     """Drop self-loops, orient u<v, deduplicate."""
     keep = u != v

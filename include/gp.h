@@ -25,6 +25,8 @@
  *   * Handles (gp_ctx, gp_graph, gp_hier) are library-owned and released with gp_free.
  *     A graph or hierarchy must be freed before its context.  Handles are not
  *     thread-safe; use one context per host thread.
+ *   * Devices: every call runs on its handle's device and leaves the calling thread's current
+ *     CUDA device as it found it, so contexts on several devices can be mixed in one process.
  */
 #ifndef GP_H
 #define GP_H
@@ -49,7 +51,7 @@ typedef enum {
     GP_ERR_OVERFLOW = 3,      /* sum(vwgt) or sum(adjwgt) exceeds INT32_MAX (R14)       */
     GP_ERR_OUT_OF_MEMORY = 4, /* device or pinned-host allocation failed               */
     GP_ERR_CUDA = 5,          /* a CUDA runtime call failed; see gp_last_error()       */
-    GP_ERR_NCCL = 6,          /* reserved for the sharded path                          */
+    GP_ERR_NCCL = 6,          /* an NCCL call of the sharded path failed (or libnccl is missing) */
     GP_ERR_INTERNAL = 7       /* library invariant violated (a bug)                     */
 } gp_status;
 
@@ -68,6 +70,10 @@ typedef void (*gp_dealloc_fn)(void *ptr, void *stream, void *user);
  *   cuda_stream  cudaStream_t to enqueue on (NULL = the legacy default stream).
  * Fails with GP_ERR_CUDA when the device is absent (there is no CPU fallback). */
 gp_status gp_ctx_create(int device, void *cuda_stream, gp_ctx *out);
+/* Route the context's device allocations through alloc/dealloc (both or neither; NULL, NULL
+ * restores cudaMallocAsync).  GP_ERR_INVALID_ARG while graphs or hierarchies created on this
+ * context are alive (their buffers would be released through the wrong allocator); the
+ * context's internal scratch is released first.  Synchronous. */
 gp_status gp_ctx_set_allocator(gp_ctx ctx, gp_alloc_fn alloc, gp_dealloc_fn dealloc, void *user);
 /* Number of SMs of the context's device (launch sizing is a multiple of it). */
 gp_status gp_ctx_num_sms(gp_ctx ctx, int32_t *out);
@@ -85,9 +91,10 @@ gp_status gp_ctx_num_sms(gp_ctx ctx, int32_t *out);
  *           memory makes the copy asynchronous).
  *           GP_VALIDATE: GP_ERR_INVALID_GRAPH unless adjp[0]=0, adjp monotone, ids in
  *           range, no self-loops, weights >= 1, no duplicate arcs and symmetric arcs with
- *           equal weights (the last two exactly when every row is sorted, otherwise by
- *           order-independent 64-bit arc fingerprints); the first offending vertex is
- *           named in gp_last_error().
+ *           equal weights -- all exact for rows in any order (sorted rows: adjacent
+ *           duplicates + binary search for the reverse arc; otherwise per-row hash sets in
+ *           a temporary 16 B/arc device table); the first offending vertex is named in
+ *           gp_last_error().
  * The weight totals are always checked (GP_ERR_OVERFLOW).  Synchronous (reads back the
  * totals).  The inputs may be reused once the call returns. */
 gp_status gp_graph_create(gp_ctx ctx, gp_vid n, const gp_vid *adjp, const gp_vid *adjncy,
@@ -271,6 +278,11 @@ gp_status gp_ctx_set_timing(gp_ctx ctx, int32_t enable);
 /* Synchronous: drains pending events into the totals, then copies them out. */
 gp_status gp_ctx_kernel_stats(gp_ctx ctx, gp_kernel_kind kind, gp_kernel_stats *out);
 gp_status gp_ctx_reset_stats(gp_ctx ctx);
+/* Synchronous: the timed launches since the last reset, in launch order: kinds[i] (a
+ * gp_kernel_kind) and ms[i] (CUDA-event time); up to cap entries are copied, *count receives
+ * the total (nullable).  gp_coarsen_to enqueues level l's matching then its contraction, so a
+ * call's launches map to its levels in order (speculative levels after the stop come last). */
+gp_status gp_ctx_launch_times(gp_ctx ctx, int32_t cap, int32_t *kinds, float *ms, int32_t *count);
 /* Kernel launches made through this context since creation (all families). */
 gp_status gp_ctx_launch_count(gp_ctx ctx, int64_t *out);
 

@@ -21,6 +21,11 @@ NVCC_FLAGS = [
 ]
 
 
+def extra_defs():
+    """Optional -D flags for instrumented builds (GP_NVCC_DEFS="-DGP_CHECKPOINTS")."""
+    return os.environ.get("GP_NVCC_DEFS", "").split()
+
+
 def sources():
     return sorted(glob.glob(os.path.join(CSRC, "*.cu")))
 
@@ -45,7 +50,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     procs = []
     for src in sources():
         obj = os.path.join(LIBDIR, os.path.basename(src)[:-3] + ".o")
-        cmd = [NVCC, *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]
+        cmd = [NVCC, *NVCC_FLAGS, *extra_defs(), "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]
         if verbose:
             print(" ".join(cmd))
         procs.append((subprocess.Popen(cmd), src))

@@ -111,6 +111,7 @@ static void drain_events(Ctx *ctx) {
         if (cudaEventElapsedTime(&ms, t.a, t.b) == cudaSuccess) {
             ctx->stats[t.kind].ms += ms;
             ctx->stats[t.kind].launches += 1;
+            ctx->launch_log.push_back({t.kind, ms});
         }
         ctx->event_pool.push_back(t.a);
         ctx->event_pool.push_back(t.b);
@@ -126,6 +127,7 @@ void graph_release(Graph *g) {
     dev_free(ctx, g->adjwgt);
     dev_free(ctx, g->vwgt);
     if (g->owns_sizes) dev_free(ctx, g->sizes);
+    if (g->counted) --ctx->live_objects;
     g->tag = 0;
     delete g;
 }
@@ -143,12 +145,17 @@ void hier_release(Hier *h) {
         }
     }
     dev_free(h->ctx, h->levdev);
+    if (h->counted) --h->ctx->live_objects;
     h->tag = 0;
     delete h;
 }
 
 // graph arrays with 4 ints of padding (TMA bulk copies round ranges up to 16 bytes)
 gp_status alloc_graph_arrays(Ctx *ctx, Graph *g, int32_t n_bound, int32_t nnz_bound, bool own_sizes) {
+    if (!g->counted) {
+        g->counted = true;
+        ++ctx->live_objects;
+    }
     gp_status st = dev_alloc(ctx, (void **)&g->adjp, sizeof(int32_t) * ((size_t)n_bound + 4));
     if (st == GP_OK) st = dev_alloc(ctx, (void **)&g->vwgt, sizeof(int32_t) * ((size_t)n_bound + 4));
     if (st == GP_OK) st = dev_alloc(ctx, (void **)&g->adjncy, sizeof(int32_t) * ((size_t)nnz_bound + 4));
@@ -246,7 +253,7 @@ gp_status gp_ctx_create(int device, void *cuda_stream, gp_ctx *out) {
         set_error("gp_ctx_create: no CUDA device " + std::to_string(device));
         return GP_ERR_INVALID_ARG;
     }
-    GP_CUDA(cudaSetDevice(device));
+    DeviceGuard dg(device);  // the caller's current device is restored on return
     cudaDeviceProp prop;
     GP_CUDA(cudaGetDeviceProperties(&prop, device));
     if (prop.major < 10) {
@@ -295,7 +302,13 @@ gp_status gp_ctx_set_allocator(gp_ctx ctx, gp_alloc_fn alloc, gp_dealloc_fn deal
         set_error("gp_ctx_set_allocator: bad context or callbacks");
         return GP_ERR_INVALID_ARG;
     }
-    // existing buffers were allocated with the previous allocator: release them first
+    if (ctx->live_objects > 0) {
+        set_error("gp_ctx_set_allocator: " + std::to_string(ctx->live_objects) +
+                  " graph(s) / hierarchy(ies) still hold buffers of the current allocator; free them first");
+        return GP_ERR_INVALID_ARG;
+    }
+    DeviceGuard dg(ctx->device);
+    // the context's own scratch was allocated with the previous allocator: release it first
     cudaStreamSynchronize(ctx->stream);
     dev_free(ctx, ctx->scratch);
     dev_free(ctx, ctx->status);
@@ -315,8 +328,13 @@ gp_status gp_ctx_num_sms(gp_ctx ctx, int32_t *out) {
     return GP_OK;
 }
 
-gp_status gp_graph_create(gp_ctx ctx, gp_vid n, const gp_vid *adjp, const gp_vid *adjncy, const gp_wgt *adjwgt,
-                          const gp_wgt *vwgt, uint32_t flags, gp_graph *out) {
+}  // extern "C"
+
+// gp_graph_create with the totals check optional (check_totals = false: the sharded create,
+// which checks the global totals after an all-gather on every rank)
+static gp_status graph_create_impl(gp_ctx ctx, gp_vid n, const gp_vid *adjp, const gp_vid *adjncy,
+                                   const gp_wgt *adjwgt, const gp_wgt *vwgt, uint32_t flags, bool check_totals,
+                                   gp_graph *out) {
     if (out) *out = nullptr;
     if (!tagged<Ctx>(ctx, kTagCtx) || !out || n < 0 || !adjp) {
         set_error("gp_graph_create: bad context, output, n or adjp");
@@ -325,7 +343,7 @@ gp_status gp_graph_create(gp_ctx ctx, gp_vid n, const gp_vid *adjp, const gp_vid
     GP_TRY_BEGIN
     const bool dev = flags & GP_INPUT_DEVICE;
     const cudaMemcpyKind kind = dev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
-    GP_CUDA(cudaSetDevice(ctx->device));
+    DeviceGuard dg(ctx->device);
     int32_t nnz = 0;
     if (dev) {
         GP_CUDA(cudaMemcpyAsync(ctx->pinned, adjp + n, sizeof(int32_t), cudaMemcpyDeviceToHost, ctx->stream));
@@ -365,7 +383,8 @@ gp_status gp_graph_create(gp_ctx ctx, gp_vid n, const gp_vid *adjp, const gp_vid
         e = cudaMemcpyAsync(g->sizes, ctx->pinned + 16, sizeof(SizeRec), cudaMemcpyHostToDevice, ctx->stream);
     }
     if (st == GP_OK && e != cudaSuccess) st = cuda_fail(e, "gp_graph_create: copy");
-    if (st == GP_OK) st = graph_totals_and_validate(ctx, g, flags & GP_VALIDATE);  // synchronises
+    if (st == GP_OK)  // synchronises
+        st = graph_totals_and_validate(ctx, g, flags & GP_VALIDATE, check_totals);
     if (st != GP_OK) {
         std::string keep = g_last_error;
         cudaStreamSynchronize(ctx->stream);
@@ -376,6 +395,13 @@ gp_status gp_graph_create(gp_ctx ctx, gp_vid n, const gp_vid *adjp, const gp_vid
     *out = g;
     return GP_OK;
     GP_TRY_END
+}
+
+extern "C" {
+
+gp_status gp_graph_create(gp_ctx ctx, gp_vid n, const gp_vid *adjp, const gp_vid *adjncy, const gp_wgt *adjwgt,
+                          const gp_wgt *vwgt, uint32_t flags, gp_graph *out) {
+    return graph_create_impl(ctx, n, adjp, adjncy, adjwgt, vwgt, flags & (GP_INPUT_DEVICE | GP_VALIDATE), true, out);
 }
 
 gp_status gp_graph_view(gp_graph g, gp_vid *n, gp_vid *nnz, const gp_vid **d_adjp, const gp_vid **d_adjncy,
@@ -399,6 +425,7 @@ gp_status gp_graph_download(gp_graph g, gp_vid *h_adjp, gp_vid *h_adjncy, gp_wgt
         return GP_ERR_INVALID_ARG;
     }
     Ctx *ctx = g->ctx;
+    DeviceGuard dg(ctx->device);
     cudaStream_t s = ctx->stream;
     if (h_adjp) GP_CUDA(cudaMemcpyAsync(h_adjp, g->adjp, sizeof(int32_t) * ((size_t)g->n + 1), cudaMemcpyDeviceToHost, s));
     if (h_adjncy && g->nnz)
@@ -432,6 +459,7 @@ gp_status gp_match_level_ex(gp_graph g, gp_vid *d_match, int32_t max_rounds, uin
     }
     GP_TRY_BEGIN
     Ctx *ctx = g->ctx;
+    DeviceGuard dg(ctx->device);
     ctx->tie_seed = tie_seed;
     if (ctx->comm) {
         set_error("gp_match_level: per-level calls are single-GPU; sharded graphs use gp_coarsen_to");
@@ -475,6 +503,7 @@ gp_status gp_contract_level(gp_graph g, const gp_vid *d_match, gp_vid *d_cmap, g
     }
     GP_TRY_BEGIN
     Ctx *ctx = g->ctx;
+    DeviceGuard dg(ctx->device);
     if (ctx->comm) {
         set_error("gp_contract_level: per-level calls are single-GPU; sharded graphs use gp_coarsen_to");
         return GP_ERR_INVALID_ARG;
@@ -556,6 +585,7 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
     }
     GP_TRY_BEGIN
     Ctx *ctx = g->ctx;
+    DeviceGuard dg(ctx->device);
     ctx->tie_seed = opts->tie_seed;
     if (ctx->comm) return dist_coarsen_to(g, opts, out);  // sharded path (dist.cu)
     const int32_t pct = opts->stall_ratio_pct ? opts->stall_ratio_pct : 95;
@@ -563,6 +593,8 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
     if (max_levels > ctx->max_reports) max_levels = ctx->max_reports;
     Hier *h = new Hier();
     h->ctx = ctx;
+    h->counted = true;
+    ++ctx->live_objects;
     if (g->n <= opts->threshold) {
         *out = h;
         return GP_OK;
@@ -686,6 +718,15 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
                             d[4], (d[0] >> 32) * 1e-3, d[0] & 0xffffffffull, d[3] * 1e-3 / d[4], d[1] >> 32,
                             d[1] & 0xffffffffull, d[2] >> 32, d[5]);
                 }
+                if (hd[l].match.ck[1][8]) {
+                    fprintf(stderr, "[gp]   warp-0 checkpoints per round (cycles: claim u p+S qq/rr decide rescan push | loop-exit flush):");
+                    for (int k = 1; k < 16 && hd[l].match.ck[k][8]; ++k) {
+                        fprintf(stderr, " [");
+                        for (int j = 0; j < 9; ++j) fprintf(stderr, "%s%lld", j ? " " : "", hd[l].match.ck[k][j]);
+                        fprintf(stderr, "]");
+                    }
+                    fprintf(stderr, "\n");
+                }
                 if (hd[l].match.lens[1]) {
                     fprintf(stderr, "[gp]   per round (live | slowest warp us | rows rescanned thread / warp):");
                     for (int k = 1; k < 16 && hd[l].match.lens[k]; ++k)
@@ -786,6 +827,7 @@ gp_status gp_hier_download_level(gp_hier h, int32_t i, gp_vid *h_match, gp_vid *
         return GP_ERR_INVALID_ARG;
     }
     const Level &l = h->levels[i];
+    DeviceGuard dg(h->ctx->device);
     cudaStream_t s = h->ctx->stream;
     if (!l.pieces.empty()) {  // sharded: the pieces' owned slices, in rank order
         size_t o = 0;
@@ -819,6 +861,7 @@ gp_status gp_hier_download_coarse(gp_hier h, int32_t i, gp_vid *h_adjp, gp_vid *
     if (l.pieces.empty()) parts.push_back(l.coarse);
     else
         for (const DistPiece &p : l.pieces) parts.push_back(p.coarse);
+    DeviceGuard dg(h->ctx->device);
     cudaStream_t s = h->ctx->stream;
     int32_t rows = 0, arcs = 0;
     for (const Graph *c : parts) {
@@ -855,6 +898,7 @@ gp_status gp_project(gp_hier h, int32_t from_level, int32_t to_level, const gp_v
         return GP_ERR_INVALID_ARG;
     }
     GP_TRY_BEGIN
+    DeviceGuard dg(h->ctx->device);
     std::vector<const int32_t *> cms;
     for (int32_t l = to_level; l <= from_level; ++l) {
         if (!h->levels[l].pieces.empty()) {
@@ -890,6 +934,7 @@ gp_status gp_ctx_create_dist(int device, void *cuda_stream, const void *nccl_uni
     }
     gp_status st = gp_ctx_create(device, cuda_stream, out);
     if (st != GP_OK) return st;
+    DeviceGuard dg(device);
     st = attach_comm(*out, dist_comm_create_nccl(*out, nccl_unique_id, rank, nranks));
     if (st != GP_OK) *out = nullptr;
     return st;
@@ -903,6 +948,7 @@ gp_status gp_ctx_create_loopback(int device, void *cuda_stream, int nranks, gp_c
     }
     gp_status st = gp_ctx_create(device, cuda_stream, out);
     if (st != GP_OK) return st;
+    DeviceGuard dg(device);
     st = attach_comm(*out, dist_comm_create_loopback(*out, nranks));
     if (st != GP_OK) *out = nullptr;
     return st;
@@ -929,19 +975,37 @@ gp_status gp_graph_create_dist(gp_ctx ctx, gp_vid n_global, gp_vid v_begin, gp_v
         return GP_ERR_INVALID_ARG;
     }
     GP_TRY_BEGIN
+    // Every rank reaches the all-gather even when its local create failed, so that a failure
+    // (or an overflow of the GLOBAL weight totals, R14) is reported on all ranks together
+    // instead of leaving the others waiting in a collective.
     gp_graph g = nullptr;
-    gp_status st = gp_graph_create(ctx, v_end - v_begin, adjp_local, adjncy, adjwgt, vwgt, flags, &g);
-    if (st != GP_OK) return st;
+    gp_status st = graph_create_impl(ctx, v_end - v_begin, adjp_local, adjncy, adjwgt, vwgt, flags, false, &g);
     const int G = dist_nranks(ctx), me = dist_rank(ctx);
-    int32_t mine[3] = {v_begin, v_end, g->nnz};
-    std::vector<int32_t> all(3 * (size_t)G);
-    st = dist_allgather_i32(ctx, mine, 3, all.data());
+    const unsigned long long sa = g ? g->sum_adjwgt : 0ull, sv = g ? g->sum_vwgt : 0ull;
+    int32_t mine[8] = {v_begin, v_end, g ? g->nnz : 0, (int32_t)st, (int32_t)(uint32_t)sa, (int32_t)(uint32_t)(sa >> 32),
+                       (int32_t)(uint32_t)sv, (int32_t)(uint32_t)(sv >> 32)};
+    std::vector<int32_t> all(8 * (size_t)G);
+    const std::string local_err = st != GP_OK ? g_last_error : std::string();
+    gp_status gst = dist_allgather_i32(ctx, mine, 8, all.data());
+    if (gst != GP_OK) {
+        if (g) gp_free(g);
+        return gst;
+    }
     long long nnz = 0;
+    unsigned long long tot_a = 0, tot_v = 0;
     std::vector<int32_t> ranges(G + 1);
-    for (int r = 0; st == GP_OK && r < G; ++r) {
-        ranges[r] = all[3 * r];
-        nnz += all[3 * r + 2];
-        if (all[3 * r] != (r == 0 ? 0 : all[3 * (r - 1) + 1]) || (r == G - 1 && all[3 * r + 1] != n_global)) {
+    for (int r = 0; r < G; ++r) {
+        const int32_t *a = &all[8 * (size_t)r];
+        if (st == GP_OK && a[3] != GP_OK) {
+            set_error("gp_graph_create_dist: rank " + std::to_string(r) + " failed to create its shard (" +
+                      gp_status_string((gp_status)a[3]) + ")");
+            st = (gp_status)a[3];
+        }
+        ranges[r] = a[0];
+        nnz += a[2];
+        tot_a += (unsigned long long)(uint32_t)a[4] | ((unsigned long long)(uint32_t)a[5] << 32);
+        tot_v += (unsigned long long)(uint32_t)a[6] | ((unsigned long long)(uint32_t)a[7] << 32);
+        if (st == GP_OK && (a[0] != (r == 0 ? 0 : all[8 * ((size_t)r - 1) + 1]) || (r == G - 1 && a[1] != n_global))) {
             set_error("gp_graph_create_dist: the shards do not tile [0, n_global) in rank order");
             st = GP_ERR_INVALID_ARG;
         }
@@ -950,9 +1014,14 @@ gp_status gp_graph_create_dist(gp_ctx ctx, gp_vid n_global, gp_vid v_begin, gp_v
         set_error("gp_graph_create_dist: total arcs exceed INT32_MAX");
         st = GP_ERR_OVERFLOW;
     }
+    if (st == GP_OK && (tot_a > (unsigned long long)INT32_MAX || tot_v > (unsigned long long)INT32_MAX)) {
+        set_error("gp_graph_create_dist: global weight totals exceed INT32_MAX: sum(adjwgt)=" + std::to_string(tot_a) +
+                  " sum(vwgt)=" + std::to_string(tot_v));
+        st = GP_ERR_OVERFLOW;
+    }
     if (st != GP_OK) {
-        std::string keep = g_last_error;
-        gp_free(g);
+        std::string keep = local_err.empty() ? g_last_error : local_err;
+        if (g) gp_free(g);
         g_last_error = keep;
         return st;
     }
@@ -973,11 +1042,15 @@ void gp_free(void *handle) {
     const uint32_t tag = *static_cast<const uint32_t *>(handle);
     if (tag == kTagGraph) {
         Graph *g = static_cast<Graph *>(handle);
+        DeviceGuard dg(g->ctx->device);
         if (!g->borrowed) graph_release(g);
     } else if (tag == kTagHier) {
-        hier_release(static_cast<Hier *>(handle));
+        Hier *h = static_cast<Hier *>(handle);
+        DeviceGuard dg(h->ctx->device);
+        hier_release(h);
     } else if (tag == kTagCtx) {
         Ctx *ctx = static_cast<Ctx *>(handle);
+        DeviceGuard dg(ctx->device);
         cudaStreamSynchronize(ctx->stream);
         dist_comm_destroy(ctx);
         drain_events(ctx);
@@ -994,6 +1067,7 @@ void gp_free(void *handle) {
 
 gp_status gp_ctx_set_timing(gp_ctx ctx, int32_t enable) {
     if (!tagged<Ctx>(ctx, kTagCtx)) return GP_ERR_INVALID_ARG;
+    DeviceGuard dg(ctx->device);
     drain_events(ctx);
     ctx->timing = enable != 0;
     return GP_OK;
@@ -1001,6 +1075,7 @@ gp_status gp_ctx_set_timing(gp_ctx ctx, int32_t enable) {
 
 gp_status gp_ctx_kernel_stats(gp_ctx ctx, gp_kernel_kind kind, gp_kernel_stats *out) {
     if (!tagged<Ctx>(ctx, kTagCtx) || !out || kind < 0 || kind >= GP_K_COUNT) return GP_ERR_INVALID_ARG;
+    DeviceGuard dg(ctx->device);
     drain_events(ctx);
     *out = ctx->stats[kind];
     return GP_OK;
@@ -1008,8 +1083,23 @@ gp_status gp_ctx_kernel_stats(gp_ctx ctx, gp_kernel_kind kind, gp_kernel_stats *
 
 gp_status gp_ctx_reset_stats(gp_ctx ctx) {
     if (!tagged<Ctx>(ctx, kTagCtx)) return GP_ERR_INVALID_ARG;
+    DeviceGuard dg(ctx->device);
     drain_events(ctx);
     for (auto &s : ctx->stats) s = gp_kernel_stats{0, 0.0};
+    ctx->launch_log.clear();
+    return GP_OK;
+}
+
+gp_status gp_ctx_launch_times(gp_ctx ctx, int32_t cap, int32_t *kinds, float *ms, int32_t *count) {
+    if (!tagged<Ctx>(ctx, kTagCtx) || cap < 0 || (cap > 0 && (!kinds || !ms))) return GP_ERR_INVALID_ARG;
+    DeviceGuard dg(ctx->device);
+    drain_events(ctx);
+    const int32_t n = (int32_t)ctx->launch_log.size();
+    for (int32_t i = 0; i < n && i < cap; ++i) {
+        kinds[i] = ctx->launch_log[(size_t)i].first;
+        ms[i] = ctx->launch_log[(size_t)i].second;
+    }
+    if (count) *count = n;
     return GP_OK;
 }
 

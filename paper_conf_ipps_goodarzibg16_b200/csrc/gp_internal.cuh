@@ -6,6 +6,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <utility>
 #include <vector>
 
 #include "../../include/gp.h"
@@ -20,6 +21,10 @@ constexpr uint32_t kTagGraph = 0x47504752u;  // "GPGR"
 constexpr uint32_t kTagHier = 0x47504849u;   // "GPHI"
 
 constexpr int kBlock = 256;  // threads per CTA of the streaming kernels
+
+// gp_graph_create flag used inside the library only (not in gp.h): measure the weight totals
+// but do not fail on them (gp_graph_create_dist checks the GLOBAL totals on every rank)
+constexpr uint32_t kInternalNoTotalsCheck = 0x80000000u;
 
 // ---------------------------------------------------------------------------------------
 // device-side control blocks of one level (zeroed once per gp_coarsen_to call)
@@ -54,6 +59,9 @@ struct MatchCtl {
     // GP_PROF=1: per round k < 16, how the live vertices ended: kept their target / took the
     // cached second choice / matched (rescans: trows)
     int32_t nkeep[16], nsec[16], nmatch[16];
+    // GP_PROF=2: clock64 checkpoints of warp 0 of block 0 through its first phase-k group of
+    // round k < 16 (cycles since the phase started)
+    long long ck[16][12];
 };
 
 constexpr int kMaxContractCtas = 1024;  // grid cap of the contraction kernel
@@ -144,6 +152,9 @@ struct gp_graph_s {
     int rank = 0;
     int32_t vbase = 0, n_global = 0, nnz_global = 0;
     std::vector<int32_t> ranges;
+    // weight totals measured at creation (R14; the sharded create checks the global sums)
+    unsigned long long sum_adjwgt = 0, sum_vwgt = 0;
+    bool counted = false;  // included in ctx->live_objects
 };
 
 namespace gp {
@@ -161,6 +172,7 @@ struct gp_hier_s {
     gp::Ctx *ctx = nullptr;
     std::vector<gp::Level> levels;
     gp::LevelDev *levdev = nullptr;  // per-level control blocks (coarse graphs' size records)
+    bool counted = false;  // included in ctx->live_objects
 };
 
 struct gp_ctx_s {
@@ -190,11 +202,16 @@ struct gp_ctx_s {
     // sharded path: NCCL (one local rank) or loopback (all ranks simulated); null = 1 GPU
     gp::DistComm *comm = nullptr;
 
+    // graphs and hierarchies alive on this context (their buffers came from its allocator:
+    // gp_ctx_set_allocator refuses to switch allocators while any exist)
+    int64_t live_objects = 0;
+
     // instrumentation
     bool timing = false;
     std::vector<gp::TimedLaunch> pending;
     std::vector<cudaEvent_t> event_pool;
     gp_kernel_stats stats[GP_K_COUNT] = {};
+    std::vector<std::pair<int, float>> launch_log;  // (kind, ms) of every timed launch since the last reset
     int64_t launches = 0;
 };
 
@@ -258,7 +275,26 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
                            SizeRec *out_sizes, LevelReport *report, const ContractParams &prm);
 size_t contract_tiles(int32_t n, int32_t nnz);
 
-gp_status graph_totals_and_validate(Ctx *ctx, const Graph *g, bool validate);
+// weight totals (stored in g->sum_*) and, with `validate`, the GP_VALIDATE contract;
+// check_totals = false skips the INT32_MAX test (the sharded create checks global sums)
+gp_status graph_totals_and_validate(Ctx *ctx, Graph *g, bool validate, bool check_totals = true);
+
+// The calling thread's current device is switched to `dev` for the scope of an ABI call and
+// restored afterwards (each entry point runs on its context's device; the caller's current
+// device is left as it was).
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        int cur = -1;
+        if (cudaGetDevice(&cur) == cudaSuccess && cur != dev && cudaSetDevice(dev) == cudaSuccess) prev = cur;
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+    DeviceGuard(const DeviceGuard &) = delete;
+    DeviceGuard &operator=(const DeviceGuard &) = delete;
+};
+constexpr int kMaxDevices = 64;  // per-device caches of kernel attributes / occupancy
 
 // projection of un-coarsening (project.cu): cms = CM of levels to..from (fine to coarse)
 gp_status enqueue_project(Ctx *ctx, const int32_t *const *cms, int nlev, int32_t n, const int32_t *part_c,

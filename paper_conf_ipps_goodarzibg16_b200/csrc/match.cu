@@ -682,30 +682,34 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
 
 // Warp-cooperative rescan of every row of a phase-k group that needs one (lazy rescan,
 // DESIGN.md §4.2): the rows' arcs are flattened into one item space (warp scan of the
-// degrees) and each lane takes kFB items at a time, so the dependent loads of ALL rows
+// degrees) and each lane takes kFB items per batch, so the dependent loads of ALL rows
 // (arc -> P_k[x] -> P_k[P_k[x]]) are in flight together instead of one row after another.
-// Top-2 per row by shared-memory 64-bit atomicMax (keys are distinct: one per neighbour).
-// Rows longer than kHubDeg go to the hub list.  All 32 lanes call; fq lives in the phase-0
-// staging buffers (idle in phase k).
+// Top-2 per row of a batch with native 32-bit shared atomics, field by field (heaviest weight,
+// then the best tie word at that weight; the same among the row's other keys; a 64-bit shared
+// atomicMax would be a CAS loop).  Rows longer than one batch keep a running top-2 that the
+// row's owner lane merges after every batch: every item is loaded ONCE (an earlier two-pass
+// version re-ran the three dependent loads per batch for the second choice, which made the
+// slowest warp of a round ~15 us on coarse levels).  Rows longer than kHubDeg go to the hub
+// list.  All 32 lanes call; fq lives in the phase-0 staging buffers (idle in phase k).
 constexpr int kFQ = 128;  // queue entries per warp (32 lanes x kVL <= 4)
-constexpr int kFB = 4;    // flat items per lane per batch
+constexpr int kFB = 8;    // flat items per lane per batch (256 per warp batch)
 struct FlatQ {
-    union {
-        struct {
-            unsigned long long k1[kFQ], k2[kFQ];  // top-2 keys (multi-batch: 64-bit CAS atomics)
-        };
-        struct {
-            uint32_t w1[kFQ], n1[kFQ], w2[kFQ], n2[kFQ];  // single batch: native 32-bit max on (w, ~v)
-        };
-    };
-    int32_t s[kFQ];
-    int32_t off[kFQ + 2];
-    uint8_t own[32 * kFB];  // single batch: queue entry of every item (no search)
+    unsigned long long a1[kFQ], a2[kFQ];          // running top-2 of rows spanning batches
+    uint32_t w1[kFQ], n1[kFQ], w2[kFQ], n2[kFQ];  // the batch's top-2 per row: (weight, tie word)
+    int32_t s[kFQ];                               // row start (arc index)
+    int32_t off[kFQ + 2];                         // row offset in the flat item space
+    uint8_t own[32 * kFB];                        // queue entry of every item of the batch
 };
-static_assert(sizeof(FlatQ) * (kNT / 32) <= sizeof(int32_t) * ((kStages - 1) * kStageArcs + kStages * kStageArcs),
+// the queues live in adj[1..2], wgt[0..2] and ap[0..2] (contiguous in MatchSmem)
+static_assert(sizeof(FlatQ) * (kNT / 32) <=
+                  sizeof(int32_t) * ((kStages - 1) * kStageArcs + kStages * kStageArcs + kStages * (kMaxVch + 8)),
               "flat rescan queues must fit the idle phase-0 buffers");
 
-template <int kVL, bool H>
+__device__ __forceinline__ unsigned long long wn_key(uint32_t w, uint32_t n) {
+    return w ? (((unsigned long long)w << 32) | n) : 0ull;
+}
+
+template <int kVL, bool H, int KFB = (kVL == 1 ? kFB : 4)>
 __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, const int32_t *Pk, int32_t *Pn,
                                             int32_t *Pkw, RoundSlot *next, const int32_t (&u)[kVL],
                                             bool (&need)[kVL], bool (&live)[kVL], unsigned long long &scanned,
@@ -740,100 +744,91 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
         T += tot;
     }
     if (qn == 0) return;  // warp-uniform
-    const bool one = T <= 32 * kFB;  // every item in registers at once: top-1 and top-2 in one pass
-    for (int r = lane; r < qn; r += 32) {  // the union's active view
-        if (one) {
-            fq.w1[r] = fq.n1[r] = fq.w2[r] = fq.n2[r] = 0u;
-        } else {
-            fq.k1[r] = 0ull;
-            fq.k2[r] = 0ull;
-        }
+    const bool multi = T > 32 * KFB;  // some row spans batches: running top-2 per row
+    for (int r = lane; r < qn; r += 32) {
+        fq.w1[r] = fq.n1[r] = fq.w2[r] = fq.n2[r] = 0u;
+        if (multi) fq.a1[r] = fq.a2[r] = 0ull;
     }
-    if (one) {  // every queued row marks its items with its entry
+    for (int32_t b0 = 0; b0 < T; b0 += 32 * KFB) {
+        const int32_t bn = min(T - b0, 32 * KFB);
+        // every queued row marks its items inside this batch with its entry
 #pragma unroll
         for (int i = 0; i < kVL; ++i)
             if (i >= i0 && i < i1 && need[i]) {
                 const int32_t o = fq.off[rpos[i]];
-                for (int32_t q = 0; q < re[i] - rs[i]; ++q) fq.own[o + q] = (uint8_t)rpos[i];
+                const int32_t lo = max(o, b0), hi = min(o + (re[i] - rs[i]), b0 + bn);
+                for (int32_t q = lo; q < hi; ++q) fq.own[q - b0] = (uint8_t)rpos[i];
             }
-    }
-    __syncwarp();
-    for (int pass = 0; pass < (one ? 1 : 2); ++pass) {
-        for (int32_t b0 = 0; b0 < T; b0 += 32 * kFB) {
-            int32_t e[kFB], x[kFB], w[kFB], px[kFB];
-            unsigned long long key[kFB];
+        __syncwarp();
+        // three dependent load levels for KFB items per lane: arc, P_k[x], P_k[P_k[x]]
+        int32_t x[KFB], w[KFB], px[KFB];
 #pragma unroll
-            for (int b = 0; b < kFB; ++b) {
-                const int32_t f = b0 + b * 32 + lane;
-                e[b] = -1;
-                x[b] = -1;
-                w[b] = 0;
-                if (f < T) {  // entry of item f: the last row with off <= f
-                    int32_t r = 0;
-                    if (one) {
-                        r = fq.own[f];
-                    } else {
-#pragma unroll
-                        for (int step = kFQ / 2; step > 0; step >>= 1)
-                            if (r + step < qn && fq.off[r + step] <= f) r += step;
-                    }
-                    e[b] = r;
-                    const int32_t j = fq.s[r] + (f - fq.off[r]);
-                    x[b] = __ldg(a.adjncy + j);
-                    w[b] = __ldg(a.adjwgt + j);
-                }
-            }
-#pragma unroll
-            for (int b = 0; b < kFB; ++b) px[b] = x[b] >= 0 ? ldcg(Pk + x[b]) : -1;
-#pragma unroll
-            for (int b = 0; b < kFB; ++b) {
-                const int32_t pp = px[b] >= 0 ? ldcg(Pk + px[b]) : -1;
-                key[b] = (x[b] >= 0 && pp != x[b]) ? pack_key<H>(a.tie_seed, w[b], x[b]) : 0ull;  // x free after round k
-            }
-            if (one) {
-                // top-2 of (w, ~x) per row with native 32-bit shared atomics, field by field
-                // (a 64-bit shared atomicMax is a CAS loop): heaviest weight, then the best tie
-                // priority (low key word) at that weight; the same among the row's other keys
-                const uint32_t NOK = 0u;
-#pragma unroll
-                for (int b = 0; b < kFB; ++b)
-                    if (key[b]) atomicMax(&fq.w1[e[b]], (uint32_t)w[b]);
-                __syncwarp();
-#pragma unroll
-                for (int b = 0; b < kFB; ++b)
-                    if (key[b] && (uint32_t)w[b] == fq.w1[e[b]]) atomicMax(&fq.n1[e[b]], (uint32_t)key[b]);
-                __syncwarp();
-#pragma unroll
-                for (int b = 0; b < kFB; ++b) {
-                    const bool top = key[b] && (uint32_t)w[b] == fq.w1[e[b]] && (uint32_t)key[b] == fq.n1[e[b]];
-                    if (key[b] && !top) atomicMax(&fq.w2[e[b]], (uint32_t)w[b]);
-                    else key[b] = NOK;  // not a second-choice candidate
-                }
-                __syncwarp();
-#pragma unroll
-                for (int b = 0; b < kFB; ++b)
-                    if (key[b] && (uint32_t)w[b] == fq.w2[e[b]]) atomicMax(&fq.n2[e[b]], (uint32_t)key[b]);
-            } else if (pass == 0) {
-#pragma unroll
-                for (int b = 0; b < kFB; ++b)
-                    if (key[b]) atomicMax(&fq.k1[e[b]], key[b]);
-            } else {
-#pragma unroll
-                for (int b = 0; b < kFB; ++b)
-                    if (key[b] && key[b] != fq.k1[e[b]]) atomicMax(&fq.k2[e[b]], key[b]);
+        for (int b = 0; b < KFB; ++b) {
+            const int32_t f = b * 32 + lane;
+            x[b] = -1;
+            w[b] = 0;
+            if (f < bn) {
+                const int32_t r = fq.own[f];
+                const int32_t j = fq.s[r] + (b0 + f - fq.off[r]);
+                x[b] = __ldg(a.adjncy + j);
+                w[b] = __ldg(a.adjwgt + j);
             }
         }
+#pragma unroll
+        for (int b = 0; b < KFB; ++b) px[b] = x[b] >= 0 ? ldcg(Pk + x[b]) : -1;
+        uint32_t t[KFB];  // tie word of a candidate (x free after round k), w = 0 otherwise
+#pragma unroll
+        for (int b = 0; b < KFB; ++b) {
+            const int32_t pp = px[b] >= 0 ? ldcg(Pk + px[b]) : -1;
+            const bool cand = x[b] >= 0 && pp != x[b];
+            t[b] = cand ? (uint32_t)pack_key<H>(a.tie_seed, w[b], x[b]) : 0u;
+            if (!cand) w[b] = 0;
+        }
+#pragma unroll
+        for (int b = 0; b < KFB; ++b)
+            if (w[b]) atomicMax(&fq.w1[fq.own[b * 32 + lane]], (uint32_t)w[b]);
         __syncwarp();
+#pragma unroll
+        for (int b = 0; b < KFB; ++b) {
+            const int r = w[b] ? fq.own[b * 32 + lane] : 0;
+            if (w[b] && (uint32_t)w[b] == fq.w1[r]) atomicMax(&fq.n1[r], t[b]);
+        }
+        __syncwarp();
+#pragma unroll
+        for (int b = 0; b < KFB; ++b) {
+            const int r = w[b] ? fq.own[b * 32 + lane] : 0;
+            if (w[b] && (uint32_t)w[b] == fq.w1[r] && t[b] == fq.n1[r]) w[b] = 0;  // the batch's top: not a second
+            else if (w[b]) atomicMax(&fq.w2[r], (uint32_t)w[b]);
+        }
+        __syncwarp();
+#pragma unroll
+        for (int b = 0; b < KFB; ++b) {
+            const int r = w[b] ? fq.own[b * 32 + lane] : 0;
+            if (w[b] && (uint32_t)w[b] == fq.w2[r]) atomicMax(&fq.n2[r], t[b]);
+        }
+        __syncwarp();
+        if (multi) {  // the rows of this batch: owner lanes merge its top-2 into the running one
+            const int r0 = fq.own[0], r1 = fq.own[bn - 1];
+            for (int r = r0 + lane; r <= r1; r += 32) {
+                const unsigned long long t1 = wn_key(fq.w1[r], fq.n1[r]), t2 = wn_key(fq.w2[r], fq.n2[r]);
+                const unsigned long long A1 = fq.a1[r], A2 = fq.a2[r];
+                const unsigned long long lo = A1 < t1 ? A1 : t1, m2 = A2 > t2 ? A2 : t2;
+                fq.a1[r] = A1 > t1 ? A1 : t1;
+                fq.a2[r] = lo > m2 ? lo : m2;
+                fq.w1[r] = fq.n1[r] = fq.w2[r] = fq.n2[r] = 0u;
+            }
+            __syncwarp();
+        }
     }
 #pragma unroll
     for (int i = 0; i < kVL; ++i) {
         if (i >= i0 && i < i1 && need[i]) {
             const int32_t r = rpos[i];
-            const unsigned long long k1 = one ? (((unsigned long long)fq.w1[r] << 32) | fq.n1[r]) : fq.k1[r];
-            const unsigned long long k2 = one ? (((unsigned long long)fq.w2[r] << 32) | fq.n2[r]) : fq.k2[r];
-            const int32_t bv = key_vertex<H>(a.tie_seed, fq.w1[r] || !one ? k1 : 0ull);
+            const unsigned long long k1 = multi ? fq.a1[r] : wn_key(fq.w1[r], fq.n1[r]);
+            const unsigned long long k2 = multi ? fq.a2[r] : wn_key(fq.w2[r], fq.n2[r]);
+            const int32_t bv = key_vertex<H>(a.tie_seed, k1);
             Pn[u[i]] = bv;
-            a.S[u[i]] = key_vertex<H>(a.tie_seed, !one || fq.w2[r] ? k2 : 0ull);
+            a.S[u[i]] = key_vertex<H>(a.tie_seed, k2);
             if (bv == kNone) Pkw[u[i]] = kNone;  // dead: NONE in both buffers
             live[i] = bv != kNone;
         }
@@ -848,10 +843,36 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
 // vertices keep their partner in P, dead ones NONE), read at the same level as P_k[u].  No list
 // load, no list append and no atomic with a return value on the round's critical path; the
 // next round's live count is a fire-and-forget reduction.
+// GP_PROF=2: cycle checkpoints of warp 0 of block 0 (first group of round k < 16)
+// (compiled in only with -DGP_CHECKPOINTS: GP_NVCC_DEFS=-DGP_CHECKPOINTS for _build)
+#ifdef GP_CHECKPOINTS
+#define GP_CK(j)                                                                                   \
+    do {                                                                                           \
+        if (ck_on && threadIdx.x == 0) a.ctl->ck[k][j] = clock64() - ck0;                          \
+    } while (0)
+#define GP_CK_ON(expr) ck_on = (expr)
+#define GP_CK_SINK(expr)                                                                           \
+    do {                                                                                           \
+        if (ck_on) {                                                                               \
+            int32_t z_ = 0;                                                                        \
+            for (int i_ = 0; i_ < kVL; ++i_) z_ += expr;                                          \
+            if (z_ == -7777777) a.ctl->ck[15][11] = z_;                                            \
+        }                                                                                          \
+    } while (0)
+#else
+#define GP_CK(j) do { } while (0)
+#define GP_CK_ON(expr) do { } while (0)
+#define GP_CK_SINK(expr) do { } while (0)
+#endif
+
 template <bool H, int kVL, bool kStatic = false>
 __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t len, bool park, const int32_t *Lover,
                              unsigned long long &scanned, unsigned long long &rows, unsigned long long &visits,
-                             int32_t &made) {
+                             int32_t &made, int vpg = 32) {
+    // vpg (kVL = 1 only): live vertices per warp group.  Short live lists take 4..16 vertices
+    // per warp so that more warps share the round, and the flat rescan still spreads a
+    // group's arcs over all 32 lanes (the old per-vertex G-lane groups walked a long row
+    // 4G arcs per dependent step).
     const int32_t *Pk = a.P[k & 1];
     int32_t *Pn = a.P[(k + 1) & 1];
     int32_t *Pkw = a.P[k & 1];
@@ -865,7 +886,12 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
     // them from a shared-memory counter.  No global atomics on a shared address: thousands
     // of warps hitting one L2 atomic unit serialise (~0.5 ns each), which dominated the
     // rounds of small levels.
-    const long long ngroups = ((long long)len + 32 * kVL - 1) / (32 * kVL);
+    const int gsz = kVL == 1 ? vpg : 32 * kVL;  // live entries per group
+#ifdef GP_CHECKPOINTS
+    bool ck_on = a.prof == 2 && blockIdx.x == 0 && threadIdx.x < 32 && k < 16;
+    const long long ck0 = clock64();
+#endif
+    const long long ngroups = ((long long)len + gsz - 1) / gsz;
     const long long g_lo = ngroups * blockIdx.x / g_nact, g_hi = ngroups * (blockIdx.x + 1) / g_nact;
     if (threadIdx.x == 0) sm.claim = 0;
     __syncthreads();
@@ -878,14 +904,17 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
         return a.interleave ? (long long)blockIdx.x + (long long)c * g_nact : g_lo + c;
     };
     for (long long g = claim_next(); g < (a.interleave ? ngroups : g_hi); g = claim_next()) {
-        const long long base = g * 32 * kVL;
+        GP_CK(0);
+        const long long base = g * gsz;
         int32_t u[kVL], p[kVL], s2[kVL], qq[kVL], rr[kVL], ps[kVL], pps[kVL];
         // level 1: the vertices; level 2: P_k[u] and the cached second candidate S[u]
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
             const long long idx = base + i * 32 + lane;
-            u[i] = idx < len ? ((kStatic || (k == 1 && !Lover)) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
+            u[i] = (idx < len && (kVL > 1 || lane < gsz)) ? ((kStatic || (k == 1 && !Lover)) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
         }
+        GP_CK_SINK(u[i_]);
+        GP_CK(1);
         int32_t rs[kVL], re[kVL];  // row bounds, loaded speculatively with P_k[u]: a rescan
                                    // then starts one dependent level earlier
 #pragma unroll
@@ -899,6 +928,7 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
 #pragma unroll
         for (int i = 0; i < kVL; ++i)
             if (p[i] == kNone) s2[i] = kNone;
+        GP_CK(2);
         // level 3: P_k[p] and P_k[s2] (freedom test of the cached candidate, P only)
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
@@ -911,6 +941,8 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
             rr[i] = (p[i] != kNone && qq[i] != u[i] && qq[i] >= 0) ? ldcg(Pk + qq[i]) : -1;
             pps[i] = ps[i] >= 0 ? ldcg(Pk + ps[i]) : -1;
         }
+        GP_CK_SINK(rr[i_] + pps[i_]);
+        GP_CK(3);
         bool need[kVL], parked_now[kVL];
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
@@ -942,20 +974,9 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
         bool live[kVL];
 #pragma unroll
         for (int i = 0; i < kVL; ++i) live[i] = u[i] >= 0 && p[i] != kNone && !need[i] && !parked_now[i];
-        {
-            // > 32*kFB items would take the two-pass CAS path: split the group's rescans in two
-            // single-batch halves instead (two dependent chains, no CAS)
-            int32_t dsum = 0;
-#pragma unroll
-            for (int i = 0; i < kVL; ++i)
-                if (need[i] && re[i] - rs[i] <= kHubDeg) dsum += re[i] - rs[i];
-            if (kVL >= 2 && warp_sum(dsum) > 32 * kFB) {
-                flat_rescan<kVL, H>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re, 0, kVL / 2);
-                flat_rescan<kVL, H>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re, kVL / 2, kVL);
-            } else {
-                flat_rescan<kVL, H>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re);
-            }
-        }
+        GP_CK(4);
+        flat_rescan<kVL, H>(a, sm, Pk, Pn, Pkw, next, u, need, live, scanned, rows, rs, re);
+        GP_CK(5);
         if (kStatic) {
 #pragma unroll
             for (int i = 0; i < kVL; ++i) qn += live[i] ? 1 : 0;  // live count only
@@ -963,14 +984,22 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
 #pragma unroll
             for (int i = 0; i < kVL; ++i) wq_push(q, qn, Ln, &next->live, live[i], u[i]);
         }
+        GP_CK(6);
+        GP_CK_ON(false);  // first group only
     }
+    GP_CK_ON(a.prof == 2 && blockIdx.x == 0 && threadIdx.x < 32 && k < 16);
+    GP_CK(7);
     if (kStatic) {
         const int32_t c = warp_sum(qn);
         if (lane == 0 && c) atomicAdd(&next->live, c);  // result unused: a RED, no round trip
     } else {
         cta_flush(sm, q, qn, Ln, &next->live);
     }
+    GP_CK(8);
 }
+#undef GP_CK
+#undef GP_CK_ON
+#undef GP_CK_SINK
 
 template <bool H>
 __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int32_t len, bool stat, bool park,
@@ -978,7 +1007,7 @@ __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int
                         unsigned long long &visits, int32_t &made) {
     (void)n;
     unsigned long long t0 = 0, rows0 = rows;
-    if (a.prof) {
+    if (a.prof == 1) {
         if (threadIdx.x == 0) sm.tmax = 0;
         __syncthreads();
         t0 = globaltimer();
@@ -989,10 +1018,14 @@ __device__ void phase_k(const MatchArgs &a, MatchSmem &sm, int32_t n, int k, int
         else phase_k_impl<H, 1, true>(a, sm, k, len, false, nullptr, scanned, rows, visits, made);
     } else if ((long long)len >= 4LL * threads) phase_k_impl<H, 4>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
     else if (a.lanes_mode == 0 || (long long)len * 2 > threads) phase_k_impl<H, 1>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
+    else if (a.lanes_mode == 2) {  // short lists: 4..16 vertices per warp, flat rescans over all 32 lanes
+        const int vpg = (long long)len * 8 <= threads ? 4 : (long long)len * 4 <= threads ? 8 : 16;
+        phase_k_impl<H, 1>(a, sm, k, len, park, Lover, scanned, rows, visits, made, vpg);
+    }
     else if ((long long)len * 8 <= threads) phase_k_lanes<8, H>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
     else if ((long long)len * 4 <= threads) phase_k_lanes<4, H>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
     else phase_k_lanes<2, H>(a, sm, k, len, park, Lover, scanned, rows, visits, made);
-    if (a.prof && k < 16) {  // one shared atomic per warp, one global atomic per CTA
+    if (a.prof == 1 && k < 16) {  // one shared atomic per warp, one global atomic per CTA
         const unsigned long long dt = globaltimer() - t0;
         const int32_t dr = warp_sum((int32_t)(rows - rows0));
         if ((threadIdx.x & 31) == 0) {
@@ -1074,7 +1107,7 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
             // any match this round: one flag store per CTA (only "> 0" is used)
             if (__syncthreads_or(made > 0) && threadIdx.x == 0) *(volatile int32_t *)&ctl->slot[k & 3].matches = 1;
             trace_mark(ctl->trace, tr++);
-            const bool bprof = a.prof && k < 16 && !tail;
+            const bool bprof = a.prof == 1 && k < 16 && !tail;
             if (bprof) {
                 __syncthreads();
                 if (threadIdx.x == 0) {
@@ -1193,8 +1226,11 @@ static int32_t match_vpc() {
 }
 
 int match_grid(Ctx *ctx) {
-    static int per_sm = -1;
-    if (per_sm < 0) {
+    // per device: cudaFuncSetAttribute applies to the current device (the ctx's, DeviceGuard)
+    static int per_sm_dev[kMaxDevices] = {0};
+    int dummy = -1;
+    int &per_sm = (ctx->device >= 0 && ctx->device < kMaxDevices) ? per_sm_dev[ctx->device] : dummy;
+    if (per_sm <= 0) {
         int b = 0;
         cudaFuncSetAttribute(k_match_level<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(MatchSmem) + 128);
         cudaFuncSetAttribute(k_match_level<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(MatchSmem) + 128);
@@ -1265,7 +1301,7 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
         static int pf = -1;
         if (pf < 0) {
             const char *e = getenv("GP_PROF");
-            pf = (e && atoi(e) == 1) ? 1 : 0;
+            pf = e ? atoi(e) : 0;
         }
         a.prof = pf;
         static int sm = -1;

@@ -11,7 +11,7 @@ namespace gp {
 
 struct ValidateOut {
     unsigned long long sum_adjwgt, sum_vwgt;
-    unsigned long long fp_fwd, fp_rev;  // order-independent arc fingerprints
+    unsigned long long fp_fwd, fp_rev;  // arc fingerprints (unused since the exact hash check)
     int32_t first_bad;                  // smallest offending vertex (INT32_MAX = none)
     int32_t bad_mask;                   // which checks failed
     int32_t unsorted;                   // some row is not strictly increasing
@@ -122,6 +122,77 @@ __global__ void k_check_symmetry_sorted(int32_t n, const int32_t *__restrict__ a
     }
 }
 
+// Exact check of rows in ANY order (R15): every row gets an open-addressing set of its arc
+// positions, p(u) = next_pow2(2 deg u) slots at tbl[4 adjp[u]] (p < 4 deg u, load <= 1/2).
+// Insert: a probe that meets an arc with the same neighbour is a duplicate.  Then every arc
+// (u, v, w) must find an arc (v, u) with weight w in v's set (no duplicates => symmetric
+// multiset, exactly).  A warp per row (hub rows stay balanced inside the warp).
+__device__ __forceinline__ uint32_t vslot_hash(uint32_t v) {
+    v ^= v >> 16; v *= 0x7feb352du; v ^= v >> 15; v *= 0x846ca68bu; v ^= v >> 16;
+    return v;
+}
+__device__ __forceinline__ uint32_t row_slots(int32_t deg) {
+    uint32_t p = 1;
+    while (p < 2u * (uint32_t)deg) p <<= 1;
+    return p;
+}
+__global__ void k_hash_insert(int32_t n, const int32_t *__restrict__ adjp, const int32_t *__restrict__ adjncy,
+                              int32_t *tbl, ValidateOut *o) {
+    const int lane = threadIdx.x & 31;
+    const long long w0 = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long uu = w0; uu < n; uu += nw) {
+        const int32_t u = (int32_t)uu, s = adjp[u], e = adjp[u + 1];
+        if (e - s < 2) continue;  // a single arc cannot be a duplicate
+        const uint32_t mask = row_slots(e - s) - 1;
+        int32_t *t = tbl + 4LL * s;
+        for (int32_t j = s + lane; j < e; j += 32) {
+            const int32_t v = adjncy[j];
+            uint32_t h = vslot_hash((uint32_t)v) & mask;
+            for (;;) {
+                const int32_t old = atomicCAS(t + h, 0, j + 1);
+                if (old == 0) break;
+                if (adjncy[old - 1] == v) {
+                    flag_bad(o, u, kBadDuplicate);
+                    break;
+                }
+                h = (h + 1) & mask;
+            }
+        }
+    }
+}
+__global__ void k_hash_symmetry(int32_t n, const int32_t *__restrict__ adjp, const int32_t *__restrict__ adjncy,
+                                const int32_t *__restrict__ adjwgt, const int32_t *__restrict__ tbl, ValidateOut *o) {
+    const int lane = threadIdx.x & 31;
+    const long long w0 = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const long long nw = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long uu = w0; uu < n; uu += nw) {
+        const int32_t u = (int32_t)uu, s = adjp[u], e = adjp[u + 1];
+        for (int32_t j = s + lane; j < e; j += 32) {
+            const int32_t v = adjncy[j], w = adjwgt[j];
+            const int32_t vs = adjp[v], ve = adjp[v + 1];
+            bool ok = false;
+            if (ve - vs == 1) {
+                ok = adjncy[vs] == u && adjwgt[vs] == w;
+            } else if (ve - vs > 1) {
+                const uint32_t mask = row_slots(ve - vs) - 1;
+                const int32_t *t = tbl + 4LL * vs;
+                uint32_t h = vslot_hash((uint32_t)u) & mask;
+                for (;;) {
+                    const int32_t k = t[h];
+                    if (k == 0) break;  // u is not in v's row
+                    if (adjncy[k - 1] == u) {
+                        ok = adjwgt[k - 1] == w;
+                        break;
+                    }
+                    h = (h + 1) & mask;
+                }
+            }
+            if (!ok) flag_bad(o, u, kBadAsymmetric);
+        }
+    }
+}
+
 static std::string describe(int32_t mask) {
     std::string s;
     if (mask & kBadOffsets) s += " offsets(adjp[0]=0, monotone, adjp[n]=nnz)";
@@ -134,7 +205,7 @@ static std::string describe(int32_t mask) {
     return s;
 }
 
-gp_status graph_totals_and_validate(Ctx *ctx, const Graph *g, bool validate) {
+gp_status graph_totals_and_validate(Ctx *ctx, Graph *g, bool validate, bool check_totals) {
     ValidateOut *d = nullptr;
     gp_status st = dev_alloc(ctx, (void **)&d, sizeof(ValidateOut));
     if (st != GP_OK) return st;
@@ -143,6 +214,7 @@ gp_status graph_totals_and_validate(Ctx *ctx, const Graph *g, bool validate) {
     h.first_bad = INT32_MAX;
     cudaStream_t s = ctx->stream;
     const int grid = persistent_grid(ctx, 4);
+    int32_t *tbl = nullptr;
     cudaError_t e = cudaMemcpyAsync(d, &h, sizeof(h), cudaMemcpyHostToDevice, s);
     if (e == cudaSuccess && validate && g->n > 0) {
         k_check_offsets<<<grid, kBlock, 0, s>>>(g->n, g->nnz, g->adjp, d);
@@ -154,27 +226,41 @@ gp_status graph_totals_and_validate(Ctx *ctx, const Graph *g, bool validate) {
             if (e == cudaSuccess) e = cudaStreamSynchronize(s);
             if (e == cudaSuccess && h.bad_mask == 0 && !h.unsorted) {
                 k_check_symmetry_sorted<<<grid, kBlock, 0, s>>>(g->n, g->adjp, g->adjncy, g->adjwgt, d);
+                ++ctx->launches;
+            } else if (e == cudaSuccess && h.bad_mask == 0 && h.unsorted && g->nnz > 0) {
+                // unsorted rows: exact per-row hash sets (duplicates first, then symmetry)
+                const size_t tb = sizeof(int32_t) * 4 * (size_t)g->nnz;
+                st = dev_alloc(ctx, (void **)&tbl, tb);
+                if (st == GP_OK) e = cudaMemsetAsync(tbl, 0, tb, s);
+                if (st == GP_OK && e == cudaSuccess) {
+                    k_hash_insert<<<grid, kBlock, 0, s>>>(g->n, g->adjp, g->adjncy, tbl, d);
+                    e = cudaMemcpyAsync(&h, d, sizeof(h), cudaMemcpyDeviceToHost, s);
+                    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+                    if (e == cudaSuccess && h.bad_mask == 0)
+                        k_hash_symmetry<<<grid, kBlock, 0, s>>>(g->n, g->adjp, g->adjncy, g->adjwgt, tbl, d);
+                    ctx->launches += 2;
+                }
             }
         }
-        ctx->launches += 3;
+        ctx->launches += 2;
     }
-    if (e == cudaSuccess && (!validate || h.bad_mask == 0)) {
+    if (st == GP_OK && e == cudaSuccess && (!validate || h.bad_mask == 0)) {
         k_totals<<<grid, kBlock, 0, s>>>(g->n, g->nnz, g->adjwgt, g->vwgt, d);
         ++ctx->launches;
         e = cudaMemcpyAsync(&h, d, sizeof(h), cudaMemcpyDeviceToHost, s);
         if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     }
+    dev_free(ctx, tbl);
     dev_free(ctx, d);
+    if (st != GP_OK) return st;
     if (e != cudaSuccess) return cuda_fail(e, "graph validation");
-    if (validate && h.bad_mask == 0 && h.unsorted && h.fp_fwd != h.fp_rev) {
-        h.bad_mask = kBadAsymmetric;
-        h.first_bad = -1;
-    }
     if (validate && h.bad_mask) {
         set_error("GP_VALIDATE: first offending vertex " + std::to_string(h.first_bad) + ":" + describe(h.bad_mask));
         return GP_ERR_INVALID_GRAPH;
     }
-    if (h.sum_adjwgt > (unsigned long long)INT32_MAX || h.sum_vwgt > (unsigned long long)INT32_MAX) {
+    g->sum_adjwgt = h.sum_adjwgt;
+    g->sum_vwgt = h.sum_vwgt;
+    if (check_totals && (h.sum_adjwgt > (unsigned long long)INT32_MAX || h.sum_vwgt > (unsigned long long)INT32_MAX)) {
         set_error("weight totals exceed INT32_MAX: sum(adjwgt)=" + std::to_string(h.sum_adjwgt) +
                   " sum(vwgt)=" + std::to_string(h.sum_vwgt));
         return GP_ERR_OVERFLOW;

@@ -12,6 +12,7 @@ from __future__ import annotations
 
 import ctypes
 import os
+import weakref
 from dataclasses import dataclass
 from typing import Dict, List, Optional
 
@@ -74,6 +75,10 @@ def _sig(name, res, args):
 _sig("gp_status_string", ctypes.c_char_p, [ctypes.c_int])
 _sig("gp_last_error", ctypes.c_char_p, [])
 _sig("gp_ctx_create", ctypes.c_int, [ctypes.c_int, _vp, ctypes.POINTER(_vp)])
+# gp_alloc_fn / gp_dealloc_fn (include/gp.h)
+ALLOC_FN = ctypes.CFUNCTYPE(_vp, ctypes.c_size_t, _vp, _vp)
+DEALLOC_FN = ctypes.CFUNCTYPE(None, _vp, _vp, _vp)
+_sig("gp_ctx_set_allocator", ctypes.c_int, [_vp, ALLOC_FN, DEALLOC_FN, _vp])
 _sig("gp_ctx_num_sms", ctypes.c_int, [_vp, _i32p])
 _sig("gp_graph_create", ctypes.c_int, [_vp, _i32, _vp, _vp, _vp, _vp, ctypes.c_uint32, ctypes.POINTER(_vp)])
 _sig("gp_graph_view", ctypes.c_int, [_vp, _i32p, _i32p, ctypes.POINTER(_vp), ctypes.POINTER(_vp),
@@ -99,6 +104,7 @@ _sig("gp_ctx_set_timing", ctypes.c_int, [_vp, _i32])
 _sig("gp_ctx_kernel_stats", ctypes.c_int, [_vp, ctypes.c_int, ctypes.POINTER(KernelStats)])
 _sig("gp_ctx_reset_stats", ctypes.c_int, [_vp])
 _sig("gp_ctx_launch_count", ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_int64)])
+_sig("gp_ctx_launch_times", ctypes.c_int, [_vp, _i32, _vp, _vp, _i32p])
 
 
 def _check(st: int, where: str) -> None:
@@ -145,6 +151,46 @@ class Context:
         else:
             _check(_lib.gp_ctx_create(device, self.stream.cuda_stream, ctypes.byref(h)), "gp_ctx_create")
         self.handle = h
+        self._children = weakref.WeakSet()  # live Graph / Hierarchy objects (closed before the context)
+        self._alloc_cbs = None              # keeps the ctypes allocator callbacks alive
+
+    def _h(self):
+        if self.handle is None or not self.handle.value:
+            raise RuntimeError("gp context is closed")
+        return self.handle
+
+    def _adopt(self, obj) -> None:
+        self._children.add(obj)
+
+    def set_allocator(self, alloc=None, dealloc=None) -> None:
+        """gp_ctx_set_allocator: route the library's device allocations through Python
+        callables alloc(nbytes, stream) -> int pointer and dealloc(ptr, stream); None restores
+        cudaMallocAsync.  Refused (GPError) while graphs or hierarchies of this context are alive."""
+        if (alloc is None) != (dealloc is None):
+            raise ValueError("alloc and dealloc go together")
+        if alloc is None:
+            cbs = (ctypes.cast(None, ALLOC_FN), ctypes.cast(None, DEALLOC_FN))
+        else:
+            def _a(nbytes, stream, user):
+                try:
+                    return int(alloc(int(nbytes), stream))
+                except Exception:  # the library reports GP_ERR_OUT_OF_MEMORY
+                    return None
+
+            def _d(ptr, stream, user):
+                try:
+                    dealloc(ptr, stream)
+                except Exception:
+                    pass
+            cbs = (ALLOC_FN(_a), DEALLOC_FN(_d))
+        _check(_lib.gp_ctx_set_allocator(self._h(), cbs[0], cbs[1], None), "gp_ctx_set_allocator")
+        self._alloc_cbs = cbs
+
+    def use_torch_allocator(self) -> None:
+        """Allocate through torch's caching allocator (stream-ordered on the context stream)."""
+        dev = self.device
+        self.set_allocator(lambda n, stream: torch.cuda.caching_allocator_alloc(n, dev, stream),
+                           lambda p, stream: torch.cuda.caching_allocator_delete(p))
 
     def dist_info(self):
         """(rank, nranks): (0, 1) single GPU, (-1, G) loopback."""
@@ -153,7 +199,15 @@ class Context:
         return r.value, g.value
 
     def close(self) -> None:
+        """Free the context; its live hierarchies and graphs are closed first (gp.h: a graph
+        or hierarchy must be freed before its context)."""
         if self.handle is not None and self.handle.value:
+            kids = list(getattr(self, "_children", ()))
+            for k in kids:
+                if isinstance(k, Hierarchy):
+                    k.close()
+            for k in kids:
+                k.close()
             _lib.gp_free(self.handle)
         self.handle = None
 
@@ -183,6 +237,16 @@ class Context:
             out[name] = {"launches": int(s.launches), "ms": float(s.ms)}
         return out
 
+    def launch_times(self):
+        """[(kind name, ms)] of every timed launch since the last reset_stats (launch order)."""
+        cnt = _i32()
+        _check(_lib.gp_ctx_launch_times(self.handle, 0, None, None, ctypes.byref(cnt)), "gp_ctx_launch_times")
+        n = cnt.value
+        kinds = (ctypes.c_int32 * max(n, 1))()
+        ms = (ctypes.c_float * max(n, 1))()
+        _check(_lib.gp_ctx_launch_times(self.handle, n, kinds, ms, ctypes.byref(cnt)), "gp_ctx_launch_times")
+        return [(KERNEL_KINDS[kinds[i]], float(ms[i])) for i in range(min(n, cnt.value))]
+
     def launch_count(self) -> int:
         v = ctypes.c_int64()
         _check(_lib.gp_ctx_launch_count(self.handle, ctypes.byref(v)), "gp_ctx_launch_count")
@@ -192,10 +256,22 @@ class Context:
 class Graph:
     """Library-owned device CSR graph (gp_graph)."""
 
-    def __init__(self, ctx: Context, handle, owned: bool = True):
+    def __init__(self, ctx: Context, handle, owned: bool = True, parent: Optional["Hierarchy"] = None):
         self.ctx = ctx
         self.handle = handle
         self.owned = owned
+        self.parent = parent  # a borrowed level graph keeps its hierarchy alive
+        if owned:
+            ctx._adopt(self)
+
+    def _h(self):
+        if self.handle is None or not self.handle.value:
+            raise RuntimeError("gp graph is closed")
+        if self.parent is not None and self.parent.handle is None:
+            raise RuntimeError("gp graph belongs to a hierarchy that was closed")
+        if self.ctx.handle is None:
+            raise RuntimeError("gp context is closed")
+        return self.handle
 
     @classmethod
     def create(cls, ctx: Context, adjp: torch.Tensor, adjncy: torch.Tensor, adjwgt: Optional[torch.Tensor] = None,
@@ -209,7 +285,7 @@ class Graph:
                 raise ValueError("inputs must all be on the device or all on the host")
         flags = (GP_INPUT_DEVICE if dev else 0) | (GP_VALIDATE if validate else 0)
         h = _vp()
-        _check(_lib.gp_graph_create(ctx.handle, n, _ptr(adjp), _ptr(adjncy), _ptr(adjwgt), _ptr(vwgt), flags,
+        _check(_lib.gp_graph_create(ctx._h(), n, _ptr(adjp), _ptr(adjncy), _ptr(adjwgt), _ptr(vwgt), flags,
                                     ctypes.byref(h)), "gp_graph_create")
         return cls(ctx, h)
 
@@ -222,12 +298,12 @@ class Graph:
         v_end = v_begin + adjp_local.numel() - 1
         flags = GP_INPUT_DEVICE if adjp_local.is_cuda else 0
         h = _vp()
-        _check(_lib.gp_graph_create_dist(ctx.handle, n_global, v_begin, v_end, _ptr(adjp_local), _ptr(adjncy),
+        _check(_lib.gp_graph_create_dist(ctx._h(), n_global, v_begin, v_end, _ptr(adjp_local), _ptr(adjncy),
                                          _ptr(adjwgt), _ptr(vwgt), flags, ctypes.byref(h)), "gp_graph_create_dist")
         return cls(ctx, h)
 
     def close(self) -> None:
-        if self.owned and self.handle is not None and self.handle.value:
+        if self.owned and self.handle is not None and self.handle.value and self.ctx.handle is not None:
             _lib.gp_free(self.handle)
         self.handle = None
 
@@ -239,7 +315,7 @@ class Graph:
 
     def view(self):
         n, nnz = _i32(), _i32()
-        _check(_lib.gp_graph_view(self.handle, ctypes.byref(n), ctypes.byref(nnz), None, None, None, None),
+        _check(_lib.gp_graph_view(self._h(), ctypes.byref(n), ctypes.byref(nnz), None, None, None, None),
                "gp_graph_view")
         return n.value, nnz.value
 
@@ -258,7 +334,7 @@ class Graph:
         if out is None:
             out = {k: torch.empty(sz, dtype=torch.int32) for k, sz in
                    (("adjp", n + 1), ("adjncy", nnz), ("adjwgt", nnz), ("vwgt", n))}
-        _check(_lib.gp_graph_download(self.handle, out["adjp"].data_ptr(), out["adjncy"].data_ptr(),
+        _check(_lib.gp_graph_download(self._h(), out["adjp"].data_ptr(), out["adjncy"].data_ptr(),
                                       out["adjwgt"].data_ptr(), out["vwgt"].data_ptr()), "gp_graph_download")
         out["n"], out["nnz"] = n, nnz
         return out
@@ -268,21 +344,21 @@ class Graph:
         """gp_match_level_ex into a caller-owned device int32[n] tensor; returns rounds.
         tie_seed != 0: equal-weight ties go to the lower lowbias32(v ^ seed) (RM, P18.s8)."""
         r = _i32()
-        _check(_lib.gp_match_level_ex(self.handle, _ptr(match), max_rounds, tie_seed & 0xFFFFFFFF,
+        _check(_lib.gp_match_level_ex(self._h(), _ptr(match), max_rounds, tie_seed & 0xFFFFFFFF,
                                       ctypes.byref(r) if sync_rounds else None), "gp_match_level_ex")
         return r.value if sync_rounds else None
 
     def contract_level(self, match: torch.Tensor, cmap: torch.Tensor) -> "Graph":
         """gp_contract_level: fills cmap, returns the coarse graph (caller-owned)."""
         h = _vp()
-        _check(_lib.gp_contract_level(self.handle, _ptr(match), _ptr(cmap), ctypes.byref(h)), "gp_contract_level")
+        _check(_lib.gp_contract_level(self._h(), _ptr(match), _ptr(cmap), ctypes.byref(h)), "gp_contract_level")
         return Graph(self.ctx, h)
 
     def coarsen_to(self, threshold: int, stall_ratio_pct: int = 95, max_levels: int = 64,
                    max_rounds: int = 0, tie_seed: int = 0) -> "Hierarchy":
         opts = CoarsenOpts(threshold, stall_ratio_pct, max_levels, max_rounds, tie_seed & 0xFFFFFFFF)
         h = _vp()
-        _check(_lib.gp_coarsen_to(self.handle, ctypes.byref(opts), ctypes.byref(h)), "gp_coarsen_to")
+        _check(_lib.gp_coarsen_to(self._h(), ctypes.byref(opts), ctypes.byref(h)), "gp_coarsen_to")
         return Hierarchy(self.ctx, h)
 
 
@@ -311,9 +387,18 @@ class Hierarchy:
     def __init__(self, ctx: Context, handle):
         self.ctx = ctx
         self.handle = handle
+        ctx._adopt(self)
+
+    def _h(self):
+        if self.handle is None or not self.handle.value:
+            raise RuntimeError("gp hierarchy is closed")
+        if self.ctx.handle is None:
+            raise RuntimeError("gp context is closed")
+        return self.handle
 
     def close(self) -> None:
-        if self.handle is not None and self.handle.value:
+        """Free the hierarchy; the borrowed level graphs (LevelInfo.coarse) become unusable."""
+        if self.handle is not None and self.handle.value and self.ctx.handle is not None:
             _lib.gp_free(self.handle)
         self.handle = None
 
@@ -325,14 +410,15 @@ class Hierarchy:
 
     def __len__(self) -> int:
         v = _i32()
-        _check(_lib.gp_hier_num_levels(self.handle, ctypes.byref(v)), "gp_hier_num_levels")
+        _check(_lib.gp_hier_num_levels(self._h(), ctypes.byref(v)), "gp_hier_num_levels")
         return v.value
 
     def level(self, i: int) -> LevelInfo:
         l = Level()
-        _check(_lib.gp_hier_level(self.handle, i, ctypes.byref(l)), "gp_hier_level")
+        _check(_lib.gp_hier_level(self._h(), i, ctypes.byref(l)), "gp_hier_level")
         return LevelInfo(l.n, l.nnz, l.n_coarse, l.cnnz, l.rounds, bool(l.maximal), l.stop_reason,
-                         l.arcs_scanned, l.rows_scanned, l.live_visits, Graph(self.ctx, _vp(l.coarse), owned=False),
+                         l.arcs_scanned, l.rows_scanned, l.live_visits,
+                         Graph(self.ctx, _vp(l.coarse), owned=False, parent=self),
                          l.v_begin, l.n_local, l.cv_begin, l.n_coarse_local)
 
     def levels(self) -> List[LevelInfo]:
@@ -347,7 +433,7 @@ class Hierarchy:
         n = info.n_local if rank >= 0 else info.n  # NCCL rank: its piece; loopback / 1 GPU: all
         m = None if not want_match else (match if match is not None else torch.empty(n, dtype=torch.int32))
         c = cmap if cmap is not None else torch.empty(n, dtype=torch.int32)
-        _check(_lib.gp_hier_download_level(self.handle, i, m.data_ptr() if m is not None else None, c.data_ptr()),
+        _check(_lib.gp_hier_download_level(self._h(), i, m.data_ptr() if m is not None else None, c.data_ptr()),
                "gp_hier_download_level")
         return m, c
 
@@ -358,7 +444,7 @@ class Hierarchy:
         carried down to level to_level's fine graph, written into part_fine (device)."""
         if from_level is None:
             from_level = len(self) - 1
-        _check(_lib.gp_project(self.handle, from_level, to_level, _ptr(part_coarse), _ptr(part_fine)), "gp_project")
+        _check(_lib.gp_project(self._h(), from_level, to_level, _ptr(part_coarse), _ptr(part_fine)), "gp_project")
         return part_fine
 
     def download_coarse(self, i: int) -> Dict[str, torch.Tensor]:
@@ -370,7 +456,7 @@ class Hierarchy:
         out = {"adjp": torch.empty(n + 1, dtype=torch.int32), "adjncy": torch.empty(max(info.cnnz, 1), dtype=torch.int32),
                "adjwgt": torch.empty(max(info.cnnz, 1), dtype=torch.int32), "vwgt": torch.empty(max(n, 1), dtype=torch.int32)}
         rows, arcs = _i32(), _i32()
-        _check(_lib.gp_hier_download_coarse(self.handle, i, out["adjp"].data_ptr(), out["adjncy"].data_ptr(),
+        _check(_lib.gp_hier_download_coarse(self._h(), i, out["adjp"].data_ptr(), out["adjncy"].data_ptr(),
                                             out["adjwgt"].data_ptr(), out["vwgt"].data_ptr(), ctypes.byref(rows),
                                             ctypes.byref(arcs)), "gp_hier_download_coarse")
         out["adjncy"] = out["adjncy"][:arcs.value]

@@ -50,6 +50,32 @@ def greedy_matching(n: int, edges: List[Tuple[int, int, int]]) -> np.ndarray:
     return m
 
 
+def one_shot_hem(g: Dict) -> np.ndarray:
+    """The paper's one-pass GPU matching with its races removed (P18.s7-13): every vertex
+    takes its heaviest neighbour -- all vertices are unmatched when the single HEM kernel runs;
+    ties go to the lower id (north_star) -- and the conflict kernel keeps a pair only if the
+    choice is mutual ("M[u] = v and M[v] != u => M[u] = u", P18.s11-12); every other vertex is
+    matched to itself.  Vectorised numpy, written from the definition (no rounds, no lists)."""
+    g = np_graph(g)
+    n = g["n"]
+    m = np.arange(n, dtype=np.int64)
+    if len(g["adjncy"]) == 0:
+        return m
+    src = np.repeat(np.arange(n), np.diff(g["adjp"]))
+    # heaviest neighbour of every row: sort arcs by (row, -w, v) and take each row's first
+    order = np.lexsort((g["adjncy"], -g["adjwgt"], src))
+    first = np.ones(len(order), dtype=bool)
+    first[1:] = src[order][1:] != src[order][:-1]
+    pick = order[first]
+    h = np.full(n, -1, dtype=np.int64)
+    h[src[pick]] = g["adjncy"][pick]
+    has = h >= 0
+    mutual = np.zeros(n, dtype=bool)
+    mutual[has] = h[h[has]] == np.arange(n)[has]
+    m[mutual] = h[mutual]
+    return m
+
+
 def max_weight_matching_bruteforce(n: int, edges: List[Tuple[int, int, int]]) -> int:
     """Exhaustive maximum matching weight (tiny graphs only)."""
     best = 0

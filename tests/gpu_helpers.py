@@ -15,9 +15,9 @@ def to_device(g: Dict) -> Dict:
             for k in ("adjp", "adjncy", "adjwgt", "vwgt")}
 
 
-def gpu_coarsen(gp, ctx, g: Dict, threshold: int, **kw) -> List[Dict]:
+def gpu_coarsen(gp, ctx, g: Dict, threshold: int, validate: bool = False, **kw) -> List[Dict]:
     d = to_device(g)
-    G = gp.Graph.create(ctx, d["adjp"], d["adjncy"], d["adjwgt"], d["vwgt"])
+    G = gp.Graph.create(ctx, d["adjp"], d["adjncy"], d["adjwgt"], d["vwgt"], validate=validate)
     H = G.coarsen_to(threshold, **kw)
     out = []
     for i, info in enumerate(H.levels()):

@@ -1,10 +1,9 @@
 """Full-size parity (-m gpu): BASELINE.json's configs at their full sizes, in the launch
 configuration bench.py times (gp_coarsen_to on a device-resident graph).
 
-C1, C2, C3 and C5 are compared with the oracle at every level, element by element.  C4
-(R-MAT scale 24, 2^28 endpoint draws) is compared with the oracle on level 0 (matching,
-cmap and coarse graph); its later levels are checked by the per-level invariants, which
-hold at any size.
+Every config is compared with the oracle at every level, element by element.  C4 (R-MAT
+scale 24, 2^28 endpoint draws) chains the oracle's per-level functions level by level on the
+already-verified coarse graphs, and also checks the per-level invariants.
 """
 import numpy as np
 import pytest
@@ -78,22 +77,31 @@ def _vector_invariants(fine, lvl):
 
 
 def test_full_rmat_s24(gp, ctx):
+    """C4 at full size, EVERY level bit-compared with the oracle: level l's oracle step
+    (match_level, cmap, contract) runs on level l-1's coarse graph, which the previous
+    iteration has already proven equal to the oracle's (so the chain is the oracle's own
+    hierarchy without keeping all of it in host memory at once)."""
     g = G.make_config("C4", device="cuda")
     got = gpu_coarsen(gp, ctx, g, threshold=100)
     gh = _host(g)
     del g
     torch.cuda.empty_cache()
-    # level 0 against the oracle, element by element
-    m, rounds, maximal = oracle.match_level(gh)
-    assert rounds == got[0]["rounds"] and maximal == got[0]["maximal"]
-    assert np.array_equal(m, got[0]["match"])
-    cm, n_c = oracle.cmap(m)
-    assert np.array_equal(cm, got[0]["cmap"]) and n_c == got[0]["n_coarse"]
-    c = oracle.contract(gh, m, cm, n_c)
-    for k in ("adjp", "adjncy", "adjwgt", "vwgt"):
-        assert np.array_equal(c[k], got[0]["coarse"][k]), k
-    # every level: invariants that hold at any size
     fine = gh
-    for lvl in got:
+    for i, lvl in enumerate(got):
+        where = f"C4 level {i}"
+        assert lvl["n"] == len(fine["adjp"]) - 1, where
+        m, rounds, maximal = oracle.match_level(fine)
+        assert rounds == lvl["rounds"] and maximal == lvl["maximal"], (where, rounds, lvl["rounds"])
+        assert np.array_equal(m, lvl["match"]), f"{where}: match"
+        cm, n_c = oracle.cmap(m)
+        assert np.array_equal(cm, lvl["cmap"]) and n_c == lvl["n_coarse"], f"{where}: cmap"
+        c = oracle.contract(fine, m, cm, n_c)
+        for k in ("adjp", "adjncy", "adjwgt", "vwgt"):
+            assert np.array_equal(c[k], lvl["coarse"][k]), f"{where}: coarse {k}"
+        stall = 100 * n_c > 95 * lvl["n"]
+        if i < len(got) - 1:
+            assert lvl["stop_reason"] == 0 and not stall and n_c > 100, where
+        else:
+            assert lvl["stop_reason"] == (oracle.STOP_STALL if stall else oracle.STOP_THRESHOLD), where
         _vector_invariants(fine, lvl)
-        fine = lvl["coarse"]
+        fine = c

@@ -67,3 +67,24 @@ def test_deterministic():
     b = G.rgg(1 << 11)
     for k in ("adjp", "adjncy", "adjwgt"):
         assert torch.equal(a[k], b[k])
+
+
+def test_shuffle_rows_keeps_the_graph():
+    g = G.rgg(1 << 10)
+    s = G.shuffle_rows(g, 3)
+    a, b = np_graph(g), np_graph(s)
+    assert np.array_equal(a["adjp"], b["adjp"]) and np.array_equal(a["vwgt"], b["vwgt"])
+    moved = 0
+    for u in range(a["n"]):
+        lo, hi = a["adjp"][u], a["adjp"][u + 1]
+        x = sorted(zip(a["adjncy"][lo:hi], a["adjwgt"][lo:hi]))
+        y = sorted(zip(b["adjncy"][lo:hi], b["adjwgt"][lo:hi]))
+        assert x == y
+        moved += int(not np.array_equal(a["adjncy"][lo:hi], b["adjncy"][lo:hi]))
+    assert moved > a["n"] // 2      # most rows are really reordered
+    check_csr(s, "shuffled")
+
+
+def test_varied_vwgt():
+    g = G.varied_vwgt(G.grid2d(5, 5), period=7)
+    assert g["vwgt"].tolist() == [1 + u % 7 for u in range(25)]

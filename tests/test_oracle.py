@@ -19,7 +19,7 @@ import torch
 
 import graphgen as G
 import oracle
-from checks import (check_csr, check_level, check_matching, contract_by_sparse_triple_product,
+from checks import (check_csr, check_level, check_matching, contract_by_sparse_triple_product, one_shot_hem,
                     edge_list, greedy_matching, max_weight_matching_bruteforce, np_graph)
 
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
@@ -204,3 +204,74 @@ def test_relabel_equivariance_distinct_weights():
     ma, _, _ = oracle.match_level(g)
     mb, _, _ = oracle.match_level(h)
     assert np.array_equal(perm[ma], mb[perm])
+
+
+# ---- stop-rule boundaries (readings R12 / R13) ------------------------------------------
+# R12 "coarsen until |V| is below a threshold" (P10.s16, P20.s30) is read as "continue while
+# n > threshold"; R13 (Metis' "difference ... less than a threshold", P12.s30) as "stop after a
+# level with 100*n_c > 95*n".  Each case sits exactly on a boundary, so the strict and the
+# non-strict comparison give different level counts (a '>=' in either test fails a case).
+
+def test_threshold_boundary_c1_closed_form():
+    # C1's closed form: n = 4096 -> 2048 -> ... -> 64, one halving per level
+    g = G.make_config("C1")
+    lv = oracle.coarsen_to(g, threshold=64)
+    assert [l["n"] for l in lv] == [4096, 2048, 1024, 512, 256, 128]       # n == 64 is not > 64: stop
+    assert lv[-1]["n_coarse"] == 64 and lv[-1]["stop_reason"] == oracle.STOP_THRESHOLD
+    lv = oracle.coarsen_to(g, threshold=63)                                  # 64 > 63: one more level
+    assert [l["n"] for l in lv][-1] == 64 and lv[-1]["n_coarse"] == 32
+    lv = oracle.coarsen_to(g, threshold=4096)                                # input already at the threshold
+    assert lv == []
+
+
+def test_stall_boundary_one_edge():
+    # 20 vertices, one edge: level 0 gives n_c = 19 and 100*19 == 95*20 -- not a stall
+    # (strict '>'); level 1 has no edge, n_c = n = 19 -> stall.  So exactly 2 levels.
+    g = G.from_edge_list(20, [(3, 11, 5)])
+    lv = oracle.coarsen_to(g, threshold=1)
+    assert [(l["n"], l["n_coarse"]) for l in lv] == [(20, 19), (19, 19)]
+    assert [l["stop_reason"] for l in lv] == [0, oracle.STOP_STALL]
+    # 21 vertices, one edge: 100*20 = 2000 > 95*21 = 1995 -> stall after level 0
+    g = G.from_edge_list(21, [(3, 11, 5)])
+    lv = oracle.coarsen_to(g, threshold=1)
+    assert [(l["n"], l["n_coarse"]) for l in lv] == [(21, 20)]
+    assert lv[0]["stop_reason"] == oracle.STOP_STALL
+    # stall_ratio_pct is the percentage of the same integer test: 100*19 > 94*20 stalls at once
+    g = G.from_edge_list(20, [(3, 11, 5)])
+    lv = oracle.coarsen_to(g, threshold=1, stall_ratio_pct=94)
+    assert len(lv) == 1 and lv[0]["stop_reason"] == oracle.STOP_STALL
+
+
+def test_max_levels_boundary():
+    g = G.make_config("C1")
+    lv = oracle.coarsen_to(g, threshold=100, max_levels=3)
+    assert len(lv) == 3 and lv[-1]["stop_reason"] == oracle.STOP_MAX_LEVELS
+    lv = oracle.coarsen_to(g, threshold=100, max_levels=6)                  # the 6th level also reaches 64
+    assert len(lv) == 6 and lv[-1]["stop_reason"] == oracle.STOP_THRESHOLD
+
+
+# ---- the paper's one-shot matching ----------------------------------
+# P18.s7-13: ONE lock-free HEM pass (every vertex grabs its heaviest neighbour) + the conflict
+# kernel (non-mutual choices self-match).  With the races removed and ties to the lower id,
+# that is exactly the pinned rule capped at one round (max_rounds = 1, leftover = the conflict
+# kernel's self-matches).  checks.one_shot_hem computes it directly from the graph.
+@pytest.mark.parametrize("seed", range(30))
+def test_one_shot_equals_max_rounds_1(seed):
+    n = 10 + 37 * seed
+    g = G.random_graph(n, 3 * n, seed + 4000, wmax=[1, 3, 100][seed % 3])
+    m, rounds, maximal = oracle.match_level(g, max_rounds=1)
+    ref = one_shot_hem(g)
+    assert np.array_equal(m.astype(np.int64), ref)
+    assert rounds == (1 if np.any(ref != np.arange(n)) else 0)
+
+
+@pytest.mark.parametrize("name,make", [("C3", lambda: G.delaunay_like(64)), ("C5", lambda: G.road_like(64)),
+                                       ("C2", lambda: G.rgg(1 << 12)), ("C4", lambda: G.rmat(10))])
+def test_one_shot_hierarchy(name, make):
+    g = make()
+    levels = oracle.coarsen_to(g, threshold=100, max_rounds=1)
+    cur = g
+    for l in levels:
+        assert np.array_equal(l["match"].astype(np.int64), one_shot_hem(cur))
+        check_matching(cur, l["match"], maximal=False)
+        cur = l["coarse"]
