@@ -213,6 +213,38 @@ gp_status gp_hier_download_coarse(gp_hier h, int32_t i, gp_vid *h_adjp, gp_vid *
 gp_status gp_project(gp_hier h, int32_t from_level, int32_t to_level, const gp_vid *d_part_coarse,
                      gp_vid *d_part_fine);
 
+/* ---- un-coarsening: refinement (PAPER.md P22.s1-22) -----------------
+ * Lock-free refinement of a k-way labelling on one graph (reading R18 of DESIGN.md §2): per
+ * pass two iterations, the first moving vertices only to HIGHER partition ids, the second only
+ * to LOWER ones (the paper's ordering method, P22.s8-10).  In an iteration every boundary
+ * vertex v of partition s requests the neighbouring partition d (in the iteration's direction)
+ * with the largest gain w(v,d) - w(v,s) > 0 (ties: lower d) if s keeps >= min_w and d stays
+ * <= max_w (P22.s4-7); each destination explores its requests in (gain desc, vertex asc) order
+ * and accepts them while its weight stays <= max_w (P22.s16-19); accepted vertices move
+ * together.  max_w = ceil(W (100 + imbalance_pct) / (100 k)), min_w = floor(W (100 -
+ * imbalance_pct) / (100 k)), W = sum(vwgt).  Stops after a pass without moves or max_passes.
+ * Deterministic: equal to the oracle bit for bit. */
+typedef struct {
+    int32_t nparts;         /* k, 1..1024                                            */
+    int32_t imbalance_pct;  /* balance tolerance in percent (the paper uses 3)       */
+    int32_t max_passes;     /* passes per level (each = two directed iterations)     */
+} gp_refine_opts;
+
+/* Refine d_part (device int32[n], labels in [0, nparts), updated in place) on graph g.
+ * moves_out / passes_out (nullable) receive the accepted moves and the passes run.
+ * Synchronous (one host read per iteration decides early termination).  Single-GPU graphs. */
+gp_status gp_refine(gp_graph g, gp_vid *d_part, const gp_refine_opts *opts, int32_t *moves_out,
+                    int32_t *passes_out);
+
+/* Un-coarsening on the GPU (P12.s41-46; P20.s41-P22.s22): starting from d_part_coarse (device
+ * int32[n_coarse of the last level]), for every level from the coarsest to level 0: project
+ * one level (as gp_project) and refine on that level's fine graph (gp_refine).  g0 is the graph
+ * the hierarchy was built from (its level-0 fine graph).  d_part_fine: device int32[n of g0],
+ * caller-owned, receives the level-0 labels.  moves_out (nullable): total moves.
+ * Synchronous.  Single-GPU hierarchies only. */
+gp_status gp_uncoarsen(gp_hier h, gp_graph g0, const gp_vid *d_part_coarse, gp_vid *d_part_fine,
+                       const gp_refine_opts *opts, int32_t *moves_out);
+
 /* ---- sharded coarsening over several GPUs -------------------
  * Vertex ranges are sharded over the ranks of one node (one process per GPU).  Each rank
  * owns the contiguous global ids [v_begin, v_end) and holds their CSR rows with GLOBAL

@@ -51,6 +51,9 @@ def _load():
         lib.oracle_tie_hash.argtypes = [ctypes.c_uint32, ctypes.c_uint32]
         lib.oracle_cmap.restype = ctypes.c_int32
         lib.oracle_cmap.argtypes = [ctypes.c_int32, _i32p, _i32p]
+        lib.oracle_refine.restype = ctypes.c_int
+        lib.oracle_refine.argtypes = [ctypes.c_int32, _i32p, _i32p, _i32p, _i32p, ctypes.c_int32, ctypes.c_int32,
+                                      ctypes.c_int32, _i32p, _i32p, _i32p]
         lib.oracle_contract.restype = ctypes.c_int64
         lib.oracle_contract.argtypes = [ctypes.c_int32, _i32p, _i32p, _i32p, _i32p, _i32p, _i32p,
                                         ctypes.c_int32, _i32p, _i32p, _i32p, _i32p]
@@ -165,6 +168,35 @@ def coarsen_to(g: Dict, threshold: int, stall_ratio_pct: int = 95, max_levels: i
     if levels and levels[-1]["stop_reason"] == 0:
         levels[-1]["stop_reason"] = STOP_THRESHOLD if cur["n"] <= threshold else STOP_MAX_LEVELS
     return levels
+
+
+def refine(g: Dict, part, nparts: int, imbalance_pct: int = 3, max_passes: int = 8):
+    """Refinement of un-coarsening (oracle.c: oracle_refine; P22.s1-22, reading R18).
+    Returns (part int32[n], moves, passes)."""
+    lib = _load()
+    g = as_numpy_graph(g)
+    p = _np32(part).copy()
+    moves, passes = ctypes.c_int32(0), ctypes.c_int32(0)
+    st = lib.oracle_refine(g["n"], _p(g["adjp"]), _p(g["adjncy"]), _p(g["adjwgt"]), _p(g["vwgt"]), int(nparts),
+                           int(imbalance_pct), int(max_passes), _p(p), ctypes.byref(moves), ctypes.byref(passes))
+    if st != 0:
+        raise ValueError("oracle_refine: bad arguments (labels outside [0, nparts)?)")
+    return p, int(moves.value), int(passes.value)
+
+
+def uncoarsen(g0: Dict, levels: List[Dict], part_coarse, nparts: int, imbalance_pct: int = 3,
+              max_passes: int = 8):
+    """Un-coarsening (P12.s41-46; P20.s41-P22.s22): from the coarsest graph down to level 0,
+    project one level (part_l[u] = part_{l+1}[CM_l[u]]) then refine on that level's fine
+    graph.  Returns (part of level 0, total moves)."""
+    part = np.asarray(part_coarse, dtype=np.int32)
+    total = 0
+    for l in range(len(levels) - 1, -1, -1):
+        part = project(levels, part, from_level=l, to_level=l)
+        fine = g0 if l == 0 else levels[l - 1]["coarse"]
+        part, mv, _ = refine(fine, part, nparts, imbalance_pct, max_passes)
+        total += mv
+    return part, total
 
 
 def project(levels: List[Dict], part_coarse, from_level: Optional[int] = None, to_level: int = 0) -> np.ndarray:

@@ -249,3 +249,127 @@ int64_t oracle_contract(int32_t n, const int32_t *adjp, const int32_t *adjncy,
     free(buf);
     return cnnz;
 }
+
+/*
+ * Refinement of un-coarsening (P22.s1-22), written out step by step; reading R18 of
+ * DESIGN.md §2 fixes what the paper leaves open (gains from the labels at the start of an
+ * iteration, ties to the lower partition id, requests explored in (gain desc, vertex asc)
+ * order, the integer balance bounds).
+ *
+ *   W = sum vwgt;  max_w = ceil(W (100 + imb) / (100 k));  min_w = floor(W (100 - imb) / (100 k))
+ *   (3 % imbalance in the paper's experiments, P22.s35).
+ *   pass = two iterations, dir = 0 (moves to a HIGHER partition id only) then dir = 1 (to a
+ *   LOWER one): the ordering method that forbids concurrent exchanges between two
+ *   neighbouring partitions (P22.s8-10).  One iteration:
+ *     request  (first kernel, P22.s4-7): every boundary vertex v (a neighbour in another
+ *              partition) of partition s takes the destination d of its neighbours' partitions,
+ *              in the iteration's direction, with the largest gain
+ *                 gain(d) = w(v, d) - w(v, s)      (w(v, X) = sum of v's edge weights into X)
+ *              if gain > 0 ("maximum reduction of the edge cut"; ties: lower d), the source
+ *              stays >= min_w without v and the destination stays <= max_w with v
+ *              ("does not underweight the source or overweight the destination").  The
+ *              request (v, gain) goes to d's buffer (P22.s11-15).
+ *     explore  (P22.s16-19): per destination d, its requests sorted by gain (descending;
+ *              equal gains: lower vertex id first) are accepted in that order while
+ *              pw[d] + vwgt[v] <= max_w, pw[d] growing with every accepted move.
+ *     apply:   the accepted vertices change partition (all at once).
+ *   A pass that moves nothing ends the refinement early (P22.s20-21); at most max_passes.
+ * part[] is updated in place.  Returns 0, or -1 on a bad argument.
+ */
+typedef struct { int32_t v; int32_t gain; } oracle_req;
+
+static int oracle_req_cmp(const void *a, const void *b)
+{
+    const oracle_req *x = (const oracle_req *)a, *y = (const oracle_req *)b;
+    if (x->gain != y->gain) return x->gain > y->gain ? -1 : 1;   /* gain descending */
+    return (x->v > y->v) - (x->v < y->v);                          /* then vertex id  */
+}
+
+int oracle_refine(int32_t n, const int32_t *adjp, const int32_t *adjncy, const int32_t *adjwgt,
+                  const int32_t *vwgt, int32_t k, int32_t imbalance_pct, int32_t max_passes,
+                  int32_t *part, int32_t *moves_out, int32_t *passes_out)
+{
+    int64_t W = 0, maxw, minw, *pw, *conn;
+    int32_t *dest, *gainv, v, pass, moves = 0, passes = 0;
+    oracle_req *req;
+    if (k < 1 || imbalance_pct < 0 || max_passes < 0) return -1;
+    for (v = 0; v < n; ++v) {
+        if (part[v] < 0 || part[v] >= k) return -1;
+        W += vwgt[v];
+    }
+    maxw = (W * (100 + imbalance_pct) + 100LL * k - 1) / (100LL * k);
+    minw = (W * (100 - imbalance_pct)) / (100LL * k);
+    pw = (int64_t *)calloc((size_t)k, sizeof(int64_t));
+    conn = (int64_t *)calloc((size_t)k, sizeof(int64_t));
+    dest = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+    gainv = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+    req = (oracle_req *)malloc(sizeof(oracle_req) * (size_t)(n > 0 ? n : 1));
+    for (v = 0; v < n; ++v) pw[part[v]] += vwgt[v];
+
+    for (pass = 0; pass < max_passes; ++pass) {
+        int32_t pass_moves = 0, dir;
+        for (dir = 0; dir < 2; ++dir) {
+            int32_t d, j;
+            /* request */
+            for (v = 0; v < n; ++v) {
+                int32_t s = part[v], boundary = 0, best = -1;
+                int64_t bestgain = 0;
+                dest[v] = -1;
+                for (j = adjp[v]; j < adjp[v + 1]; ++j) {
+                    int32_t p = part[adjncy[j]];
+                    conn[p] += adjwgt[j];
+                    if (p != s) boundary = 1;
+                }
+                if (boundary) {
+                    for (j = adjp[v]; j < adjp[v + 1]; ++j) {
+                        int64_t g;
+                        d = part[adjncy[j]];
+                        if (d == s || (dir == 0 ? d < s : d > s)) continue;
+                        g = conn[d] - conn[s];
+                        if (g > 0 && (best < 0 || g > bestgain || (g == bestgain && d < best))) {
+                            best = d;
+                            bestgain = g;
+                        }
+                    }
+                    if (best >= 0 && pw[s] - vwgt[v] >= minw && pw[best] + vwgt[v] <= maxw) {
+                        dest[v] = best;
+                        gainv[v] = (int32_t)bestgain;
+                    }
+                }
+                for (j = adjp[v]; j < adjp[v + 1]; ++j) conn[part[adjncy[j]]] = 0;
+            }
+            /* explore, one destination partition at a time */
+            for (d = 0; d < k; ++d) {
+                int32_t m = 0, i;
+                int64_t cur = pw[d];
+                for (v = 0; v < n; ++v)
+                    if (dest[v] == d) { req[m].v = v; req[m].gain = gainv[v]; ++m; }
+                qsort(req, (size_t)m, sizeof(oracle_req), oracle_req_cmp);
+                for (i = 0; i < m; ++i) {
+                    int32_t u = req[i].v;
+                    if (cur + vwgt[u] <= maxw) cur += vwgt[u];
+                    else dest[u] = -1;                       /* rejected */
+                }
+            }
+            /* apply */
+            for (v = 0; v < n; ++v)
+                if (dest[v] >= 0) {
+                    pw[part[v]] -= vwgt[v];
+                    pw[dest[v]] += vwgt[v];
+                    part[v] = dest[v];
+                    ++pass_moves;
+                }
+        }
+        moves += pass_moves;
+        ++passes;
+        if (pass_moves == 0) break;
+    }
+    free(pw);
+    free(conn);
+    free(dest);
+    free(gainv);
+    free(req);
+    if (moves_out) *moves_out = moves;
+    if (passes_out) *passes_out = passes;
+    return 0;
+}

@@ -34,6 +34,7 @@
 
 #include "device_util.cuh"
 #include "gp_internal.cuh"
+#include "merge_util.cuh"
 
 namespace gp {
 
@@ -75,7 +76,12 @@ struct ContractArgs {
     // host takes the stop decision.  Single GPU: dist = 0, cbase = 0.
     int32_t dist, cbase, tb_fixed, nnz_ub;
     int32_t prof;    // GP_PROF=1: slowest C2a warp tile (ctl->dbg)
+    // single-pass coarse CSR assembly (single GPU): decoupled look-back over the C2 warp tiles
+    unsigned long long *status;  // one status word per tile (ctx->status; epoch-tagged, never reset)
+    uint32_t epoch;
+    int32_t knobs;  // bit 0: route 65..kWB rows of small levels to C1h (GP_C1H_SMALL=1); bit 1: two-pass only (GP_C2_SP=0)
 };
+__device__ __forceinline__ bool small_hub_on(const ContractArgs &a) { return a.knobs & 1; }
 
 struct ContractSmem {
     unsigned long long buf[kBuf];
@@ -97,87 +103,6 @@ __device__ __forceinline__ void cswap(unsigned long long &a, unsigned long long 
     const unsigned long long lo = a < b ? a : b, hi = a < b ? b : a;
     a = lo;
     b = hi;
-}
-
-// Batcher odd-even merge sort network for 16 inputs (63 comparators; generated and checked
-// against sorted() offline).
-// sort (cx, w) pairs by cx only: equal coarse ids are summed afterwards, so their order is
-// irrelevant; a comparator is one 32-bit compare and four selects
-__device__ __forceinline__ void cx_sort16(uint32_t (&cx)[16], int32_t (&w)[16]) {
-#define GP_CE(i, j)                                                      \
-    {                                                                    \
-        const bool sw = cx[i] > cx[j];                                   \
-        const uint32_t c0 = sw ? cx[j] : cx[i], c1 = sw ? cx[i] : cx[j]; \
-        const int32_t w0 = sw ? w[j] : w[i], w1 = sw ? w[i] : w[j];      \
-        cx[i] = c0;                                                      \
-        cx[j] = c1;                                                      \
-        w[i] = w0;                                                       \
-        w[j] = w1;                                                       \
-    }
-    GP_CE(0, 1)
-    GP_CE(2, 3)
-    GP_CE(0, 2)
-    GP_CE(1, 3)
-    GP_CE(1, 2)
-    GP_CE(4, 5)
-    GP_CE(6, 7)
-    GP_CE(4, 6)
-    GP_CE(5, 7)
-    GP_CE(5, 6)
-    GP_CE(0, 4)
-    GP_CE(2, 6)
-    GP_CE(2, 4)
-    GP_CE(1, 5)
-    GP_CE(3, 7)
-    GP_CE(3, 5)
-    GP_CE(1, 2)
-    GP_CE(3, 4)
-    GP_CE(5, 6)
-    GP_CE(8, 9)
-    GP_CE(10, 11)
-    GP_CE(8, 10)
-    GP_CE(9, 11)
-    GP_CE(9, 10)
-    GP_CE(12, 13)
-    GP_CE(14, 15)
-    GP_CE(12, 14)
-    GP_CE(13, 15)
-    GP_CE(13, 14)
-    GP_CE(8, 12)
-    GP_CE(10, 14)
-    GP_CE(10, 12)
-    GP_CE(9, 13)
-    GP_CE(11, 15)
-    GP_CE(11, 13)
-    GP_CE(9, 10)
-    GP_CE(11, 12)
-    GP_CE(13, 14)
-    GP_CE(0, 8)
-    GP_CE(4, 12)
-    GP_CE(4, 8)
-    GP_CE(2, 10)
-    GP_CE(6, 14)
-    GP_CE(6, 10)
-    GP_CE(2, 4)
-    GP_CE(6, 8)
-    GP_CE(10, 12)
-    GP_CE(1, 9)
-    GP_CE(5, 13)
-    GP_CE(5, 9)
-    GP_CE(3, 11)
-    GP_CE(7, 15)
-    GP_CE(7, 11)
-    GP_CE(3, 5)
-    GP_CE(7, 9)
-    GP_CE(11, 13)
-    GP_CE(1, 2)
-    GP_CE(3, 4)
-    GP_CE(5, 6)
-    GP_CE(7, 8)
-    GP_CE(9, 10)
-    GP_CE(11, 12)
-    GP_CE(13, 14)
-#undef GP_CE
 }
 
 // ascending bitonic network on N registers (flip formulation: all comparators ascending)
@@ -542,7 +467,7 @@ __device__ void phase_c1a(const ContractArgs &a, int32_t n, int nt1, int T1) {
 // ---------------------------------------------------------------------------------------
 // C1b: CM, cvwgt, off, seg, C2 warp-tile starts, huge rows
 // ---------------------------------------------------------------------------------------
-__device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, int nt1, int T1) {
+__device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, int nt1, int T1, int32_t hub_ub) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int t_lo = blockIdx.x * T1, t_hi = min(nt1, t_lo + T1);
     if (t_lo >= t_hi) return;
@@ -601,7 +526,7 @@ __device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, in
                 a.cvwgt[cc] = vw[i];
                 a.off[cc] = oo;
                 a.seg[cc] = make_int4(su[i], dl, sv[i], d - dl);
-                if (d > kWB) a.huge[atomicAdd(&a.ctl->n_huge, 1)] = cc;
+                if (d > hub_ub) a.huge[atomicAdd(&a.ctl->n_huge, 1)] = cc;
             }
             c += __popc(bl);
             o += dtot;
@@ -843,7 +768,8 @@ __device__ __noinline__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, 
 // ---------------------------------------------------------------------------------------
 // C2a: warp tiles: merge every row, write the tile compacted to tout at its ub offset
 // ---------------------------------------------------------------------------------------
-__device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntiles2, int T2, int32_t nc, int32_t rt) {
+__device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntiles2, int T2, int32_t nc, int32_t rt,
+                          bool single_pass, int32_t hub_ub) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int gw = blockIdx.x * kCW + wib, nw = g_cact * kCW;
     unsigned long long *wb = sm.buf + wib * 2 * kWB;  // this warp's slots (2*kWB entries)
@@ -867,6 +793,14 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
         }
         unsigned long long *out = a.tout + (r0 < r1 ? __ldcg(a.off + r0) : 0);
         int32_t run = 0;
+        // single-pass assembly (single GPU): a tile whose rows merge in ONE pass keeps them in
+        // its slot area (C1h rows stay in gkeys) until its look-back prefix is known, then
+        // writes them straight into cadjncy / cadjwgt; a multi-pass tile stages its passes in
+        // tout (the slot area is reused) and copies them out after the look-back.
+        const bool sp1 = single_pass;
+        bool spilled = false;                      // an earlier pass of this tile went to tout
+        int32_t myoff = INT32_MAX, myslot = 0;     // this lane's row: offset in the tile, slot
+        bool myhub = false;                        // ... merged by C1h (keys in gkeys)
         for (int32_t g0 = r0; g0 < r1; g0 += 32) {
             const int32_t c = g0 + lane;
             int32_t ub = 0, hcnt = 0;
@@ -875,21 +809,21 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
                 const int32_t o0 = __ldcg(a.off + c);
                 ub = __ldcg(a.off + c + 1) - o0;
                 if (ub <= kWarpNet) sg = __ldcg(a.seg + c);
-                if (ub > kWB) hcnt = __ldcg(a.cnt + c);  // merged by C1h
+                if (ub > hub_ub) hcnt = __ldcg(a.cnt + c);  // merged by C1h
             }
             // Passes over the 32 rows: a pass takes the next lanes whose slots (ub of rows
             // <= kWB; C1h rows take none) fit the warp's 2kWB slot area -- one pass unless the
             // rows are long.  The first lane of a pass always fits (ub <= kWB).
             for (int32_t first = 0;;) {
             const bool inr = c < r1 && lane >= first;
-            const int32_t used = warp_incl_scan((inr && ub <= kWB) ? ub : 0);  // all lanes: a shuffle scan
+            const int32_t used = warp_incl_scan((inr && ub <= hub_ub) ? ub : 0);  // all lanes: a shuffle scan
             const bool act = inr && used <= 2 * kWB;
             const unsigned pm = __ballot_sync(0xffffffffu, act);
-            int32_t cntc = (act && ub > kWB) ? hcnt : 0;
+            int32_t cntc = (act && ub > hub_ub) ? hcnt : 0;
             // Positions in the slot area: rows with ub <= 64 (staged) packed first, rows of
             // 65..kWB entries after them.
             const bool srow = act && ub <= kWarpNet;
-            const bool mrow = act && ub > kWarpNet && ub <= kWB;
+            const bool mrow = act && ub > kWarpNet && ub <= hub_ub;
             int32_t S, Mt;
             const int32_t sp = warp_excl(srow ? ub : 0, S);
             const int32_t sq = S + warp_excl(mrow ? ub : 0, Mt);
@@ -1055,13 +989,22 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
             }
             int32_t part;
             const int32_t ex = warp_excl(cntc, part);
+            const bool last_pass = first + __popc(pm) >= 32 || g0 + first + __popc(pm) >= r1;
+            const bool keep = sp1 && last_pass && !spilled && g0 + 32 >= r1;  // whole tile in one pass
             if (act) {
-                a.lofs[c] = run + ex;
-                if (ub <= kWB)
+                if (sp1) {
+                    myoff = run + ex;
+                    myslot = slot;
+                    myhub = ub > hub_ub;
+                } else {
+                    a.lofs[c] = run + ex;
+                }
+                if (ub <= hub_ub && !keep)
                     for (int32_t j = 0; j < cntc; ++j) __stcs(out + run + ex + j, wb[slot + j]);
             }
+            if (!keep) spilled = true;
             // rows merged by C1h: the warp copies them in
-            unsigned mh = __ballot_sync(0xffffffffu, act && ub > kWB);
+            unsigned mh = keep ? 0u : __ballot_sync(0xffffffffu, act && ub > hub_ub);
             while (mh) {
                 const int src = __ffs(mh) - 1;
                 mh &= mh - 1;
@@ -1098,9 +1041,63 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
             atomicAdd(&a.ctl->dbg[4], 1ull);
             atomicAdd(&a.ctl->dbg[5], (unsigned long long)nw64);
         }
+        if (sp1) {
+            // decoupled look-back over the tiles in claim order (every earlier tile is already
+            // claimed by a running warp, so the chain always completes)
+            const int32_t prefix = lookback_prefix(a.status, a.epoch, wt, run);
+            const int32_t c = r0 + lane;
+            if (c < r1) a.cadjp[c] = prefix + myoff;  // (R11)
+            if (wt == ntiles2 - 1 && lane == 0) {
+                a.cadjp[nc] = prefix + run;
+                a.ctl->cnnz = prefix + run;
+            }
+            if (!spilled) {
+                // the tile's rows from the slot area / gkeys, coalesced: entry e belongs to the
+                // last row whose offset is <= e (binary search over the lanes' offsets)
+                const int32_t hbase = (c < r1 && myhub) ? __ldcg(a.off + c) : 0;
+                for (int32_t e = lane; e - lane < run; e += 32) {
+                    int r = 0;
+#pragma unroll
+                    for (int step = 16; step > 0; step >>= 1) {
+                        const int32_t o = __shfl_sync(0xffffffffu, myoff, r + step);
+                        if (o <= e) r += step;
+                    }
+                    const int32_t j = e - __shfl_sync(0xffffffffu, myoff, r);
+                    const int32_t sl = __shfl_sync(0xffffffffu, myslot, r);
+                    const bool hub = __shfl_sync(0xffffffffu, myhub ? 1 : 0, r) != 0;
+                    const int32_t hb = __shfl_sync(0xffffffffu, hbase, r);
+                    if (e < run) {
+                        const unsigned long long kv = hub ? __ldcg(a.gkeys + hb + j) : wb[sl + j];
+                        a.cadjncy[prefix + e] = (int32_t)(kv >> 32);
+                        a.cadjwgt[prefix + e] = (int32_t)(uint32_t)kv;
+                    }
+                }
+            } else {
+                __syncwarp();
+                for (int32_t j0 = 0; j0 < run; j0 += 32 * 8) {  // staged passes: tout -> final
+                    unsigned long long kk[8];
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) {
+                        const int32_t j = j0 + q * 32 + lane;
+                        kk[q] = j < run ? __ldcg(out + j) : 0ull;
+                    }
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) {
+                        const int32_t j = j0 + q * 32 + lane;
+                        if (j < run) {
+                            a.cadjncy[prefix + j] = (int32_t)(kk[q] >> 32);
+                            a.cadjwgt[prefix + j] = (int32_t)(uint32_t)kk[q];
+                        }
+                    }
+                }
+            }
+            __syncwarp();  // the slot area is rebuilt by the next tile
+        }
         if (lane == 0) {
-            a.ttot[wt] = run;
-            atomicAdd(&a.ctl->chunk2[wt / T2], run);
+            if (!sp1) {
+                a.ttot[wt] = run;
+                atomicAdd(&a.ctl->chunk2[wt / T2], run);
+            }
             wt = nw + (int)atomicAdd(&a.ctl->tile_ctr, 1u);
         }
     }
@@ -1238,6 +1235,12 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
     }
     unsigned bar_epoch = 0;  // grid barriers passed (thread 0)
     const int nt1 = (n + kVW - 1) / kVW;
+    // Rows merged by one CTA each (C1h): ub > kWB.  GP_C1H_SMALL=1 also routes the 65..kWB rows
+    // of small levels (about one C2 tile per warp) to C1h -- measured slower on C3 (C1h took
+    // ~20 us at L10/L11 for a few rows per CTA), so off by default.  Sharded levels keep kWB
+    // (dist.cu builds their C1h list).
+    const int32_t hub_ub =
+        (a.dist || (long long)n > 32LL * 2 * g_cact * kCW || !small_hub_on(a)) ? kWB : kWarpNet;
     const int T1 = (nt1 + g_cact - 1) / g_cact;            // C1b tiles per CTA
     trace_mark(ctl->trace, 0);
     if (n > 0 && !a.dist) {
@@ -1245,7 +1248,7 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
         trace_mark(ctl->trace, 1);
         grid_barrier(ctl->bar, bar_epoch, g_cact);
         trace_mark(ctl->trace, 2);
-        phase_c1b(a, sm, n, nt1, T1);
+        phase_c1b(a, sm, n, nt1, T1, hub_ub);
         trace_mark(ctl->trace, 3);
         grid_barrier(ctl->bar, bar_epoch, g_cact);
     }
@@ -1265,11 +1268,19 @@ __global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constan
     const int32_t ntiles2 = nnz <= 0 ? 0 : a.dist ? (nnz + a.tb_fixed - 1) / a.tb_fixed : (nc + rt - 1) / rt;
     const int T2 = (ntiles2 + g_cact - 1) / g_cact;  // C2b tiles (and chunk sums) per CTA
     if (ntiles2 > 0) {
-        phase_c2a(a, sm, ntiles2, T2, nc, rt);
+        // Single-pass assembly (decoupled look-back) while the tiles are few: every warp then
+        // has ~1-2 tiles and the look-back chains stay short.  With many more tiles than warps
+        // (C3 levels 0-3) the inclusive prefixes advance ~32 tiles per L2 round trip behind
+        // ~4700 concurrent tiles, which measured slower (L0 C2: 351 us vs 242 us) than the
+        // two-pass assembly (tile totals, one grid barrier, C2b copy).  Sharded levels: two-pass.
+        const bool single_pass = !a.dist && !(a.knobs & 2) && ntiles2 <= 2 * g_cact * kCW;
+        phase_c2a(a, sm, ntiles2, T2, nc, rt, single_pass, hub_ub);
         trace_mark(ctl->trace, 6);
-        grid_barrier(ctl->bar, bar_epoch, g_cact);
-        trace_mark(ctl->trace, 7);
-        phase_c2b(a, sm, nc, ntiles2, T2, rt);
+        if (!single_pass) {
+            grid_barrier(ctl->bar, bar_epoch, g_cact);
+            trace_mark(ctl->trace, 7);
+            phase_c2b(a, sm, nc, ntiles2, T2, rt);
+        }
     } else {  // no arcs: every coarse row is empty
         for (long long c = (long long)blockIdx.x * kCNT + threadIdx.x; c <= nc; c += (long long)g_cact * kCNT)
             a.cadjp[c] = 0;
@@ -1322,8 +1333,11 @@ static int32_t contract_vpc() {
 }
 
 int contract_grid(Ctx *ctx) {
-    static int per_sm = -1;
-    if (per_sm < 0) {
+    // per device: cudaFuncSetAttribute applies to the current device (the ctx's, DeviceGuard)
+    static int per_sm_dev[kMaxDevices] = {0};
+    int dummy = -1;
+    int &per_sm = (ctx->device >= 0 && ctx->device < kMaxDevices) ? per_sm_dev[ctx->device] : dummy;
+    if (per_sm <= 0) {
         int b = 0;
         cudaFuncSetAttribute(k_contract_level, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)sizeof(ContractSmem) + 128);
@@ -1376,6 +1390,20 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
     a.cbase = prm.cbase;
     a.tb_fixed = prm.tb;
     a.nnz_ub = prm.nnz_ub;
+    a.status = nullptr;
+    a.epoch = 0;
+    {
+        const char *e1 = getenv("GP_C1H_SMALL"), *e2 = getenv("GP_C2_SP");  // tuning knobs (results never depend on them)
+        a.knobs = ((e1 && atoi(e1) == 1) ? 1 : 0) | ((e2 && atoi(e2) == 0) ? 2 : 0);
+    }
+    if (!prm.dist) {
+        const size_t tiles = ((size_t)(prm.n_bound > 0 ? prm.n_bound : 1) + kRT - 1) / kRT + 1;
+        gp_status st = ensure_status(ctx, tiles);
+        if (st != GP_OK) return st;
+        a.status = ctx->status;
+        a.epoch = ctx->epoch++ & 0x3FFFFFFFu;  // 30-bit tag (lookback_prefix)
+        if (a.epoch == 0) a.epoch = ctx->epoch++ & 0x3FFFFFFFu;
+    }
     {
         static int pf = -1;
         if (pf < 0) {

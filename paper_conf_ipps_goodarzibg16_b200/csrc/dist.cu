@@ -626,6 +626,8 @@ gp_status dist_coarsen_to(Graph *g0, const gp_coarsen_opts *opts, Hier **out) {
     const int32_t max_levels = opts->max_levels ? opts->max_levels : 64;
     Hier *h = new Hier();
     h->ctx = ctx;
+    h->counted = true;
+    ++ctx->live_objects;
     *out = nullptr;
     std::vector<Shard> shards;
     gp_status st = GP_OK;
@@ -662,6 +664,7 @@ gp_status dist_coarsen_to(Graph *g0, const gp_coarsen_opts *opts, Hier **out) {
     std::vector<RankWork> W;
     // results of one level (set by run_level)
     int32_t rounds = 0, maximal = 0, NC = 0;
+    int32_t prev_rounds = 7;  // round count of the previous level (first batch size of the next)
     long long CNNZ = 0;
     int64_t stat_arcs = 0, stat_rows = 0, stat_visits = 0;
     std::vector<int32_t> cranges;
@@ -769,42 +772,62 @@ gp_status dist_coarsen_to(Graph *g0, const gp_coarsen_opts *opts, Hier **out) {
         if (st == GP_OK) st = unpack_match(1);
         rounds = 0;
         maximal = 0;
-        for (int k = 1; st == GP_OK; ++k) {
+        // Rounds are enqueued in batches with ONE host synchronisation per batch: after the
+        // fixpoint a round is a no-op (empty live lists, unchanged boundary records), so the
+        // rounds of a batch beyond the last live one change nothing; every round's gathered
+        // header {live, made} is copied to its own pinned slot and the batch is evaluated in
+        // order (rounds that made a match are counted, R4).  With a max_rounds cap the batch
+        // is 1 (a round past the cap would change the result).  The batch grows geometrically
+        // from the previous level's round count.
+        int batch = opts->max_rounds > 0 ? 1 : std::max(2, std::min(16, prev_rounds + 1));
+        bool done = false;
+        for (int k = 1; st == GP_OK && !done;) {
             if (k > N + 2) {
                 set_error("dist: round loop did not terminate (protocol bug)");
                 st = GP_ERR_INTERNAL;
                 break;
             }
-            for (int i = 0; i < NL && st == GP_OK; ++i) {
-                RankWork &w = W[i];
-                GP_CUDA(cudaMemsetAsync(w.ld->match.bar, 0, sizeof(w.ld->match.bar), ctx->stream));
-                st = enqueue_match(ctx, bufs_of(w), w.M, &w.ld->match, opts->max_rounds, true, ad, w.vbase,
-                                   kMatchRound, k);
+            const int kb = std::max(1, std::min(batch, 1024 / (2 * G)));  // header slots in the 4 KiB pinned buffer
+            for (int b = 0; b < kb && st == GP_OK; ++b) {
+                const int kk = k + b;
+                for (int i = 0; i < NL && st == GP_OK; ++i) {
+                    RankWork &w = W[i];
+                    GP_CUDA(cudaMemsetAsync(w.ld->match.bar, 0, sizeof(w.ld->match.bar), ctx->stream));
+                    st = enqueue_match(ctx, bufs_of(w), w.M, &w.ld->match, opts->max_rounds, true, ad, w.vbase,
+                                       kMatchRound, kk);
+                    if (st == GP_OK)
+                        GP_LAUNCH(k_pack_match<<<grid_for(w.nb), kDT, 0, ctx->stream>>>(
+                            w.B, w.nb, w.P[(kk + 1) & 1], w.vbase, w.nloc, &w.ld->match.slot[(kk + 1) & 3].live, 0,
+                            &w.ld->match.slot[kk & 3].matches, w.rs));
+                }
+                if (st == GP_OK) st = allgather(ctx, vs, vr, (size_t)RS);
+                if (st == GP_OK) st = unpack_match((kk + 1) & 1);
+                // every rank's header {live, made} of round kk (all in the first local receive buffer)
                 if (st == GP_OK)
-                    GP_LAUNCH(k_pack_match<<<grid_for(w.nb), kDT, 0, ctx->stream>>>(
-                        w.B, w.nb, w.P[(k + 1) & 1], w.vbase, w.nloc, &w.ld->match.slot[(k + 1) & 3].live, 0,
-                        &w.ld->match.slot[k & 3].matches, w.rs));
+                    GP_CUDA(cudaMemcpy2DAsync(pin + (size_t)b * 2 * G, 2 * sizeof(int32_t), W[0].rr, RS * sizeof(int32_t),
+                                              2 * sizeof(int32_t), G, cudaMemcpyDeviceToHost, ctx->stream));
             }
-            if (st == GP_OK) st = allgather(ctx, vs, vr, (size_t)RS);
-            if (st == GP_OK) st = unpack_match((k + 1) & 1);
             if (st != GP_OK) break;
-            // every rank's header {live, made} (all in the first local receive buffer)
-            GP_CUDA(cudaMemcpy2DAsync(pin, 4 * sizeof(int32_t), W[0].rr, RS * sizeof(int32_t), 2 * sizeof(int32_t), G,
-                                      cudaMemcpyDeviceToHost, ctx->stream));
             GP_CUDA(cudaStreamSynchronize(ctx->stream));
-            long long live = 0;
-            bool made = false;
-            for (int s = 0; s < G; ++s) {
-                live += pin[4 * s];
-                made = made || pin[4 * s + 1] != 0;
+            for (int b = 0; b < kb && !done; ++b) {
+                long long live = 0;
+                bool made = false;
+                for (int s = 0; s < G; ++s) {
+                    live += pin[(size_t)b * 2 * G + 2 * s];
+                    made = made || pin[(size_t)b * 2 * G + 2 * s + 1] != 0;
+                }
+                if (made) ++rounds;
+                if (live == 0) {
+                    maximal = 1;
+                    done = true;
+                } else if (opts->max_rounds > 0 && rounds >= opts->max_rounds) {
+                    done = true;
+                }
             }
-            if (made) ++rounds;
-            if (live == 0) {
-                maximal = 1;
-                break;
-            }
-            if (opts->max_rounds > 0 && rounds >= opts->max_rounds) break;
+            k += kb;
+            if (opts->max_rounds == 0) batch = std::min(2 * batch, 64);
         }
+        prev_rounds = rounds;
         for (int i = 0; i < NL && st == GP_OK; ++i)  // leftover pass (P18.s12-13)
             st = enqueue_match(ctx, bufs_of(W[i]), W[i].M, &W[i].ld->match, opts->max_rounds, true, ad, W[i].vbase,
                                kMatchFinish);

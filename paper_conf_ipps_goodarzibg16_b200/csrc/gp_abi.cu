@@ -122,10 +122,12 @@ static void drain_events(Ctx *ctx) {
 void graph_release(Graph *g) {
     if (!g) return;
     Ctx *ctx = g->ctx;
-    dev_free(ctx, g->adjp);
-    dev_free(ctx, g->adjncy);
-    dev_free(ctx, g->adjwgt);
-    dev_free(ctx, g->vwgt);
+    if (!g->arena) {
+        dev_free(ctx, g->adjp);
+        dev_free(ctx, g->adjncy);
+        dev_free(ctx, g->adjwgt);
+        dev_free(ctx, g->vwgt);
+    }
     if (g->owns_sizes) dev_free(ctx, g->sizes);
     if (g->counted) --ctx->live_objects;
     g->tag = 0;
@@ -135,8 +137,10 @@ void graph_release(Graph *g) {
 void hier_release(Hier *h) {
     if (!h) return;
     for (auto &l : h->levels) {
-        dev_free(h->ctx, l.match);
-        dev_free(h->ctx, l.cmap);
+        if (!l.arena) {
+            dev_free(h->ctx, l.match);
+            dev_free(h->ctx, l.cmap);
+        }
         graph_release(l.coarse);
         for (auto &p : l.pieces) {
             dev_free(h->ctx, p.M);
@@ -145,6 +149,7 @@ void hier_release(Hier *h) {
         }
     }
     dev_free(h->ctx, h->levdev);
+    for (void *p : h->arenas) dev_free(h->ctx, p);
     if (h->counted) --h->ctx->live_objects;
     h->tag = 0;
     delete h;
@@ -644,10 +649,82 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
                                 &ctx->reports_dev[l], prm);
     };
 
+    // Coarse-level tail (small.cu): once the level bounds fit one SM's
+    // shared memory, ONE launch of one CTA runs every remaining level.  The host creates the
+    // levels up front (arrays in one arena slot per level) and reads their reports as usual.
+    std::vector<std::vector<unsigned char>> keep_host;
+    auto enqueue_tail = [&](int l0) -> gp_status {
+        const int32_t n_b = tight_n, m_b = tight_m;
+        const int ns = max_levels - l0;
+        const size_t slot = small_slot_ints(n_b, m_b);
+        void *arena = nullptr, *desc = nullptr;
+        gp_status s2 = dev_alloc(ctx, &arena, sizeof(int32_t) * slot * (size_t)ns);
+        if (s2 == GP_OK) h->arenas.push_back(arena);
+        if (s2 == GP_OK) s2 = dev_alloc(ctx, &desc, small_slot_desc_bytes() * (size_t)ns);
+        if (s2 == GP_OK) h->arenas.push_back(desc);
+        if (s2 != GP_OK) return s2;
+        std::vector<unsigned char> hd((size_t)ns * small_slot_desc_bytes());
+        for (int i = 0; i < ns; ++i) {
+            int32_t *base = static_cast<int32_t *>(arena) + slot * (size_t)i;
+            small_slot_carve(base, n_b, m_b, hd.data() + (size_t)i * small_slot_desc_bytes());
+            struct D { int32_t *M, *CM, *cadjp, *cadjncy, *cadjwgt, *cvwgt; };
+            const D *d = reinterpret_cast<const D *>(hd.data() + (size_t)i * small_slot_desc_bytes());
+            Level L;
+            L.n = n_b;
+            L.nnz = m_b;
+            L.arena = true;
+            L.match = d->M;
+            L.cmap = d->CM;
+            Graph *cg = new Graph();
+            cg->ctx = ctx;
+            cg->borrowed = true;
+            cg->arena = true;
+            cg->owns_sizes = false;
+            cg->adjp = d->cadjp;
+            cg->adjncy = d->cadjncy;
+            cg->adjwgt = d->cadjwgt;
+            cg->vwgt = d->cvwgt;
+            cg->sizes = &h->levdev[l0 + i].out;
+            cg->counted = true;
+            ++ctx->live_objects;
+            L.coarse = cg;
+            lv.push_back(L);
+        }
+        // the descriptors are small: a pinned staging copy is not needed (synchronous copy)
+        GP_CUDA(cudaMemcpyAsync(desc, hd.data(), hd.size(), cudaMemcpyHostToDevice, ctx->stream));
+        const Graph *in = (l0 == 0) ? g : lv[l0 - 1].coarse;
+        SmallLaunch sl;
+        sl.in = (l0 == 0) ? in0 : in->sizes;
+        sl.adjp = in->adjp;
+        sl.adjncy = in->adjncy;
+        sl.adjwgt = in->adjwgt;
+        sl.vwgt = in->vwgt;
+        sl.slots = desc;
+        sl.nslots = ns;
+        sl.level0 = l0;
+        sl.cap_n = n_b;
+        sl.cap_nnz = m_b;
+        sl.levdev = h->levdev;
+        sl.reports = ctx->reports_dev;
+        sl.threshold = opts->threshold;
+        sl.stall_pct = pct;
+        sl.max_levels = max_levels;
+        sl.max_rounds = opts->max_rounds;
+        s2 = enqueue_small(ctx, sl);
+        keep_host.push_back(std::move(hd));  // read by the async copy: alive until the final sync
+        return s2;
+    };
+
     int enq = 0, obs = 0, last_real = -1;
     bool stop_seen = false;
     while (st == GP_OK) {
         while (st == GP_OK && !stop_seen && enq < max_levels && enq - obs < kAhead) {
+            if (small_use(tight_n, tight_m)) {
+                GP_DBG("enqueue tail levels %d.. in one CTA (bounds n=%d nnz=%d)\n", enq, tight_n, tight_m);
+                st = enqueue_tail(enq);
+                enq = max_levels;
+                break;
+            }
             GP_DBG("enqueue level %d (bounds n=%d nnz=%d)\n", enq, tight_n, tight_m);
             st = enqueue_level(enq);
             ++enq;
@@ -751,8 +828,10 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
         if (st == GP_OK && l <= last_real) {
             h->levels.push_back(lv[l]);
         } else {
-            dev_free(ctx, lv[l].match);
-            dev_free(ctx, lv[l].cmap);
+            if (!lv[l].arena) {
+                dev_free(ctx, lv[l].match);
+                dev_free(ctx, lv[l].cmap);
+            }
             graph_release(lv[l].coarse);
         }
     }
@@ -908,6 +987,66 @@ gp_status gp_project(gp_hier h, int32_t from_level, int32_t to_level, const gp_v
         cms.push_back(h->levels[l].cmap);
     }
     return enqueue_project(h->ctx, cms.data(), (int)cms.size(), h->levels[to_level].n, d_part_coarse, d_part_fine);
+    GP_TRY_END
+}
+
+gp_status gp_refine(gp_graph g, gp_vid *d_part, const gp_refine_opts *opts, int32_t *moves_out, int32_t *passes_out) {
+    if (!tagged<Graph>(g, kTagGraph) || !opts || (!d_part && g->n > 0)) {
+        set_error("gp_refine: bad graph, labels or options");
+        return GP_ERR_INVALID_ARG;
+    }
+    GP_TRY_BEGIN
+    Ctx *ctx = g->ctx;
+    DeviceGuard dg(ctx->device);
+    if (ctx->comm || g->dist) {
+        set_error("gp_refine: single-GPU graphs only");
+        return GP_ERR_INVALID_ARG;
+    }
+    return refine_graph(ctx, g, d_part, *opts, moves_out, passes_out);
+    GP_TRY_END
+}
+
+gp_status gp_uncoarsen(gp_hier h, gp_graph g0, const gp_vid *d_part_coarse, gp_vid *d_part_fine,
+                       const gp_refine_opts *opts, int32_t *moves_out) {
+    if (!tagged<Hier>(h, kTagHier) || !tagged<Graph>(g0, kTagGraph) || !opts || !d_part_coarse || !d_part_fine) {
+        set_error("gp_uncoarsen: bad hierarchy, graph, labels or options");
+        return GP_ERR_INVALID_ARG;
+    }
+    GP_TRY_BEGIN
+    Ctx *ctx = h->ctx;
+    DeviceGuard dg(ctx->device);
+    const int L = (int)h->levels.size();
+    if (L == 0 || g0->n != h->levels[0].n || g0->ctx != ctx) {
+        set_error("gp_uncoarsen: g0 is not the fine graph of this hierarchy's level 0");
+        return GP_ERR_INVALID_ARG;
+    }
+    for (const Level &l : h->levels)
+        if (!l.pieces.empty()) {
+            set_error("gp_uncoarsen: single-GPU hierarchies only");
+            return GP_ERR_INVALID_ARG;
+        }
+    // two label buffers (the coarsest labels are read in place)
+    int32_t *buf[2] = {nullptr, nullptr};
+    gp_status st = dev_alloc(ctx, (void **)&buf[0], sizeof(int32_t) * (size_t)(g0->n + 1));
+    if (st == GP_OK) st = dev_alloc(ctx, (void **)&buf[1], sizeof(int32_t) * (size_t)(g0->n + 1));
+    const int32_t *cur = d_part_coarse;
+    int32_t total = 0;
+    for (int l = L - 1; st == GP_OK && l >= 0; --l) {
+        int32_t *dst = (l == 0) ? d_part_fine : buf[l & 1];
+        const int32_t *cm = h->levels[l].cmap;
+        st = enqueue_project(ctx, &cm, 1, h->levels[l].n, cur, dst);  // P20.s41-P22.s0
+        const Graph *fine = (l == 0) ? g0 : h->levels[l - 1].coarse;
+        int32_t mv = 0;
+        if (st == GP_OK) st = refine_graph(ctx, fine, dst, *opts, &mv, nullptr);  // P22.s1-22
+        total += mv;
+        cur = dst;
+    }
+    cudaError_t e = cudaStreamSynchronize(ctx->stream);
+    dev_free(ctx, buf[0]);
+    dev_free(ctx, buf[1]);
+    if (st == GP_OK && e != cudaSuccess) st = cuda_fail(e, "gp_uncoarsen");
+    if (st == GP_OK && moves_out) *moves_out = total;
+    return st;
     GP_TRY_END
 }
 

@@ -155,6 +155,7 @@ struct gp_graph_s {
     // weight totals measured at creation (R14; the sharded create checks the global sums)
     unsigned long long sum_adjwgt = 0, sum_vwgt = 0;
     bool counted = false;  // included in ctx->live_objects
+    bool arena = false;    // arrays live in a hierarchy arena (small.cu): not freed individually
 };
 
 namespace gp {
@@ -164,6 +165,7 @@ struct Level {
     int32_t *match = nullptr, *cmap = nullptr;
     Graph *coarse = nullptr;
     std::vector<DistPiece> pieces;  // sharded levels: one piece per local rank
+    bool arena = false;             // match / cmap / coarse arrays live in a hierarchy arena
 };
 }  // namespace gp
 
@@ -173,6 +175,7 @@ struct gp_hier_s {
     std::vector<gp::Level> levels;
     gp::LevelDev *levdev = nullptr;  // per-level control blocks (coarse graphs' size records)
     bool counted = false;  // included in ctx->live_objects
+    std::vector<void *> arenas;  // device arenas of tail levels (small.cu), freed with the hierarchy
 };
 
 struct gp_ctx_s {
@@ -295,6 +298,28 @@ struct DeviceGuard {
     DeviceGuard &operator=(const DeviceGuard &) = delete;
 };
 constexpr int kMaxDevices = 64;  // per-device caches of kernel attributes / occupancy
+
+// coarse-level tail in one CTA (small.cu): every remaining level of a graph that fits one SM's
+// shared memory, in one launch
+struct SmallLaunch {
+    const SizeRec *in;
+    const int32_t *adjp, *adjncy, *adjwgt, *vwgt;
+    void *slots;  // device array of per-level output descriptors
+    int32_t nslots, level0, cap_n, cap_nnz;
+    LevelDev *levdev;
+    LevelReport *reports;
+    int32_t threshold, stall_pct, max_levels, max_rounds;
+};
+bool small_fits(int32_t n, int32_t nnz);
+bool small_use(int32_t n_bound, int32_t nnz_bound);
+size_t small_slot_ints(int32_t n, int32_t nnz);
+void small_slot_carve(int32_t *base, int32_t n, int32_t nnz, void *out_slot);
+size_t small_slot_desc_bytes();
+gp_status enqueue_small(Ctx *ctx, const SmallLaunch &L);
+
+// refinement of un-coarsening (refine.cu)
+gp_status refine_graph(Ctx *ctx, const Graph *g, int32_t *d_part, const gp_refine_opts &o, int32_t *moves_out,
+                       int32_t *passes_out);
 
 // projection of un-coarsening (project.cu): cms = CM of levels to..from (fine to coarse)
 gp_status enqueue_project(Ctx *ctx, const int32_t *const *cms, int nlev, int32_t n, const int32_t *part_c,

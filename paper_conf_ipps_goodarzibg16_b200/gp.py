@@ -61,6 +61,10 @@ class Level(ctypes.Structure):
                 ("v_begin", _i32), ("n_local", _i32), ("cv_begin", _i32), ("n_coarse_local", _i32)]
 
 
+class RefineOpts(ctypes.Structure):
+    _fields_ = [("nparts", _i32), ("imbalance_pct", _i32), ("max_passes", _i32)]
+
+
 class KernelStats(ctypes.Structure):
     _fields_ = [("launches", ctypes.c_int64), ("ms", ctypes.c_double)]
 
@@ -94,6 +98,8 @@ _sig("gp_hier_download_level", ctypes.c_int, [_vp, _i32, _vp, _vp])
 _sig("gp_hier_download_coarse", ctypes.c_int, [_vp, _i32, _vp, _vp, _vp, _vp, _i32p, _i32p])
 _sig("gp_nccl_unique_id", ctypes.c_int, [_vp])
 _sig("gp_project", ctypes.c_int, [_vp, _i32, _i32, _vp, _vp])
+_sig("gp_refine", ctypes.c_int, [_vp, _vp, ctypes.POINTER(RefineOpts), _i32p, _i32p])
+_sig("gp_uncoarsen", ctypes.c_int, [_vp, _vp, _vp, _vp, ctypes.POINTER(RefineOpts), _i32p])
 _sig("gp_ctx_create_dist", ctypes.c_int, [ctypes.c_int, _vp, _vp, ctypes.c_int, ctypes.c_int, ctypes.POINTER(_vp)])
 _sig("gp_ctx_create_loopback", ctypes.c_int, [ctypes.c_int, _vp, ctypes.c_int, ctypes.POINTER(_vp)])
 _sig("gp_ctx_dist_info", ctypes.c_int, [_vp, _i32p, _i32p])
@@ -354,6 +360,14 @@ class Graph:
         _check(_lib.gp_contract_level(self._h(), _ptr(match), _ptr(cmap), ctypes.byref(h)), "gp_contract_level")
         return Graph(self.ctx, h)
 
+    def refine(self, part: torch.Tensor, nparts: int, imbalance_pct: int = 3, max_passes: int = 8):
+        """gp_refine: refine the device int32[n] labelling `part` in place (P22.s1-22);
+        returns (moves, passes)."""
+        o = RefineOpts(nparts, imbalance_pct, max_passes)
+        mv, ps = _i32(), _i32()
+        _check(_lib.gp_refine(self._h(), _ptr(part), ctypes.byref(o), ctypes.byref(mv), ctypes.byref(ps)), "gp_refine")
+        return mv.value, ps.value
+
     def coarsen_to(self, threshold: int, stall_ratio_pct: int = 95, max_levels: int = 64,
                    max_rounds: int = 0, tie_seed: int = 0) -> "Hierarchy":
         opts = CoarsenOpts(threshold, stall_ratio_pct, max_levels, max_rounds, tie_seed & 0xFFFFFFFF)
@@ -446,6 +460,16 @@ class Hierarchy:
             from_level = len(self) - 1
         _check(_lib.gp_project(self._h(), from_level, to_level, _ptr(part_coarse), _ptr(part_fine)), "gp_project")
         return part_fine
+
+    def uncoarsen(self, g0: "Graph", part_coarse: torch.Tensor, part_fine: torch.Tensor, nparts: int,
+                  imbalance_pct: int = 3, max_passes: int = 8) -> int:
+        """gp_uncoarsen: project + refine level by level from the coarsest labels to level 0
+        (written into part_fine); returns the total moves."""
+        o = RefineOpts(nparts, imbalance_pct, max_passes)
+        mv = _i32()
+        _check(_lib.gp_uncoarsen(self._h(), g0._h(), _ptr(part_coarse), _ptr(part_fine), ctypes.byref(o),
+                                 ctypes.byref(mv)), "gp_uncoarsen")
+        return mv.value
 
     def download_coarse(self, i: int) -> Dict[str, torch.Tensor]:
         """Coarse graph of level i as host int32 tensors (gp_hier_download_coarse): the whole
