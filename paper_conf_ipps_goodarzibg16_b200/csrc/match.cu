@@ -929,17 +929,30 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
         for (int i = 0; i < kVL; ++i)
             if (p[i] == kNone) s2[i] = kNone;
         GP_CK(2);
+        // The freedom test of the cached candidate (P_k[s2], P_k[P_k[s2]]) is issued with the
+        // test of p (same dependent levels) on latency-bound short lists; on long lists (kVL = 4:
+        // the big levels, bound by the LSU's random-gather rate) only for the vertices whose
+        // target p was matched by someone else, which saves two gathers for every vertex that
+        // matches or keeps p (most of them).
+        constexpr bool kSpecS = kVL < 4;
         // level 3: P_k[p] and P_k[s2] (freedom test of the cached candidate, P only)
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
             qq[i] = p[i] != kNone ? ldcg(Pk + p[i]) : kNone;
-            ps[i] = s2[i] != kNone ? ldcg(Pk + s2[i]) : -1;
+            ps[i] = (kSpecS && s2[i] != kNone) ? ldcg(Pk + s2[i]) : -1;
         }
         // level 4: P_k[q] (did p match q?) and P_k[P_k[s2]]
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
             rr[i] = (p[i] != kNone && qq[i] != u[i] && qq[i] >= 0) ? ldcg(Pk + qq[i]) : -1;
             pps[i] = ps[i] >= 0 ? ldcg(Pk + ps[i]) : -1;
+        }
+        if (!kSpecS) {  // deferred: only where p matched q != u this round
+#pragma unroll
+            for (int i = 0; i < kVL; ++i)
+                ps[i] = (p[i] != kNone && qq[i] != u[i] && rr[i] == p[i] && s2[i] != kNone) ? ldcg(Pk + s2[i]) : -1;
+#pragma unroll
+            for (int i = 0; i < kVL; ++i) pps[i] = ps[i] >= 0 ? ldcg(Pk + ps[i]) : -1;
         }
         GP_CK_SINK(rr[i_] + pps[i_]);
         GP_CK(3);

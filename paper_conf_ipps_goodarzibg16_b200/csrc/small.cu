@@ -34,7 +34,7 @@
 namespace gp {
 
 constexpr int kSNT = 512;                  // threads of the one CTA (128 registers each: no spills)
-constexpr int kSVPT = 16;                  // vertices per thread, their M / P kept in registers
+constexpr int kSVPT = 16;                  // cap: at most 16 vertices per thread (n <= 8192)
 constexpr size_t kSmallSmemMax = 227 * 1024;
 
 struct SmallLevelOut {  // one arena slot (device pointers)
@@ -56,7 +56,7 @@ struct SmallArgs {
 
 // shared-memory layout (int32 words), each array 16-byte aligned
 struct SmallLayout {
-    int32_t adjp, adjncy, adjwgt, vwgt, M, P, CM, scan, total;
+    int32_t adjp, adjncy, adjwgt, M, P, CM, R, stamp, scan, total;
 };
 __host__ __device__ inline int32_t small_round4(int32_t x) { return (x + 3) & ~3; }
 __host__ __device__ inline SmallLayout small_layout(int32_t cap_n, int32_t cap_nnz) {
@@ -65,10 +65,11 @@ __host__ __device__ inline SmallLayout small_layout(int32_t cap_n, int32_t cap_n
     L.adjp = o;   o += small_round4(cap_n + 1);
     L.adjncy = o; o += small_round4(cap_nnz);
     L.adjwgt = o; o += small_round4(cap_nnz);
-    L.vwgt = o;   o += small_round4(cap_n);
     L.M = o;      o += small_round4(cap_n);
     L.P = o;      o += small_round4(cap_n);
-    L.CM = o;     o += small_round4(cap_n);
+    L.CM = o;     o += small_round4(cap_n);   // also the rescan list of the even rounds
+    L.R = o;      o += small_round4(cap_n);   // the rescan list of the odd rounds
+    L.stamp = o;  o += small_round4((cap_n + 3) / 4);  // 1 byte per vertex: "changed this round"
     L.scan = o;   o += 64;
     L.total = o;
     return L;
@@ -145,10 +146,12 @@ template <bool H>
 __global__ void __launch_bounds__(kSNT, 1) k_small(const __grid_constant__ SmallArgs a) {
     extern __shared__ __align__(16) int32_t sw[];
     const SmallLayout Lo = small_layout(a.cap_n, a.cap_nnz);
-    int32_t *adjp = sw + Lo.adjp, *adjncy = sw + Lo.adjncy, *adjwgt = sw + Lo.adjwgt, *vwgt = sw + Lo.vwgt;
+    int32_t *adjp = sw + Lo.adjp, *adjncy = sw + Lo.adjncy, *adjwgt = sw + Lo.adjwgt;
     int32_t *M = sw + Lo.M, *P = sw + Lo.P, *CM = sw + Lo.CM, *scan = sw + Lo.scan;
+    int32_t *Rl[2] = {CM, sw + Lo.R};
+    uint8_t *stamp = reinterpret_cast<uint8_t *>(sw + Lo.stamp);
     const int t = threadIdx.x;
-    __shared__ int32_t s_n, s_nnz;
+    __shared__ int32_t s_n, s_nnz, s_rn, s_pairs, s_dead;
 
     const volatile SizeRec *in = a.in;
     int32_t n = in->n, nnz = in->nnz;
@@ -165,88 +168,144 @@ __global__ void __launch_bounds__(kSNT, 1) k_small(const __grid_constant__ Small
         small_load(adjp, gadjp, n + 1);
         small_load(adjncy, gadjncy, nnz);
         small_load(adjwgt, gadjwgt, nnz);
-        small_load(vwgt, gvwgt, n);
-        // this thread's vertices u = t + i * kSNT: their M / P in registers (owner writes only);
-        // the shared copies are what the other threads read
-        int32_t Mu[kSVPT], Pu[kSVPT];
-#pragma unroll
-        for (int i = 0; i < kSVPT; ++i) {
-            Mu[i] = kFree;
-            Pu[i] = kNone;
-            const int32_t u = t + i * kSNT;
-            if (u < n) {
-                M[u] = kFree;
-                P[u] = kNone;
-            }
+        for (int32_t u = t; u < n; u += kSNT) {
+            M[u] = kFree;
+            stamp[u] = 1;  // round 1: every vertex proposes
         }
         __syncthreads();
         trace_mark(tr, 1);
-        // ---- matching rounds (A2-A4) ----
+        // ---- matching rounds (A2-A4), event driven ----
+        // The synchronous rule simulated exactly, with work proportional to what changes:
+        //  * a free vertex's proposal changes only when its target gets matched (the free set
+        //    only shrinks, so a still-free target stays the heaviest free neighbour): those
+        //    vertices -- the rescan list R -- rescan, nobody else;
+        //  * a mutual pair appears only where one of its ends changed its proposal this round
+        //    (else it was mutual a round earlier and matched then): the commit looks at the
+        //    changed vertices only (stamp = 1), the pair is handled by its changed end (the
+        //    lower id when both changed), which writes both M entries and lists the neighbours
+        //    that proposed to either end for the next round's rescans (each such vertex proposes
+        //    to one vertex, so it is listed once).
+        //  live = free vertices with a proposal; a round with live > 0 matches >= 1 pair (§2.1).
         unsigned long long arcs = 0, rows = 0, visits = 0;
         int32_t rounds = 0, maximal = 0;
-        for (int k = 1;; ++k) {
-            // propose: a free vertex keeps a still-free target, else rescans its row
-            bool prop = false;
+        auto rescan = [&](int32_t u) -> int32_t {  // heaviest free neighbour of u, or -2
+            unsigned long long best = 0;
+            const int32_t s0 = adjp[u], e0 = adjp[u + 1];
+            int32_t j = s0;
+            for (; j + 4 <= e0; j += 4) {  // four independent shared-memory chains
+                int32_t x[4], w[4], f[4];
 #pragma unroll
-            for (int i = 0; i < kSVPT; ++i) {
-                const int32_t u = t + i * kSNT;
-                if (u >= n || Mu[i] != kFree || Pu[i] == -2) continue;  // matched / dead for good
-                if (k == 1 || M[Pu[i]] != kFree) {
-                    unsigned long long best = 0;
-                    const int32_t s0 = adjp[u], e0 = adjp[u + 1];
-                    int32_t j = s0;
-                    for (; j + 4 <= e0; j += 4) {  // four independent shared-memory chains
-                        int32_t x[4], w[4], f[4];
-#pragma unroll
-                        for (int q = 0; q < 4; ++q) {
-                            x[q] = adjncy[j + q];
-                            w[q] = adjwgt[j + q];
-                        }
-#pragma unroll
-                        for (int q = 0; q < 4; ++q) f[q] = M[x[q]];
-#pragma unroll
-                        for (int q = 0; q < 4; ++q)
-                            if (f[q] == kFree) {
-                                const unsigned long long kk = skey<H>(a.tie_seed, w[q], x[q]);
-                                best = kk > best ? kk : best;
-                            }
-                    }
-                    for (; j < e0; ++j) {
-                        const int32_t x = adjncy[j];
-                        if (M[x] == kFree) {
-                            const unsigned long long kk = skey<H>(a.tie_seed, adjwgt[j], x);
-                            best = kk > best ? kk : best;
-                        }
-                    }
-                    arcs += (unsigned long long)(e0 - s0);
-                    if (k > 1) ++rows;
-                    const int32_t b = key_vertex<H>(a.tie_seed, best);
-                    Pu[i] = b == kNone ? -2 : b;
-                    P[u] = Pu[i];
+                for (int q = 0; q < 4; ++q) {
+                    x[q] = adjncy[j + q];
+                    w[q] = adjwgt[j + q];
                 }
-                prop = prop || Pu[i] >= 0;
+#pragma unroll
+                for (int q = 0; q < 4; ++q) f[q] = M[x[q]];
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+                    if (f[q] == kFree) {
+                        const unsigned long long kk = skey<H>(a.tie_seed, w[q], x[q]);
+                        best = kk > best ? kk : best;
+                    }
             }
-            if (!__syncthreads_or(prop)) {
+            for (; j < e0; ++j) {
+                const int32_t x = adjncy[j];
+                if (M[x] == kFree) {
+                    const unsigned long long kk = skey<H>(a.tie_seed, adjwgt[j], x);
+                    best = kk > best ? kk : best;
+                }
+            }
+            arcs += (unsigned long long)(e0 - s0);
+            const int32_t b = key_vertex<H>(a.tie_seed, best);
+            return b == kNone ? -2 : b;
+        };
+        // round 1 proposals: every vertex
+        int32_t mylive = 0;
+        for (int32_t u = t; u < n; u += kSNT) {
+            P[u] = rescan(u);
+            mylive += P[u] >= 0;
+        }
+        int32_t live;
+        sblock_scan(mylive, scan, live);  // (block total; syncs: P complete)
+        int32_t rn = n, cur = 0;           // the changed vertices of this round: all (round 1)
+#ifdef GP_CHECKPOINTS
+        long long ck0 = clock64();
+#define GP_SCK(j) do { if (t == 0 && k < 16) a.levdev[gl].match.ck[k][j] = clock64() - ck0; } while (0)
+#else
+#define GP_SCK(j) do { } while (0)
+#endif
+        for (int k = 1;; ++k) {
+#ifdef GP_CHECKPOINTS
+            ck0 = clock64();
+#endif
+            if (live == 0) {
                 maximal = 1;
                 break;
             }
             if (a.max_rounds > 0 && rounds >= a.max_rounds) break;
-            // commit (handshake): reads P only, each endpoint writes its own M
-            bool made = false;
-#pragma unroll
-            for (int i = 0; i < kSVPT; ++i) {
-                const int32_t u = t + i * kSNT;
-                if (u >= n || Mu[i] != kFree || Pu[i] < 0) continue;
+            if (t == 0) {
+                s_rn = 0;
+                s_pairs = 0;
+                s_dead = 0;
+            }
+            __syncthreads();
+            GP_SCK(0);
+            // commit (handshake) over the changed vertices
+            int32_t *Rn = Rl[cur ^ 1];
+            for (int32_t i = t; i < rn; i += kSNT) {
+                const int32_t x = k == 1 ? i : Rl[cur][i];
+                if (M[x] != kFree) continue;
+                const int32_t d = P[x];
+                if (d < 0) continue;
                 ++visits;
-                if (P[Pu[i]] == u) {
-                    Mu[i] = Pu[i];
-                    M[u] = Pu[i];
-                    made = true;
+                if (P[d] != x) continue;
+                if (stamp[d] && d < x) continue;  // both ends changed: the lower id handles it
+                M[x] = d;
+                M[d] = x;
+                atomicAdd(&s_pairs, 1);
+                // neighbours that proposed to x or d rescan next round
+#pragma unroll 1
+                for (int e = 0; e < 2; ++e) {
+                    const int32_t y0 = e ? d : x, other = e ? x : d;
+                    for (int32_t j = adjp[y0]; j < adjp[y0 + 1]; ++j) {
+                        const int32_t y = adjncy[j];
+                        if (y != other && P[y] == y0) Rn[atomicAdd(&s_rn, 1)] = y;
+                    }
                 }
             }
-            if (__syncthreads_or(made)) ++rounds;
+            GP_SCK(1);
+            __syncthreads();
+            GP_SCK(2);
+            // the stamps of this round's changed vertices are cleared, the next ones set
+            for (int32_t i = t; i < rn; i += kSNT) stamp[k == 1 ? i : Rl[cur][i]] = 0;
+            const int32_t pairs = s_pairs, rnn = s_rn;
+            if (pairs > 0) ++rounds;
+            live -= 2 * pairs;
+            __syncthreads();
+            GP_SCK(3);
+            // round k+1 proposals: the rescans (a vertex matched this round is skipped)
+            int32_t dead = 0;
+            for (int32_t i = t; i < rnn; i += kSNT) {
+                const int32_t y = Rn[i];
+                stamp[y] = 1;
+                if (M[y] != kFree) continue;
+                ++rows;
+                const int32_t b = rescan(y);
+                P[y] = b;
+                dead += b < 0;
+            }
+            if (dead) atomicAdd(&s_dead, dead);
+            GP_SCK(4);
+            __syncthreads();
+            GP_SCK(5);
+            live -= s_dead;
+            rn = rnn;
+            cur ^= 1;
             if (k > n + 2) __trap();  // each round with proposals matches >= 1 pair
+            GP_SCK(6);
+            if (t == 0 && k < 16) a.levdev[gl].match.ck[k][7] = rn, a.levdev[gl].match.ck[k][8] = rn + 1;
         }
+#undef GP_SCK
         trace_mark(tr, 2);
         // ---- leftover (P18.s12-13) + cmap (P18.s16-27) ----
         const int32_t per = (n + kSNT - 1) / kSNT;
@@ -270,7 +329,7 @@ __global__ void __launch_bounds__(kSNT, 1) k_small(const __grid_constant__ Small
         for (int32_t u = t; u < n; u += kSNT) {
             const int32_t m = M[u], cu = CM[u];
             o.CM[u] = cu;
-            if (u <= m) o.cvwgt[cu] = vwgt[u] + (m != u ? vwgt[m] : 0);  // P12.s27
+            if (u <= m) o.cvwgt[cu] = __ldcg(gvwgt + u) + (m != u ? __ldcg(gvwgt + m) : 0);  // P12.s27
         }
         // leaders by coarse id (P is free from here on) and the widest merged row
         int32_t *lead_of = P;
