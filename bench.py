@@ -288,14 +288,20 @@ def run_ours(args, rank, world, local_rank):
     # level l's matching then its contraction (speculative levels after the stop come last);
     # the median over the timed steps of each launch's CUDA-event time
     per_step = len(ltimes) // args.steps if args.steps else 0
-    level_rows = []
-    if not sharded and args.loopback <= 1 and per_step >= 2 * len(levels):
-        for i, l in enumerate(levels):
+    level_rows, tail = [], None
+    if not sharded and args.loopback <= 1 and per_step >= 1:
+        # levels on the level kernels: 2 launches each (propose = k_match_level, contract =
+        # k_contract_level); the coarse-level tail (one 'other' launch) runs the rest
+        step0 = ltimes[:per_step]
+        nreg = 0
+        while 2 * nreg + 1 < per_step and nreg < len(levels) and step0[2 * nreg][0] == "propose" \
+                and step0[2 * nreg + 1][0] == "contract":
+            nreg += 1
+        for i in range(nreg):
+            l = levels[i]
             t = {}
-            for fam, kind, off in (("match", "propose", 0), ("contract", "contract", 1)):
-                xs = [ltimes[st * per_step + 2 * i + off] for st in range(args.steps)]
-                assert all(k == kind for k, _ in xs), "launch order does not map to levels"
-                t[fam] = statistics.median(m for _, m in xs)
+            for fam, off in (("match", 0), ("contract", 1)):
+                t[fam] = statistics.median(ltimes[st * per_step + 2 * i + off][1] for st in range(args.steps))
             b = level_bytes(l)
             tl = t["match"] + t["contract"]
             level_rows.append({
@@ -306,6 +312,14 @@ def run_ours(args, rank, world, local_rank):
                 "GBps_match": b["match"] / (t["match"] / 1e3) / 1e9, "GBps_contract": b["contract"] / (t["contract"] / 1e3) / 1e9,
                 "frac_match": b["match"] / (t["match"] / 1e3) / 1e9 / peak,
                 "frac_contract": b["contract"] / (t["contract"] / 1e3) / 1e9 / peak})
+        if nreg < len(levels) and 2 * nreg < per_step and step0[2 * nreg][0] == "other":
+            tus = 1e3 * statistics.median(ltimes[st * per_step + 2 * nreg][1] for st in range(args.steps))
+            rest = levels[nreg:]
+            tail = {"levels": [nreg, len(levels) - 1], "launches": 1, "us": round(tus, 2),
+                    "n_first": rest[0]["n"], "edges": sum(l["nnz"] // 2 for l in rest),
+                    "rounds": [l["rounds"] for l in rest],
+                    "edges_per_s": sum(l["nnz"] // 2 for l in rest) / (tus / 1e6),
+                    "kernel": "coarse-level tail: k_small (one CTA, shared memory) or k_medium (one cluster, L2)"}
 
     # projection: a synthetic labelling of the coarsest graph (c mod 64)
     # carried down to level 0 in one launch; algorithmic bytes = CM_0 read + labels written +
@@ -391,6 +405,7 @@ def run_ours(args, rank, world, local_rank):
                     "edges_per_s": level_rows[0]["edges_per_s"], "peak_GBps": peak, "peak_kind": peak_kind}
                    if level_rows else None),
         "levels": level_rows,
+        "tail": tail,
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "peak_kind": peak_kind,
                      "unit": "GB/s", "frac": achieved / peak,
                      "traffic": traffic[0] if traffic else None,

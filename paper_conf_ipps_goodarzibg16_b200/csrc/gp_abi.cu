@@ -710,7 +710,19 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
         sl.stall_pct = pct;
         sl.max_levels = max_levels;
         sl.max_rounds = opts->max_rounds;
-        s2 = enqueue_small(ctx, sl);
+        if (small_use(n_b, m_b)) {
+            s2 = enqueue_small(ctx, sl);
+        } else {  // one thread-block cluster, state in global memory
+            MediumLaunch ml;
+            static_cast<SmallLaunch &>(ml) = sl;
+            void *scr = nullptr;
+            s2 = dev_alloc(ctx, &scr, medium_scratch_bytes(n_b, m_b));
+            if (s2 == GP_OK) {
+                h->arenas.push_back(scr);
+                ml.scratch = scr;
+                s2 = enqueue_medium(ctx, ml);
+            }
+        }
         keep_host.push_back(std::move(hd));  // read by the async copy: alive until the final sync
         return s2;
     };
@@ -719,8 +731,8 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
     bool stop_seen = false;
     while (st == GP_OK) {
         while (st == GP_OK && !stop_seen && enq < max_levels && enq - obs < kAhead) {
-            if (small_use(tight_n, tight_m)) {
-                GP_DBG("enqueue tail levels %d.. in one CTA (bounds n=%d nnz=%d)\n", enq, tight_n, tight_m);
+            if (small_use(tight_n, tight_m) || medium_use(tight_n, tight_m)) {
+                GP_DBG("enqueue tail levels %d.. in one CTA / cluster (bounds n=%d nnz=%d)\n", enq, tight_n, tight_m);
                 st = enqueue_tail(enq);
                 enq = max_levels;
                 break;

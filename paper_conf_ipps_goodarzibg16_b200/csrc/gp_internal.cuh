@@ -316,6 +316,14 @@ size_t small_slot_ints(int32_t n, int32_t nnz);
 void small_slot_carve(int32_t *base, int32_t n, int32_t nnz, void *out_slot);
 size_t small_slot_desc_bytes();
 gp_status enqueue_small(Ctx *ctx, const SmallLaunch &L);
+// coarse-level tail in one thread-block cluster (medium.cu): the same per-level outputs as the
+// single-CTA tail, graph and state in global memory (L2), for levels too big for one SM
+struct MediumLaunch : SmallLaunch {
+    void *scratch;  // medium_scratch_bytes(cap_n, cap_nnz)
+};
+bool medium_use(int32_t n_bound, int32_t nnz_bound);
+size_t medium_scratch_bytes(int32_t n, int32_t nnz);
+gp_status enqueue_medium(Ctx *ctx, const MediumLaunch &L);
 
 // refinement of un-coarsening (refine.cu)
 gp_status refine_graph(Ctx *ctx, const Graph *g, int32_t *d_part, const gp_refine_opts &o, int32_t *moves_out,

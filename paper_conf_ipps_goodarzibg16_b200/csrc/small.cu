@@ -151,7 +151,10 @@ __global__ void __launch_bounds__(kSNT, 1) k_small(const __grid_constant__ Small
     int32_t *Rl[2] = {CM, sw + Lo.R};
     uint8_t *stamp = reinterpret_cast<uint8_t *>(sw + Lo.stamp);
     const int t = threadIdx.x;
-    __shared__ int32_t s_n, s_nnz, s_rn, s_pairs, s_dead;
+    __shared__ int32_t s_n, s_nnz;
+    // round counters by round parity: slot k & 1 is reset in round k - 1 (after the barrier that
+    // follows every read of round k - 2's values) and read in round k after its barriers
+    __shared__ int32_t s_rn[2], s_pairs[2], s_dead[2];
 
     const volatile SizeRec *in = a.in;
     int32_t n = in->n, nnz = in->nnz;
@@ -243,18 +246,16 @@ __global__ void __launch_bounds__(kSNT, 1) k_small(const __grid_constant__ Small
                 break;
             }
             if (a.max_rounds > 0 && rounds >= a.max_rounds) break;
-            if (t == 0) {
-                s_rn = 0;
-                s_pairs = 0;
-                s_dead = 0;
-            }
+            if (k == 1 && t == 0) s_rn[1] = s_pairs[1] = s_dead[1] = 0;
             __syncthreads();
+            if (t == 0) s_rn[(k + 1) & 1] = s_pairs[(k + 1) & 1] = s_dead[(k + 1) & 1] = 0;
+            const int sl = k & 1;
             GP_SCK(0);
             // commit (handshake) over the changed vertices
             int32_t *Rn = Rl[cur ^ 1];
             for (int32_t i = t; i < rn; i += kSNT) {
                 const int32_t x = k == 1 ? i : Rl[cur][i];
-                if (M[x] != kFree) continue;
+                if (x < 0) continue;  // matched in the previous round (marked by the rescan pass)
                 const int32_t d = P[x];
                 if (d < 0) continue;
                 ++visits;
@@ -262,14 +263,14 @@ __global__ void __launch_bounds__(kSNT, 1) k_small(const __grid_constant__ Small
                 if (stamp[d] && d < x) continue;  // both ends changed: the lower id handles it
                 M[x] = d;
                 M[d] = x;
-                atomicAdd(&s_pairs, 1);
+                atomicAdd(&s_pairs[sl], 1);
                 // neighbours that proposed to x or d rescan next round
 #pragma unroll 1
                 for (int e = 0; e < 2; ++e) {
                     const int32_t y0 = e ? d : x, other = e ? x : d;
                     for (int32_t j = adjp[y0]; j < adjp[y0 + 1]; ++j) {
                         const int32_t y = adjncy[j];
-                        if (y != other && P[y] == y0) Rn[atomicAdd(&s_rn, 1)] = y;
+                        if (y != other && P[y] == y0) Rn[atomicAdd(&s_rn[sl], 1)] = y;
                     }
                 }
             }
@@ -277,8 +278,11 @@ __global__ void __launch_bounds__(kSNT, 1) k_small(const __grid_constant__ Small
             __syncthreads();
             GP_SCK(2);
             // the stamps of this round's changed vertices are cleared, the next ones set
-            for (int32_t i = t; i < rn; i += kSNT) stamp[k == 1 ? i : Rl[cur][i]] = 0;
-            const int32_t pairs = s_pairs, rnn = s_rn;
+            for (int32_t i = t; i < rn; i += kSNT) {
+                const int32_t x = k == 1 ? i : Rl[cur][i];
+                if (x >= 0) stamp[x] = 0;
+            }
+            const int32_t pairs = s_pairs[sl], rnn = s_rn[sl];
             if (pairs > 0) ++rounds;
             live -= 2 * pairs;
             __syncthreads();
@@ -287,18 +291,21 @@ __global__ void __launch_bounds__(kSNT, 1) k_small(const __grid_constant__ Small
             int32_t dead = 0;
             for (int32_t i = t; i < rnn; i += kSNT) {
                 const int32_t y = Rn[i];
+                if (M[y] != kFree) {  // matched this round: out of the next round's list
+                    Rn[i] = -1;
+                    continue;
+                }
                 stamp[y] = 1;
-                if (M[y] != kFree) continue;
                 ++rows;
                 const int32_t b = rescan(y);
                 P[y] = b;
                 dead += b < 0;
             }
-            if (dead) atomicAdd(&s_dead, dead);
+            if (dead) atomicAdd(&s_dead[sl], dead);
             GP_SCK(4);
             __syncthreads();
             GP_SCK(5);
-            live -= s_dead;
+            live -= s_dead[sl];
             rn = rnn;
             cur ^= 1;
             if (k > n + 2) __trap();  // each round with proposals matches >= 1 pair

@@ -19,6 +19,27 @@ elif case == "star5000":
     ctx, g, thr = gp.Context(0), G.from_edge_list(5001, edges), 2
 elif case == "loopback3":
     ctx, g, thr = gp.Context(0, loopback=3), G.delaunay_like(64), 20
+elif case == "c1_tail":  # the coarse-level tail kernel (csrc/small.cu) runs every level of C1
+    ctx, g, thr = gp.Context(0), G.make_config("C1"), 100
+elif case == "medium_tail":  # the cluster tail (csrc/medium.cu): forced for a 16 K-vertex mesh
+    os.environ["GP_SMALL"] = "0"
+    os.environ["GP_MEDIUM"] = "1"
+    ctx, g, thr = gp.Context(0), G.delaunay_like(128), 100
+elif case == "refine":  # gp_uncoarsen: projection + refinement kernels (csrc/refine.cu)
+    import numpy as np
+    import torch
+    ctx, g = gp.Context(0), G.rmat(12)
+    levels = oracle.coarsen_to(g, threshold=100)
+    pc = (np.arange(levels[-1]["n_coarse"]) % 8).astype(np.int32)
+    ref, moves = oracle.uncoarsen(g, levels, pc, 8)
+    d = {k: g[k].cuda() for k in ("adjp", "adjncy", "adjwgt", "vwgt")}
+    Gr = gp.Graph.create(ctx, d["adjp"], d["adjncy"], d["adjwgt"], d["vwgt"])
+    H = Gr.coarsen_to(100)
+    out = torch.empty(g["n"], dtype=torch.int32, device="cuda")
+    mv = H.uncoarsen(Gr, torch.from_numpy(pc).cuda(), out, 8)
+    assert np.array_equal(out.cpu().numpy(), ref) and mv == moves
+    print(f"refine: uncoarsen of {len(levels)} levels bit-exact vs the oracle ({mv} moves)")
+    raise SystemExit(0)
 else:
     raise SystemExit(f"unknown case {case}")
 got = gpu_coarsen(gp, ctx, g, threshold=thr)

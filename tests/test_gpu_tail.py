@@ -1,6 +1,11 @@
-"""Coarse-level tail (csrc/small.cu), -m gpu: once a level's graph fits one
-SM's shared memory, one CTA runs every remaining level in one launch.  Its hierarchies must be
-bit-identical to the oracle and to the level kernels (GP_SMALL=0 forces the level kernels)."""
+"""Coarse-level tail, -m gpu: once the level bounds are small, ONE launch runs
+every remaining level -- one CTA with the graph in shared memory (csrc/small.cu) when it fits one
+SM, else one thread-block cluster with the graph in L2 (csrc/medium.cu).  Each hierarchy must be
+bit-identical to the oracle and to the level kernels, in all three modes:
+  small   (default)                  single CTA when it fits, else the level kernels
+  medium  (GP_SMALL=0, GP_MEDIUM=1)  the cluster kernel (opt-in: measured slower)
+                                     even for graphs that fit one SM
+  levels  (GP_SMALL=0, GP_MEDIUM=0)  the grid-wide level kernels only."""
 import os
 
 import numpy as np
@@ -26,18 +31,25 @@ def ctx(gp):
     c.close()
 
 
-def _run(gp, ctx, g, small, **kw):
-    old = os.environ.get("GP_SMALL")
-    os.environ["GP_SMALL"] = "1" if small else "0"
+MODES = {"small": {}, "medium": {"GP_SMALL": "0", "GP_MEDIUM": "1"}, "levels": {"GP_SMALL": "0", "GP_MEDIUM": "0"}}
+
+
+def _run(gp, ctx, g, mode, **kw):
+    env = MODES[mode]
+    old = {k: os.environ.get(k) for k in ("GP_SMALL", "GP_MEDIUM")}
+    for k in old:
+        os.environ.pop(k, None)
+    os.environ.update(env)
     try:
         l0 = ctx.launch_count()
         got = gpu_coarsen(gp, ctx, g, **kw)
         return got, ctx.launch_count() - l0
     finally:
-        if old is None:
-            del os.environ["GP_SMALL"]
-        else:
-            os.environ["GP_SMALL"] = old
+        for k, v in old.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
 
 
 def _star(n_leaves, wmax=100):
@@ -70,15 +82,28 @@ def test_tail_equals_oracle_and_level_kernels(gp, ctx, name):
     make, kw = CASES[name]
     g = make()
     ref = oracle.coarsen_to(g, **kw)
-    small, l_small = _run(gp, ctx, g, True, **kw)
-    big, l_big = _run(gp, ctx, g, False, **kw)
-    assert_levels_equal(small, ref, f"{name} tail")
-    assert_levels_equal(big, ref, f"{name} level kernels")
-    if len(ref) > 1:
-        assert l_small < l_big, (l_small, l_big)  # the tail really ran (fewer launches)
+    launches = {}
+    for mode in MODES:
+        got, launches[mode] = _run(gp, ctx, g, mode, **kw)
+        assert_levels_equal(got, ref, f"{name} {mode}")
+    if len(ref) > 1:  # the tail really ran (fewer launches than the level kernels)
+        assert launches["medium"] < launches["levels"], launches
+        if g["n"] <= 8192:
+            assert launches["small"] < launches["levels"], launches
 
 
 def test_tail_is_one_launch_on_c1(gp, ctx):
     g = G.make_config("C1")
-    got, launches = _run(gp, ctx, g, True, threshold=100)
-    assert len(got) == 6 and launches <= 2  # (+ the input's size record copy is not a launch)
+    got, launches = _run(gp, ctx, g, "small", threshold=100)
+    assert len(got) == 6 and launches <= 2  # (graph creation's totals kernel + the tail)
+
+
+@pytest.mark.parametrize("name", ["C3_512", "C2_2^16", "road_256", "rmat14_w4"])
+def test_medium_tail_mid_hierarchy(gp, ctx, name):
+    """Graphs whose hierarchies enter the cluster tail after a few level kernels."""
+    g = {"C3_512": lambda: G.delaunay_like(512), "C2_2^16": lambda: G.rgg(1 << 16),
+         "road_256": lambda: G.road_like(256), "rmat14_w4": lambda: G.rmat(14, wmax=4)}[name]()
+    ref = oracle.coarsen_to(g, threshold=100)
+    for mode in ("small", "medium", "levels"):
+        got, _ = _run(gp, ctx, g, mode, threshold=100)
+        assert_levels_equal(got, ref, f"{name} {mode}")
