@@ -95,6 +95,15 @@ struct ContractSmem {
 // ---------------------------------------------------------------------------------------
 // merge helpers
 // ---------------------------------------------------------------------------------------
+// CM gathers: L2 (ld.global.cg) by default; GP_CM_CA=1 at build time reads them through L1
+// (safe: CM is written by C1b, a phase that ends with a grid barrier whose acquire invalidates
+// every SM's L1).
+#ifdef GP_CM_CA
+__device__ __forceinline__ int32_t ldCM(const int32_t *p) { return __ldca(p); }
+#else
+__device__ __forceinline__ int32_t ldCM(const int32_t *p) { return __ldcg(p); }
+#endif
+
 __device__ __forceinline__ unsigned long long ckey(int32_t cx, int32_t w) {
     return ((unsigned long long)(uint32_t)cx << 32) | (uint32_t)w;
 }
@@ -550,7 +559,7 @@ __device__ __forceinline__ void gather_row(const ContractArgs &a, int32_t c, int
     for (int side = 0; side < 2; ++side) {
         const int32_t s = side ? sg.z : sg.x, e = s + (side ? sg.w : sg.y);
         for (int32_t j = s + tid; j < e; j += nthr) {
-            const int32_t cx = __ldcg(a.CM + __ldcs(a.adjncy + j));
+            const int32_t cx = ldCM(a.CM + __ldcs(a.adjncy + j));
             if (cx != c + a.cbase) dst[claim()] = ckey(cx, __ldcs(a.adjwgt + j));  // drop the collapsed edge (R9)
         }
     }
@@ -719,7 +728,7 @@ __device__ __noinline__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, 
                 w[q] = p < ub ? __ldcs(a.adjwgt + j) : 0;
             }
 #pragma unroll
-            for (int q = 0; q < 4; ++q) cx[q] = x[q] >= 0 ? __ldcg(a.CM + x[q]) : 0;
+            for (int q = 0; q < 4; ++q) cx[q] = x[q] >= 0 ? ldCM(a.CM + x[q]) : 0;
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
                 const int32_t p = p0 + q * kCNT;
@@ -867,7 +876,7 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
                     for (int k = 0; k < kB; ++k) {
                         const int32_t idx = b0 + k * 32 + lane;
                         const int32_t x = idx < S ? (int32_t)wb32[2 * idx + 1] : -1;
-                        cx[k] = x >= 0 ? __ldcg(a.CM + x) : 0;
+                        cx[k] = x >= 0 ? ldCM(a.CM + x) : 0;
                     }
 #pragma unroll
                     for (int k = 0; k < kB; ++k) {

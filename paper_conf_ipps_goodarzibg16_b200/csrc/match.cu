@@ -97,6 +97,17 @@ struct MatchSmem {
 };
 
 __device__ __forceinline__ int32_t ldcg(const int32_t *p) { return __ldcg(p); }
+// Loads of the current round's proposals P_k, its live list and S.  L2 (ld.global.cg) by
+// default; GP_P_CA=1 at build time reads them through L1 (safe: they were written in an earlier
+// phase and every phase starts after a grid barrier whose acquire invalidates the SM's L1; the
+// only writes within a phase mark dead vertices NONE, which a stale read cannot turn into a
+// handshake).  Measured equal on C3 / C2 / C5 (3.31 vs 3.30, 2.80 vs 2.82, 29.5 vs 29.0 ms):
+// the mesh locality of these gathers is already captured by coalescing within a warp.
+#ifdef GP_P_CA
+__device__ __forceinline__ int32_t ldP(const int32_t *p) { return __ldca(p); }
+#else
+__device__ __forceinline__ int32_t ldP(const int32_t *p) { return __ldcg(p); }
+#endif
 __device__ __forceinline__ int4 ld_volatile_v4(const int4 *p) {
     int4 v;
     asm volatile("ld.volatile.global.v4.s32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p)
@@ -131,8 +142,8 @@ __device__ __forceinline__ void wq_push(int32_t *q, int32_t &qn, int32_t *list, 
 // round <= k has P_k[P_k[x]] == x (matched vertices keep their partner in both proposal
 // buffers), and a dead vertex (P = NONE) never neighbours a vertex that still rescans.
 __device__ __forceinline__ bool free_after(int32_t x, const int32_t *Pk) {
-    const int32_t px = ldcg(Pk + x);
-    return !(px >= 0 && ldcg(Pk + px) == x);
+    const int32_t px = ldP(Pk + x);
+    return !(px >= 0 && ldP(Pk + px) == x);
 }
 
 // top-2 of packed keys (k1 > k2, both 0 = none)
@@ -413,10 +424,10 @@ __device__ __noinline__ void hub_phase_mc(const MatchArgs &a, MatchSmem &sm, int
             unsigned long long key = 0;
             if (check) {
 #pragma unroll
-                for (int q = 0; q < 8; ++q) px[q] = x[q] >= 0 ? ldcg(Pk + x[q]) : -1;
+                for (int q = 0; q < 8; ++q) px[q] = x[q] >= 0 ? ldP(Pk + x[q]) : -1;
 #pragma unroll
                 for (int q = 0; q < 8; ++q) {
-                    const int32_t pp = px[q] >= 0 ? ldcg(Pk + px[q]) : -1;
+                    const int32_t pp = px[q] >= 0 ? ldP(Pk + px[q]) : -1;
                     if (x[q] >= 0 && pp != x[q]) key = umax64(key, pack_key<H>(a.tie_seed, w[q], x[q]));  // x free after round k
                 }
             } else {
@@ -548,7 +559,7 @@ __device__ __noinline__ void wake_phase(const MatchArgs &a, MatchSmem &sm, int32
                 x[q] = j < c1 ? __ldg(a.adjncy + j) : -1;
             }
 #pragma unroll
-            for (int q = 0; q < 8; ++q) px[q] = x[q] >= 0 ? ldcg(Pk + x[q]) : -1;
+            for (int q = 0; q < 8; ++q) px[q] = x[q] >= 0 ? ldP(Pk + x[q]) : -1;
 #pragma unroll
             for (int q = 0; q < 8; ++q)
                 if (px[q] == vv && ldcg(a.parked + x[q])) {  // parked on the matched vv: resolve it
@@ -593,16 +604,16 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
     };
     for (long long g = claim_next(); g < (a.interleave ? ngroups : g_hi); g = claim_next()) {
         const long long idx = g * VPW + lane / G;
-        int32_t u = idx < len ? ((k == 1 && !Lover) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
-        const int32_t p = u >= 0 ? ldcg(Pk + u) : kNone;
-        const int32_t s2r = u >= 0 ? ldcg(a.S + u) : kNone;  // not predicated on p: same load level
+        int32_t u = idx < len ? ((k == 1 && !Lover) ? a.vbase + (int32_t)idx : ldP(Lk + idx)) : -1;
+        const int32_t p = u >= 0 ? ldP(Pk + u) : kNone;
+        const int32_t s2r = u >= 0 ? ldP(a.S + u) : kNone;  // not predicated on p: same load level
         const int32_t rs0 = u >= 0 ? __ldg(a.adjp + (u - a.vbase)) : 0;  // speculative row bounds
         const int32_t re0 = u >= 0 ? __ldg(a.adjp + (u - a.vbase) + 1) : 0;
         const int32_t s2 = p != kNone ? s2r : kNone;
-        const int32_t qq = p != kNone ? ldcg(Pk + p) : kNone;
-        const int32_t ps = s2 != kNone ? ldcg(Pk + s2) : -1;
-        const int32_t rr = (p != kNone && qq != u && qq >= 0) ? ldcg(Pk + qq) : -1;
-        const int32_t pps = ps >= 0 ? ldcg(Pk + ps) : -1;
+        const int32_t qq = p != kNone ? ldP(Pk + p) : kNone;
+        const int32_t ps = s2 != kNone ? ldP(Pk + s2) : -1;
+        const int32_t rr = (p != kNone && qq != u && qq >= 0) ? ldP(Pk + qq) : -1;
+        const int32_t pps = ps >= 0 ? ldP(Pk + ps) : -1;
         bool need = false, live = false;
         if (p != kNone) {
             if (gl == 0) ++visits;
@@ -660,9 +671,9 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
                 w[b] = (need && j < e) ? __ldg(a.adjwgt + j) : 0;
             }
 #pragma unroll
-            for (int b = 0; b < 4; ++b) px[b] = x[b] >= 0 ? ldcg(Pk + x[b]) : -1;
+            for (int b = 0; b < 4; ++b) px[b] = x[b] >= 0 ? ldP(Pk + x[b]) : -1;
 #pragma unroll
-            for (int b = 0; b < 4; ++b) pp[b] = px[b] >= 0 ? ldcg(Pk + px[b]) : -1;
+            for (int b = 0; b < 4; ++b) pp[b] = px[b] >= 0 ? ldP(Pk + px[b]) : -1;
 #pragma unroll
             for (int b = 0; b < 4; ++b)
                 if (x[b] >= 0 && pp[b] != x[b]) top2_add(key, key2, pack_key<H>(a.tie_seed, w[b], x[b]));  // x free after round k
@@ -775,11 +786,11 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
             }
         }
 #pragma unroll
-        for (int b = 0; b < KFB; ++b) px[b] = x[b] >= 0 ? ldcg(Pk + x[b]) : -1;
+        for (int b = 0; b < KFB; ++b) px[b] = x[b] >= 0 ? ldP(Pk + x[b]) : -1;
         uint32_t t[KFB];  // tie word of a candidate (x free after round k), w = 0 otherwise
 #pragma unroll
         for (int b = 0; b < KFB; ++b) {
-            const int32_t pp = px[b] >= 0 ? ldcg(Pk + px[b]) : -1;
+            const int32_t pp = px[b] >= 0 ? ldP(Pk + px[b]) : -1;
             const bool cand = x[b] >= 0 && pp != x[b];
             t[b] = cand ? (uint32_t)pack_key<H>(a.tie_seed, w[b], x[b]) : 0u;
             if (!cand) w[b] = 0;
@@ -911,7 +922,7 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
             const long long idx = base + i * 32 + lane;
-            u[i] = (idx < len && (kVL > 1 || lane < gsz)) ? ((kStatic || (k == 1 && !Lover)) ? a.vbase + (int32_t)idx : ldcg(Lk + idx)) : -1;
+            u[i] = (idx < len && (kVL > 1 || lane < gsz)) ? ((kStatic || (k == 1 && !Lover)) ? a.vbase + (int32_t)idx : ldP(Lk + idx)) : -1;
         }
         GP_CK_SINK(u[i_]);
         GP_CK(1);
@@ -919,8 +930,8 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
                                    // then starts one dependent level earlier
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
-            p[i] = u[i] >= 0 ? ldcg(Pk + u[i]) : kNone;
-            s2[i] = u[i] >= 0 ? ldcg(a.S + u[i]) : kNone;  // not predicated on p: same load level
+            p[i] = u[i] >= 0 ? ldP(Pk + u[i]) : kNone;
+            s2[i] = u[i] >= 0 ? ldP(a.S + u[i]) : kNone;  // not predicated on p: same load level
             rs[i] = u[i] >= 0 ? __ldg(a.adjp + (u[i] - a.vbase)) : 0;
             re[i] = u[i] >= 0 ? __ldg(a.adjp + (u[i] - a.vbase) + 1) : 0;
             if (kStatic && u[i] >= 0 && k > 1 && ldcg(a.M + u[i]) != kFree) p[i] = kNone;  // matched: not live
@@ -938,21 +949,21 @@ __device__ void phase_k_impl(const MatchArgs &a, MatchSmem &sm, int k, int32_t l
         // level 3: P_k[p] and P_k[s2] (freedom test of the cached candidate, P only)
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
-            qq[i] = p[i] != kNone ? ldcg(Pk + p[i]) : kNone;
-            ps[i] = (kSpecS && s2[i] != kNone) ? ldcg(Pk + s2[i]) : -1;
+            qq[i] = p[i] != kNone ? ldP(Pk + p[i]) : kNone;
+            ps[i] = (kSpecS && s2[i] != kNone) ? ldP(Pk + s2[i]) : -1;
         }
         // level 4: P_k[q] (did p match q?) and P_k[P_k[s2]]
 #pragma unroll
         for (int i = 0; i < kVL; ++i) {
-            rr[i] = (p[i] != kNone && qq[i] != u[i] && qq[i] >= 0) ? ldcg(Pk + qq[i]) : -1;
-            pps[i] = ps[i] >= 0 ? ldcg(Pk + ps[i]) : -1;
+            rr[i] = (p[i] != kNone && qq[i] != u[i] && qq[i] >= 0) ? ldP(Pk + qq[i]) : -1;
+            pps[i] = ps[i] >= 0 ? ldP(Pk + ps[i]) : -1;
         }
         if (!kSpecS) {  // deferred: only where p matched q != u this round
 #pragma unroll
             for (int i = 0; i < kVL; ++i)
-                ps[i] = (p[i] != kNone && qq[i] != u[i] && rr[i] == p[i] && s2[i] != kNone) ? ldcg(Pk + s2[i]) : -1;
+                ps[i] = (p[i] != kNone && qq[i] != u[i] && rr[i] == p[i] && s2[i] != kNone) ? ldP(Pk + s2[i]) : -1;
 #pragma unroll
-            for (int i = 0; i < kVL; ++i) pps[i] = ps[i] >= 0 ? ldcg(Pk + ps[i]) : -1;
+            for (int i = 0; i < kVL; ++i) pps[i] = ps[i] >= 0 ? ldP(Pk + ps[i]) : -1;
         }
         GP_CK_SINK(rr[i_] + pps[i_]);
         GP_CK(3);
