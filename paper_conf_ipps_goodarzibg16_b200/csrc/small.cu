@@ -253,6 +253,7 @@ __global__ void __launch_bounds__(kSNT, 1) k_small(const __grid_constant__ Small
             GP_SCK(0);
             // commit (handshake) over the changed vertices
             int32_t *Rn = Rl[cur ^ 1];
+            int32_t mypairs = 0;
             for (int32_t i = t; i < rn; i += kSNT) {
                 const int32_t x = k == 1 ? i : Rl[cur][i];
                 if (x < 0) continue;  // matched in the previous round (marked by the rescan pass)
@@ -263,17 +264,32 @@ __global__ void __launch_bounds__(kSNT, 1) k_small(const __grid_constant__ Small
                 if (stamp[d] && d < x) continue;  // both ends changed: the lower id handles it
                 M[x] = d;
                 M[d] = x;
-                atomicAdd(&s_pairs[sl], 1);
-                // neighbours that proposed to x or d rescan next round
+                ++mypairs;
+                // neighbours that proposed to x or d rescan next round: four arcs at a time
+                // (independent loads), one list reservation per four arcs
 #pragma unroll 1
                 for (int e = 0; e < 2; ++e) {
                     const int32_t y0 = e ? d : x, other = e ? x : d;
-                    for (int32_t j = adjp[y0]; j < adjp[y0 + 1]; ++j) {
-                        const int32_t y = adjncy[j];
-                        if (y != other && P[y] == y0) Rn[atomicAdd(&s_rn[sl], 1)] = y;
+                    const int32_t j1 = adjp[y0 + 1];
+                    for (int32_t j = adjp[y0]; j < j1; j += 4) {
+                        int32_t y[4], py[4];
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) y[q] = j + q < j1 ? adjncy[j + q] : other;
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) py[q] = y[q] != other ? P[y[q]] : -1;
+                        int32_t c = 0;
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) c += py[q] == y0;
+                        if (c) {
+                            int32_t w = atomicAdd(&s_rn[sl], c);
+#pragma unroll
+                            for (int q = 0; q < 4; ++q)
+                                if (py[q] == y0) Rn[w++] = y[q];
+                        }
                     }
                 }
             }
+            if (mypairs) atomicAdd(&s_pairs[sl], mypairs);
             GP_SCK(1);
             __syncthreads();
             GP_SCK(2);
