@@ -77,7 +77,10 @@ struct MatchArgs {
     int32_t mode;  // kMatchWhole, or one launch per phase for the sharded path
     int32_t k;     // round of a kMatchRound launch
     uint32_t tie_seed;  // 0: lower id wins ties (north_star); else RM tie priority (R17, P18.s8)
+    int32_t hub_deg_small, hub_small_n;  // levels of <= hub_small_n vertices send rescans of rows
+                                         // longer than hub_deg_small to the hub phase (knobs)
 };
+__shared__ int32_t g_hubdeg;  // this launch's hub threshold (kHubDeg or hub_deg_small)
 
 
 struct MatchSmem {
@@ -644,7 +647,7 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
         if (need) {
             s = rs0;
             e = re0;
-            if (e - s > kHubDeg) {
+            if (e - s > g_hubdeg) {
                 if (gl == 0) {
                     const int32_t h = atomicAdd(&next->nhub, 1);
                     a.H[h] = u;
@@ -704,12 +707,15 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
 // list.  All 32 lanes call; fq lives in the phase-0 staging buffers (idle in phase k).
 constexpr int kFQ = 128;  // queue entries per warp (32 lanes x kVL <= 4)
 constexpr int kFB = 8;    // flat items per lane per batch (256 per warp batch)
+#ifndef GP_KFB1
+#define GP_KFB1 8         // items per lane per batch of the kVL = 1 groups (build-time A/B)
+#endif
 struct FlatQ {
     unsigned long long a1[kFQ], a2[kFQ];          // running top-2 of rows spanning batches
     uint32_t w1[kFQ], n1[kFQ], w2[kFQ], n2[kFQ];  // the batch's top-2 per row: (weight, tie word)
     int32_t s[kFQ];                               // row start (arc index)
     int32_t off[kFQ + 2];                         // row offset in the flat item space
-    uint8_t own[32 * kFB];                        // queue entry of every item of the batch
+    uint8_t own[32 * (kFB > GP_KFB1 ? kFB : GP_KFB1)];  // queue entry of every item of the batch
 };
 // the queues live in adj[1..2], wgt[0..2] and ap[0..2] (contiguous in MatchSmem)
 static_assert(sizeof(FlatQ) * (kNT / 32) <=
@@ -720,7 +726,7 @@ __device__ __forceinline__ unsigned long long wn_key(uint32_t w, uint32_t n) {
     return w ? (((unsigned long long)w << 32) | n) : 0ull;
 }
 
-template <int kVL, bool H, int KFB = (kVL == 1 ? kFB : 4)>
+template <int kVL, bool H, int KFB = (kVL == 1 ? GP_KFB1 : 4)>
 __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, const int32_t *Pk, int32_t *Pn,
                                             int32_t *Pkw, RoundSlot *next, const int32_t (&u)[kVL],
                                             bool (&need)[kVL], bool (&live)[kVL], unsigned long long &scanned,
@@ -735,7 +741,7 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
         if (i < i0 || i >= i1) continue;  // (warp-uniform)
         int32_t d = need[i] ? re[i] - rs[i] : 0;
         if (need[i]) ++rows;
-        if (need[i] && d > kHubDeg) {
+        if (need[i] && d > g_hubdeg) {
             const int32_t h = atomicAdd(&next->nhub, 1);
             a.H[h] = u[i];
             if (a.hk) a.hk[h] = 0ull;  // (sharded launches: per-CTA hub_phase, no hk)
@@ -1081,7 +1087,10 @@ __global__ void __launch_bounds__(kNT, 2) k_match_level(const __grid_constant__ 
         const long long want = ((long long)n + a.vpc - 1) / a.vpc;
         const int nact = (int)(want < 1 ? 1 : (want < (long long)gridDim.x ? want : (long long)gridDim.x));
         if ((int)blockIdx.x >= nact) return;  // retired: this level is too small for it
-        if (threadIdx.x == 0) g_nact = nact;
+        if (threadIdx.x == 0) {
+            g_nact = nact;
+            g_hubdeg = (n <= a.hub_small_n && a.hub_deg_small > 0 && a.hub_deg_small < kHubDeg) ? a.hub_deg_small : kHubDeg;
+        }
         __syncthreads();
     }
     unsigned long long scanned = 0, rows = 0, visits = 0;
@@ -1302,6 +1311,11 @@ gp_status enqueue_match(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl
     a.tie_seed = ctx->tie_seed;
     a.leftover = leftover ? 1 : 0;
     a.G = choose_group(avg_deg_hint);
+    {
+        const char *e1 = getenv("GP_HUB_DEG_SMALL"), *e2 = getenv("GP_HUB_SMALL_N");  // tuning knobs
+        a.hub_deg_small = e1 ? atoi(e1) : kHubDeg;
+        a.hub_small_n = e2 ? atoi(e2) : 0;
+    }
     a.vpc = match_vpc();
     {
         static int lm = -1;

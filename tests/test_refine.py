@@ -179,3 +179,32 @@ def test_gpu_uncoarsen_equals_oracle(gp, ctx, name, k):
     assert np.array_equal(out.cpu().numpy(), ref) and mv == moves
     H.close()
     Gr.close()
+
+
+@pytest.mark.gpu
+def test_gpu_refine_rejects_bad_input(gp, ctx):
+    g = G.grid2d(8, 8)
+    d = {kk: g[kk].cuda() for kk in ("adjp", "adjncy", "adjwgt", "vwgt")}
+    Gr = gp.Graph.create(ctx, d["adjp"], d["adjncy"], d["adjwgt"], d["vwgt"])
+    part = torch.zeros(64, dtype=torch.int32, device="cuda")
+    part[5] = 9  # outside [0, nparts)
+    with pytest.raises(gp.GPError) as e:
+        Gr.refine(part, 4)
+    assert e.value.status == 1
+    for bad_k in (0, 2000):
+        with pytest.raises(gp.GPError):
+            Gr.refine(torch.zeros(64, dtype=torch.int32, device="cuda"), bad_k)
+    # max_passes = 0: nothing moves
+    p0 = (torch.arange(64, device="cuda", dtype=torch.int32) % 4).contiguous()
+    p1 = p0.clone()
+    assert Gr.refine(p1, 4, max_passes=0) == (0, 0) and torch.equal(p0, p1)
+    # gp_uncoarsen needs the hierarchy's own level-0 graph
+    H = Gr.coarsen_to(4)
+    other = gp.Graph.create(ctx, *[G.grid2d(4, 4)[kk].cuda() for kk in ("adjp", "adjncy", "adjwgt", "vwgt")])
+    pc = torch.zeros(H.level(len(H) - 1).n_coarse, dtype=torch.int32, device="cuda")
+    out = torch.empty(64, dtype=torch.int32, device="cuda")
+    with pytest.raises(gp.GPError):
+        H.uncoarsen(other, pc, out, 2)
+    H.close()
+    other.close()
+    Gr.close()
