@@ -1207,7 +1207,14 @@ __device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, i
     }
 }
 
-__global__ void __launch_bounds__(kCNT, 4) k_contract_level(const __grid_constant__ ContractArgs a) {
+// Two instantiations that differ only in __launch_bounds__ (co-resident CTAs per SM):
+// 3 (80 registers, 72 B of spills) and 4 (64 registers, 280 B of spills).  Measured
+// (scripts/r2_minb.sh, r2_fold.sh): 3 is faster on C3 (3.17 vs 3.26 ms) and C2 (2.68 vs
+// 2.81 ms), 4 on the n >= 2^24 graphs, C5 (29.0 vs 29.4 ms) and C4 (495 vs 521 ms: more CTAs in
+// flight for the hub merges); enqueue_contract picks by the level's size bound (kBigLevel).
+constexpr int32_t kBigLevel = 1 << 24;
+template <int kMinB>
+__global__ void __launch_bounds__(kCNT, kMinB) k_contract_level(const __grid_constant__ ContractArgs a) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     // 128-byte alignment by POINTER arithmetic on the __shared__ symbol: the compiler keeps the
     // shared address space (LDS/STS/ATOMS); an integer round trip made every access generic
@@ -1341,20 +1348,34 @@ static int32_t contract_vpc() {
     return v;
 }
 
-int contract_grid(Ctx *ctx) {
+template <int kMinB>
+static int contract_grid_of(Ctx *ctx) {
     // per device: cudaFuncSetAttribute applies to the current device (the ctx's, DeviceGuard)
     static int per_sm_dev[kMaxDevices] = {0};
     int dummy = -1;
     int &per_sm = (ctx->device >= 0 && ctx->device < kMaxDevices) ? per_sm_dev[ctx->device] : dummy;
     if (per_sm <= 0) {
         int b = 0;
-        cudaFuncSetAttribute(k_contract_level, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        cudaFuncSetAttribute(k_contract_level<kMinB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)sizeof(ContractSmem) + 128);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_contract_level, kCNT, sizeof(ContractSmem) + 128);
-        per_sm = b > 0 ? (b > 4 ? 4 : b) : 1;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_contract_level<kMinB>, kCNT, sizeof(ContractSmem) + 128);
+        per_sm = b > 0 ? (b > kMinB ? kMinB : b) : 1;
     }
     const int g = ctx->num_sms * per_sm;
     return g < kMaxContractCtas ? g : kMaxContractCtas;
+}
+
+static bool contract_big(int32_t n_bound) {
+    static int mb = -1;  // GP_CONTRACT_MINB=3|4 forces one instantiation (tuning knob)
+    if (mb < 0) {
+        const char *e = getenv("GP_CONTRACT_MINB");
+        mb = e ? atoi(e) : 0;
+    }
+    return mb == 4 || (mb != 3 && n_bound >= kBigLevel);
+}
+
+int contract_grid(Ctx *ctx, int32_t n_bound) {
+    return contract_big(n_bound) ? contract_grid_of<4>(ctx) : contract_grid_of<3>(ctx);
 }
 
 size_t contract_tiles(int32_t n, int32_t nnz) {
@@ -1423,7 +1444,9 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
     }
     void *args[] = {&a};
     LaunchScope ls(ctx, GP_K_CONTRACT);
-    GP_CUDA(cudaLaunchCooperativeKernel((const void *)k_contract_level, dim3(contract_grid(ctx)), dim3(kCNT), args,
+    const bool big = contract_big(prm.n_bound);
+    GP_CUDA(cudaLaunchCooperativeKernel(big ? (const void *)k_contract_level<4> : (const void *)k_contract_level<3>,
+                                        dim3(contract_grid(ctx, prm.n_bound)), dim3(kCNT), args,
                                         sizeof(ContractSmem) + 128, ctx->stream));
     ++ctx->launches;
     return GP_OK;

@@ -597,6 +597,21 @@ static gp_status split_graph(Ctx *ctx, const Graph *g, int G, std::vector<Shard>
     return GP_OK;
 }
 
+// folding: one rank's piece of the gathered coarse graph -> rows of the full CSR
+__global__ void k_fold_adjp(const int32_t *piece_adjp, int32_t rows, int32_t arc_base, int32_t *full_adjp) {
+    for (int32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < rows; r += gridDim.x * blockDim.x)
+        full_adjp[r] = piece_adjp[r] + arc_base;
+}
+
+// Folding (PT-Scotch's folding, P14.s21-23): once the coarse graph has at
+// most GP_FOLD_N vertices (default 500 000; 0 = never), every rank gathers it whole and finishes
+// the hierarchy on the single-GPU pipeline (tail kernels included) -- redundantly on every
+// rank, with no per-round collective.  The results are the 1-GPU results by construction.
+static int32_t fold_limit() {
+    const char *e = getenv("GP_FOLD_N");  // knob read per call (results never depend on it)
+    return e ? atoi(e) : 500000;
+}
+
 // per-rank working state of one level
 struct RankWork {
     Shard sh;
@@ -976,7 +991,7 @@ gp_status dist_coarsen_to(Graph *g0, const gp_coarsen_opts *opts, Hier **out) {
                     *ttot = nullptr;
             unsigned long long *gkeys = nullptr, *tout = nullptr;
             int32_t tb = kContractTileBudget;
-            while (tb > 32 && (long long)ubn < 4LL * tb * contract_grid(ctx) * 8) tb >>= 1;
+            while (tb > 32 && (long long)ubn < 4LL * tb * contract_grid(ctx, w.nloc) * 8) tb >>= 1;
             const int32_t ntiles2 = ubn > 0 ? (ubn + tb - 1) / tb : 0;
             st = ar.get(&seg, nc);
             if (st == GP_OK) st = ar.get(&ub, (size_t)nc + 1);
@@ -1065,6 +1080,129 @@ gp_status dist_coarsen_to(Graph *g0, const gp_coarsen_opts *opts, Hier **out) {
         return st;
     };
 
+    // gather the (small) coarse graph onto every rank and finish on the single-GPU pipeline
+    auto fold = [&](int levels_done) -> gp_status {
+        std::vector<long long> rows(G), arcs(G), abase(G + 1, 0);
+        for (int r = 0; r < G; ++r) rows[r] = ranges[r + 1] - ranges[r];
+        if (comm->loopback()) {
+            for (int i = 0; i < NL; ++i) arcs[i] = shards[i].g->nnz;
+        } else {
+            int32_t mine = shards[0].g->nnz;
+            std::vector<int32_t> all(G);
+            gp_status s2 = dist_allgather_i32(ctx, &mine, 1, all.data());
+            if (s2 != GP_OK) return s2;
+            for (int r = 0; r < G; ++r) arcs[r] = all[r];
+        }
+        long long maxr = 0, maxa = 0;
+        for (int r = 0; r < G; ++r) {
+            maxr = std::max(maxr, rows[r]);
+            maxa = std::max(maxa, arcs[r]);
+            abase[r + 1] = abase[r] + arcs[r];
+        }
+        const long long PS = (maxr + 4) + (maxr + 4) + 2 * (maxa + 4);  // adjp | vwgt | adjncy | adjwgt
+        const long long oV = maxr + 4, oA = 2 * (maxr + 4), oW = oA + maxa + 4;
+        Arena ar(ctx);
+        std::vector<int32_t *> vs(NL), vr(NL);
+        for (int i = 0; i < NL; ++i) {
+            gp_status s2 = ar.get(&vs[i], (size_t)PS);
+            if (s2 == GP_OK) s2 = ar.get(&vr[i], (size_t)PS * G);
+            if (s2 != GP_OK) return s2;
+            const Graph *sg = shards[i].g;
+            GP_CUDA(cudaMemcpyAsync(vs[i], sg->adjp, sizeof(int32_t) * ((size_t)sg->n + 1), cudaMemcpyDeviceToDevice,
+                                    ctx->stream));
+            if (sg->n > 0)
+                GP_CUDA(cudaMemcpyAsync(vs[i] + oV, sg->vwgt, sizeof(int32_t) * (size_t)sg->n, cudaMemcpyDeviceToDevice,
+                                        ctx->stream));
+            if (sg->nnz > 0) {
+                GP_CUDA(cudaMemcpyAsync(vs[i] + oA, sg->adjncy, sizeof(int32_t) * (size_t)sg->nnz,
+                                        cudaMemcpyDeviceToDevice, ctx->stream));
+                GP_CUDA(cudaMemcpyAsync(vs[i] + oW, sg->adjwgt, sizeof(int32_t) * (size_t)sg->nnz,
+                                        cudaMemcpyDeviceToDevice, ctx->stream));
+            }
+        }
+        gp_status s2 = allgather(ctx, vs, vr, (size_t)PS);
+        if (s2 != GP_OK) return s2;
+        // the whole coarse graph on this process (every local rank would hold the same bytes)
+        Graph *fg = new Graph();
+        fg->ctx = ctx;
+        fg->n = N;
+        fg->nnz = (int32_t)NNZ;
+        s2 = alloc_graph_arrays(ctx, fg, N, (int32_t)NNZ, true);
+        for (int r = 0; s2 == GP_OK && r < G; ++r) {
+            const int32_t *pc = vr[0] + (size_t)r * PS;
+            if (rows[r] > 0) {
+                GP_LAUNCH(k_fold_adjp<<<grid_for(rows[r]), kDT, 0, ctx->stream>>>(pc, (int32_t)rows[r], (int32_t)abase[r],
+                                                                                 fg->adjp + ranges[r]));
+                GP_CUDA(cudaMemcpyAsync(fg->vwgt + ranges[r], pc + oV, sizeof(int32_t) * (size_t)rows[r],
+                                        cudaMemcpyDeviceToDevice, ctx->stream));
+            }
+            if (arcs[r] > 0) {
+                GP_CUDA(cudaMemcpyAsync(fg->adjncy + abase[r], pc + oA, sizeof(int32_t) * (size_t)arcs[r],
+                                        cudaMemcpyDeviceToDevice, ctx->stream));
+                GP_CUDA(cudaMemcpyAsync(fg->adjwgt + abase[r], pc + oW, sizeof(int32_t) * (size_t)arcs[r],
+                                        cudaMemcpyDeviceToDevice, ctx->stream));
+            }
+        }
+        const int32_t tail_words[2] = {(int32_t)NNZ, 0};
+        const SizeRec rec{N, (int32_t)NNZ, 0, 0};
+        if (s2 == GP_OK) {
+            GP_CUDA(cudaMemcpyAsync(fg->adjp + N, tail_words, sizeof(int32_t), cudaMemcpyHostToDevice, ctx->stream));
+            GP_CUDA(cudaMemcpyAsync(fg->sizes, &rec, sizeof(rec), cudaMemcpyHostToDevice, ctx->stream));
+            GP_CUDA(cudaStreamSynchronize(ctx->stream));  // host words leave scope; the arena is freed
+        }
+        Hier *sub = nullptr;
+        gp_coarsen_opts o2 = *opts;
+        o2.max_levels = max_levels - levels_done;
+        o2.stall_ratio_pct = pct;
+        if (s2 == GP_OK) s2 = coarsen_single(fg, &o2, &sub);
+        cudaStreamSynchronize(ctx->stream);
+        graph_release(fg);
+        if (s2 != GP_OK) return s2;
+        h->subs.push_back(sub);
+        // the folded levels, as sharded levels whose piece on rank 0 is the whole level
+        for (const Level &ls : sub->levels) {
+            Level L;
+            L.n = ls.n;
+            L.nnz = ls.nnz;
+            L.n_coarse = ls.n_coarse;
+            L.cnnz = ls.cnnz;
+            L.rounds = ls.rounds;
+            L.maximal = ls.maximal;
+            L.stop_reason = ls.stop_reason;
+            L.arcs_scanned = ls.arcs_scanned;
+            L.rows_scanned = ls.rows_scanned;
+            L.live_visits = ls.live_visits;
+            L.borrowed = true;
+            for (int i = 0; i < NL; ++i) {
+                DistPiece p;
+                p.rank = comm->grank(i);
+                if (p.rank == 0) {
+                    p.vbase = 0;
+                    p.nloc = ls.n;
+                    p.M = ls.match;
+                    p.CM = ls.cmap;
+                    p.coarse = ls.coarse;
+                } else {  // an empty piece (zero rows, adjp = {0})
+                    Graph *eg = new Graph();
+                    eg->ctx = ctx;
+                    h->extra.push_back(eg);
+                    gp_status s3 = alloc_graph_arrays(ctx, eg, 0, 0, true);
+                    if (s3 != GP_OK) return s3;
+                    GP_CUDA(cudaMemsetAsync(eg->adjp, 0, sizeof(int32_t), ctx->stream));
+                    eg->vbase = ls.n_coarse;
+                    p.vbase = ls.n;  // M + vbase: one past the end of the level's arrays
+                    p.nloc = 0;
+                    p.M = ls.match;
+                    p.CM = ls.cmap;
+                    p.coarse = eg;
+                }
+                L.pieces.push_back(p);
+            }
+            h->levels.push_back(L);
+        }
+        return GP_OK;
+    };
+
     for (int level = 0; st == GP_OK && N > opts->threshold && level < max_levels; ++level) {
         W.assign(NL, RankWork());
         {
@@ -1109,6 +1247,10 @@ gp_status dist_coarsen_to(Graph *g0, const gp_coarsen_opts *opts, Hier **out) {
         NNZ = CNNZ;
         ranges = cranges;
         if (reason != GP_STOP_NONE) break;
+        if (N <= fold_limit() && level + 1 < max_levels) {
+            st = fold(level + 1);
+            break;
+        }
     }
     release_shards();
     if (st != GP_OK) {

@@ -137,6 +137,7 @@ void graph_release(Graph *g) {
 void hier_release(Hier *h) {
     if (!h) return;
     for (auto &l : h->levels) {
+        if (l.borrowed) continue;  // owned by a sub-hierarchy (folded sharded levels)
         if (!l.arena) {
             dev_free(h->ctx, l.match);
             dev_free(h->ctx, l.cmap);
@@ -148,6 +149,8 @@ void hier_release(Hier *h) {
             graph_release(p.coarse);
         }
     }
+    for (Hier *sub : h->subs) hier_release(sub);
+    for (Graph *x : h->extra) graph_release(x);
     dev_free(h->ctx, h->levdev);
     for (void *p : h->arenas) dev_free(h->ctx, p);
     if (h->counted) --h->ctx->live_objects;
@@ -581,18 +584,13 @@ static bool debug_on() {
         }                                         \
     } while (0)
 
-gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
-    if (out) *out = nullptr;
-    if (!tagged<Graph>(g, kTagGraph) || !opts || !out || opts->threshold < 0 || opts->stall_ratio_pct < 0 ||
-        opts->max_levels < 0 || opts->max_rounds < 0) {
-        set_error("gp_coarsen_to: bad graph, options or output");
-        return GP_ERR_INVALID_ARG;
-    }
-    GP_TRY_BEGIN
+}  // extern "C"
+
+namespace gp {
+// the single-GPU level pipeline of gp_coarsen_to (also run by the sharded driver once the graph
+// is folded onto every rank, dist.cu)
+gp_status coarsen_single(Graph *g, const gp_coarsen_opts *opts, Hier **out) {
     Ctx *ctx = g->ctx;
-    DeviceGuard dg(ctx->device);
-    ctx->tie_seed = opts->tie_seed;
-    if (ctx->comm) return dist_coarsen_to(g, opts, out);  // sharded path (dist.cu)
     const int32_t pct = opts->stall_ratio_pct ? opts->stall_ratio_pct : 95;
     int32_t max_levels = opts->max_levels ? opts->max_levels : 64;
     if (max_levels > ctx->max_reports) max_levels = ctx->max_reports;
@@ -856,6 +854,24 @@ gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
     }
     *out = h;
     return GP_OK;
+}
+}  // namespace gp
+
+extern "C" {
+
+gp_status gp_coarsen_to(gp_graph g, const gp_coarsen_opts *opts, gp_hier *out) {
+    if (out) *out = nullptr;
+    if (!tagged<Graph>(g, kTagGraph) || !opts || !out || opts->threshold < 0 || opts->stall_ratio_pct < 0 ||
+        opts->max_levels < 0 || opts->max_rounds < 0) {
+        set_error("gp_coarsen_to: bad graph, options or output");
+        return GP_ERR_INVALID_ARG;
+    }
+    GP_TRY_BEGIN
+    Ctx *ctx = g->ctx;
+    DeviceGuard dg(ctx->device);
+    ctx->tie_seed = opts->tie_seed;
+    if (ctx->comm) return dist_coarsen_to(g, opts, out);  // sharded path (dist.cu)
+    return coarsen_single(g, opts, out);
     GP_TRY_END
 }
 

@@ -166,6 +166,7 @@ struct Level {
     Graph *coarse = nullptr;
     std::vector<DistPiece> pieces;  // sharded levels: one piece per local rank
     bool arena = false;             // match / cmap / coarse arrays live in a hierarchy arena
+    bool borrowed = false;          // folded sharded level: its arrays belong to a sub-hierarchy
 };
 }  // namespace gp
 
@@ -176,6 +177,8 @@ struct gp_hier_s {
     gp::LevelDev *levdev = nullptr;  // per-level control blocks (coarse graphs' size records)
     bool counted = false;  // included in ctx->live_objects
     std::vector<void *> arenas;  // device arenas of tail levels (small.cu), freed with the hierarchy
+    std::vector<gp_hier_s *> subs;        // folded levels of a sharded hierarchy (dist.cu)
+    std::vector<gp_graph_s *> extra;      // empty coarse pieces of folded levels
 };
 
 struct gp_ctx_s {
@@ -273,7 +276,7 @@ struct ContractParams {
     int32_t dist = 0, cbase = 0, tb = 0, nnz_ub = 0;
 };
 constexpr int kContractTileBudget = 256;  // C2 warp-tile budget (upper-bound entries), kWB
-int contract_grid(Ctx *ctx);
+int contract_grid(Ctx *ctx, int32_t n_bound);
 gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *CM, Graph *coarse, ContractCtl *ctl,
                            SizeRec *out_sizes, LevelReport *report, const ContractParams &prm);
 size_t contract_tiles(int32_t n, int32_t nnz);
@@ -335,6 +338,8 @@ gp_status enqueue_project(Ctx *ctx, const int32_t *const *cms, int nlev, int32_t
 
 // sharded path (dist.cu)
 gp_status dist_coarsen_to(Graph *g, const gp_coarsen_opts *opts, Hier **out);
+// the single-GPU level pipeline (gp_abi.cu); ctx->tie_seed must be set
+gp_status coarsen_single(Graph *g, const gp_coarsen_opts *opts, Hier **out);
 gp_status dist_comm_create_nccl(Ctx *ctx, const void *uid, int rank, int nranks);
 gp_status dist_comm_create_loopback(Ctx *ctx, int nranks);
 void dist_comm_destroy(Ctx *ctx);

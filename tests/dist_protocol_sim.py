@@ -278,12 +278,37 @@ def contract_level(sh: Shard, M: np.ndarray):
     return CM, coarse
 
 
+def fold(sh: Shard) -> Shard:
+    """Folding (csrc/dist.cu fold): every rank gathers the coarse pieces --
+    rows (adjp shifted by the arc base of the rank) | vwgt | adjncy | adjwgt -- and the rest of
+    the hierarchy runs on the whole graph.  Here that graph is re-sharded onto rank 0 (the
+    piece layout the CUDA driver reports for folded levels: rank 0 owns every vertex)."""
+    G, me = dist.get_world_size(), dist.get_rank()
+    rows = _allgather_rows(np.stack([sh.adjp[1:] - sh.adjp[:-1], sh.vwgt], axis=1) if sh.nloc else
+                           np.zeros((0, 2), dtype=np.int64), 2)
+    arcs = _allgather_rows(np.stack([sh.adjncy, sh.adjwgt], axis=1) if len(sh.adjncy) else
+                           np.zeros((0, 2), dtype=np.int64), 2)
+    deg = np.concatenate([r[:, 0] for r in rows]).astype(np.int64)
+    assert len(deg) == sh.N
+    adjp = np.concatenate([[0], np.cumsum(deg)]).astype(np.int64)
+    vwgt = np.concatenate([r[:, 1] for r in rows]).astype(np.int64)
+    adjncy = np.concatenate([a[:, 0] for a in arcs]).astype(np.int64)
+    adjwgt = np.concatenate([a[:, 1] for a in arcs]).astype(np.int64)
+    ranges = np.array([0] + [sh.N] * G, dtype=np.int64)
+    if me == 0:
+        return Shard(sh.N, 0, adjp, adjncy, adjwgt, vwgt, ranges)
+    e = np.zeros(0, dtype=np.int64)
+    return Shard(sh.N, sh.N, np.zeros(1, dtype=np.int64), e, e, e, ranges)
+
+
 def coarsen_to(sh: Shard, threshold: int, stall_ratio_pct: int = 95, max_levels: int = 64, max_rounds: int = 0,
-               tie_seed: int = 0):
-    """Levels of this rank: list of dicts with the rank's slices of M / CM and coarse piece."""
+               tie_seed: int = 0, fold_n: int = 0):
+    """Levels of this rank: list of dicts with the rank's slices of M / CM and coarse piece.
+    fold_n > 0: fold once a coarse graph has at most fold_n vertices (csrc/dist.cu GP_FOLD_N)."""
     global TIE_SEED
     TIE_SEED = tie_seed & 0xFFFFFFFF
     levels = []
+    folded = False
     while sh.N > threshold and len(levels) < max_levels:
         M, rounds, maximal = match_level(sh, max_rounds)
         CM, cg = contract_level(sh, M)
@@ -294,4 +319,7 @@ def coarsen_to(sh: Shard, threshold: int, stall_ratio_pct: int = 95, max_levels:
         sh = cg
         if stall:
             break
+        if fold_n > 0 and not folded and sh.N <= fold_n and sh.N > threshold and len(levels) < max_levels:
+            sh = fold(sh)
+            folded = True
     return levels

@@ -39,7 +39,7 @@ def _graphs():
     }
 
 
-def _worker(rank, world, port, out_dir, threshold, max_rounds, tie_seed=0):
+def _worker(rank, world, port, out_dir, threshold, max_rounds, tie_seed=0, fold_n=0):
     try:
         sys.path.insert(0, ROOT)
         sys.path.insert(0, os.path.join(ROOT, "tests"))
@@ -54,7 +54,7 @@ def _worker(rank, world, port, out_dir, threshold, max_rounds, tie_seed=0):
         for name, g in _graphs().items():
             g = {k: (v.numpy() if hasattr(v, "numpy") else v) for k, v in g.items()}
             levels = sim.coarsen_to(sim.shard_of(g, rank, world), threshold, max_rounds=max_rounds,
-                                    tie_seed=tie_seed)
+                                    tie_seed=tie_seed, fold_n=fold_n)
             pieces = [None] * world
             dist.all_gather_object(pieces, [{"n": l["n"], "rounds": l["rounds"], "maximal": l["maximal"],
                                              "match": l["match"], "cmap": l["cmap"], "n_coarse": l["n_coarse"],
@@ -91,12 +91,16 @@ def _concat(pieces, i):
             "rounds": lv[0]["rounds"], "maximal": lv[0]["maximal"], "n_coarse": lv[0]["n_coarse"]}
 
 
-@pytest.mark.parametrize("world,max_rounds,tie_seed", [(2, 0, 0), (3, 0, 0), (2, 2, 0), (2, 0, 0x9E3779B9)])
-def test_sharded_protocol_equals_oracle(tmp_path, world, max_rounds, tie_seed):
+@pytest.mark.parametrize("world,max_rounds,tie_seed,fold_n", [(2, 0, 0, 0), (3, 0, 0, 0), (2, 2, 0, 0),
+                                                             (2, 0, 0x9E3779B9, 0), (2, 0, 0, 40), (3, 2, 0, 60)])
+def test_sharded_protocol_equals_oracle(tmp_path, world, max_rounds, tie_seed, fold_n):
+    """fold_n > 0: the sharded levels until the coarse graph has <= fold_n vertices, then the
+    gathered graph (re-sharded onto rank 0) for the rest: the same hierarchy."""
     import oracle
 
     port = _free_port()
-    mp.start_processes(_worker, args=(world, port, str(tmp_path), 8, max_rounds, tie_seed), nprocs=world, join=True,
+    mp.start_processes(_worker, args=(world, port, str(tmp_path), 8, max_rounds, tie_seed, fold_n), nprocs=world,
+                       join=True,
                        start_method="spawn")
     errs = [p for p in os.listdir(tmp_path) if p.startswith("error")]
     assert not errs, open(os.path.join(tmp_path, errs[0])).read()

@@ -29,9 +29,15 @@ def _levels(gp, H):
     return out
 
 
-def test_nccl_transport_one_rank(gp):
+@pytest.mark.parametrize("fold", ["off", "default"])
+def test_nccl_transport_one_rank(gp, fold, monkeypatch):
     """gp_ctx_create_dist with a real (1-rank) NCCL communicator: gp_graph_create_dist, the
-    sharded driver's ncclAllGather / grouped send-recv calls, bit-exact vs the oracle."""
+    sharded driver's ncclAllGather / grouped send-recv calls, bit-exact vs the oracle; with
+    folding on, the gather of the coarse graph is an ncclAllGather too."""
+    if fold == "off":
+        monkeypatch.setenv("GP_FOLD_N", "0")
+    else:
+        monkeypatch.delenv("GP_FOLD_N", raising=False)
     uid = gp.nccl_unique_id()
     ctx = gp.Context(0, nccl_id=uid, rank=0, nranks=1)
     assert ctx.dist_info() == (0, 1)
