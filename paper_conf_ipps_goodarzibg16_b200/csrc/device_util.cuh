@@ -299,13 +299,25 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned parity) {
     const long long guard = spin_start();
     while (!mbar_try_wait(bar, parity)) spin_check(guard);
 }
+#ifndef GP_L2HINT
+#define GP_L2HINT 1  // L2 cache-policy hints on streamed arcs (match.cu ldArc)
+#endif
 // bytes must be a multiple of 16; src and dst 16-byte aligned
 __device__ __forceinline__ void tma_load_1d(void *dst, const void *src, unsigned bytes, uint64_t *bar) {
+#if GP_L2HINT >= 1
+    asm volatile(
+        "{\n\t.reg .b64 pol;\n\tcreatepolicy.fractional.L2::evict_first.b64 pol, 1.0;\n\t"
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], pol;\n\t}" ::"r"(
+            smem_addr(dst)),
+        "l"(src), "r"(bytes), "r"(smem_addr(bar))
+        : "memory");
+#else
     asm volatile(
         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
             smem_addr(dst)),
         "l"(src), "r"(bytes), "r"(smem_addr(bar))
         : "memory");
+#endif
 }
 
 }  // namespace gp

@@ -106,10 +106,35 @@ __device__ __forceinline__ int32_t ldcg(const int32_t *p) { return __ldcg(p); }
 // only writes within a phase mark dead vertices NONE, which a stale read cannot turn into a
 // handshake).  Measured equal on C3 / C2 / C5 (3.31 vs 3.30, 2.80 vs 2.82, 29.5 vs 29.0 ms):
 // the mesh locality of these gathers is already captured by coalescing within a warp.
-#ifdef GP_P_CA
+#if defined(GP_P_CA)
 __device__ __forceinline__ int32_t ldP(const int32_t *p) { return __ldca(p); }
+#elif GP_L2HINT >= 2
+// GP_L2HINT=2: the gathered proposal arrays carry an L2 evict_last policy (C3 level 0:
+// P[2] + S + M = 64 MB of the 126 MB L2)
+__device__ __forceinline__ int32_t ldP(const int32_t *p) {
+    int32_t v;
+    asm("{\n\t.reg .b64 pol;\n\tcreatepolicy.fractional.L2::evict_last.b64 pol, 1.0;\n\t"
+        "ld.global.cg.L2::cache_hint.s32 %0, [%1], pol;\n\t}" : "=r"(v) : "l"(p));
+    return v;
+}
 #else
 __device__ __forceinline__ int32_t ldP(const int32_t *p) { return __ldcg(p); }
+#endif
+// GP_L2HINT >= 1 (default): the streamed arcs (rescans, phase-0 TMA stages) carry an L2
+// evict_first policy so that they do not push the gathered proposal arrays out of L2.
+// Measured (scripts/r2_l2hint.sh): C3 3.17 -> 3.11 ms (level-0 match 441 -> 420 us), C5
+// unchanged; adding evict_last on the P / S gathers (=2) was slower than arcs alone (3.14 ms),
+// and an L2 set-aside for it (cudaLimitPersistingL2CacheSize 64 MB) slower still (3.36 ms,
+// C5 34 ms).  GP_L2HINT=0 at build time removes the hints.
+#if GP_L2HINT >= 1
+__device__ __forceinline__ int32_t ldArc(const int32_t *p) {
+    int32_t v;
+    asm("{\n\t.reg .b64 pol;\n\tcreatepolicy.fractional.L2::evict_first.b64 pol, 1.0;\n\t"
+        "ld.global.nc.L2::cache_hint.s32 %0, [%1], pol;\n\t}" : "=r"(v) : "l"(p));
+    return v;
+}
+#else
+__device__ __forceinline__ int32_t ldArc(const int32_t *p) { return __ldg(p); }
 #endif
 __device__ __forceinline__ int4 ld_volatile_v4(const int4 *p) {
     int4 v;
@@ -296,8 +321,8 @@ __device__ void phase0(const MatchArgs &a, MatchSmem &sm, int32_t n, unsigned lo
 #pragma unroll
                         for (int q = 0; q < 8; ++q) {
                             const int32_t j = j0 + q * G;
-                            xv[q] = j < e ? __ldg(a.adjncy + j) : -1;
-                            wv[q] = j < e ? __ldg(a.adjwgt + j) : 0;
+                            xv[q] = j < e ? ldArc(a.adjncy + j) : -1;
+                            wv[q] = j < e ? ldArc(a.adjwgt + j) : 0;
                         }
 #pragma unroll
                         for (int q = 0; q < 8; ++q)
@@ -353,8 +378,8 @@ __device__ __noinline__ void hub_phase(const MatchArgs &a, MatchSmem &sm, int32_
         const int32_t s = __ldg(a.adjp + (u - a.vbase)), e = __ldg(a.adjp + (u - a.vbase) + 1);
         unsigned long long key = 0;
         for (int32_t j = s + threadIdx.x; j < e; j += kNT) {
-            const int32_t x = __ldg(a.adjncy + j);
-            if (!check || free_after(x, Pk)) key = umax64(key, pack_key<H>(a.tie_seed, __ldg(a.adjwgt + j), x));
+            const int32_t x = ldArc(a.adjncy + j);
+            if (!check || free_after(x, Pk)) key = umax64(key, pack_key<H>(a.tie_seed, ldArc(a.adjwgt + j), x));
         }
         key = group_max64<32>(key);
         if (lane == 0) sm.red[wib] = key;
@@ -421,8 +446,8 @@ __device__ __noinline__ void hub_phase_mc(const MatchArgs &a, MatchSmem &sm, int
 #pragma unroll
             for (int q = 0; q < 8; ++q) {
                 const int32_t j = c0 + q * kNT + t;
-                x[q] = j < c1 ? __ldg(a.adjncy + j) : -1;
-                w[q] = j < c1 ? __ldg(a.adjwgt + j) : 0;
+                x[q] = j < c1 ? ldArc(a.adjncy + j) : -1;
+                w[q] = j < c1 ? ldArc(a.adjwgt + j) : 0;
             }
             unsigned long long key = 0;
             if (check) {
@@ -559,7 +584,7 @@ __device__ __noinline__ void wake_phase(const MatchArgs &a, MatchSmem &sm, int32
 #pragma unroll
             for (int q = 0; q < 8; ++q) {
                 const int32_t j = c0 + q * kNT + t;
-                x[q] = j < c1 ? __ldg(a.adjncy + j) : -1;
+                x[q] = j < c1 ? ldArc(a.adjncy + j) : -1;
             }
 #pragma unroll
             for (int q = 0; q < 8; ++q) px[q] = x[q] >= 0 ? ldP(Pk + x[q]) : -1;
@@ -670,8 +695,8 @@ __device__ void phase_k_lanes(const MatchArgs &a, MatchSmem &sm, int k, int32_t 
 #pragma unroll
             for (int b = 0; b < 4; ++b) {
                 const int32_t j = s + (t * 4 + b) * G + gl;
-                x[b] = (need && j < e) ? __ldg(a.adjncy + j) : -1;
-                w[b] = (need && j < e) ? __ldg(a.adjwgt + j) : 0;
+                x[b] = (need && j < e) ? ldArc(a.adjncy + j) : -1;
+                w[b] = (need && j < e) ? ldArc(a.adjwgt + j) : 0;
             }
 #pragma unroll
             for (int b = 0; b < 4; ++b) px[b] = x[b] >= 0 ? ldP(Pk + x[b]) : -1;
@@ -787,8 +812,8 @@ __device__ __forceinline__ void flat_rescan(const MatchArgs &a, MatchSmem &sm, c
             if (f < bn) {
                 const int32_t r = fq.own[f];
                 const int32_t j = fq.s[r] + (b0 + f - fq.off[r]);
-                x[b] = __ldg(a.adjncy + j);
-                w[b] = __ldg(a.adjwgt + j);
+                x[b] = ldArc(a.adjncy + j);
+                w[b] = ldArc(a.adjwgt + j);
             }
         }
 #pragma unroll
