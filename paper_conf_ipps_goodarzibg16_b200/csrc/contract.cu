@@ -139,11 +139,13 @@ template <typename Sync>
 __device__ __forceinline__ void coop_sort(unsigned long long *keys, int len, int tid, int nthr, Sync sync) {
     int S = 1;
     while (S < len) S <<= 1;
-    for (int size = 2; size <= S; size <<= 1) {
-        const int half = size >> 1;
+    // power-of-two strides: index arithmetic by shifts and masks (a runtime division per
+    // comparator was most of the instruction count of the C1h sorts)
+    for (int lh = 0; (2 << lh) <= S; ++lh) {
+        const int size = 2 << lh, half = 1 << lh;
         for (int i = tid; i < S / 2; i += nthr) {
-            const int blk = i / half, o = i % half;
-            const int x = blk * size + o, y = blk * size + size - 1 - o;
+            const int base = (i >> lh) << (lh + 1), o = i & (half - 1);
+            const int x = base + o, y = base + size - 1 - o;
             if (y < len) {
                 const unsigned long long p = keys[x], q = keys[y];
                 if (p > q) {
@@ -153,9 +155,10 @@ __device__ __forceinline__ void coop_sort(unsigned long long *keys, int len, int
             }
         }
         sync();
-        for (int j = size / 4; j > 0; j >>= 1) {
+        for (int lj = lh - 1; lj >= 0; --lj) {
+            const int j = 1 << lj;
             for (int i = tid; i < S / 2; i += nthr) {
-                const int x = (i / j) * 2 * j + (i % j), y = x + j;
+                const int x = ((i >> lj) << (lj + 1)) + (i & (j - 1)), y = x + j;
                 if (y < len) {
                     const unsigned long long p = keys[x], q = keys[y];
                     if (p > q) {
@@ -1106,6 +1109,7 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
             if (!sp1) {
                 a.ttot[wt] = run;
                 atomicAdd(&a.ctl->chunk2[wt / T2], run);
+                if (run > kBigTile) a.ctl->big_flag = 1;  // read by every CTA after the grid barrier
             }
             wt = nw + (int)atomicAdd(&a.ctl->tile_ctr, 1u);
         }
@@ -1115,7 +1119,8 @@ __device__ void phase_c2a(const ContractArgs &a, ContractSmem &sm, int32_t ntile
 // ---------------------------------------------------------------------------------------
 // C2b: cadjp + coalesced copy of the tiles of this CTA's chunk into the final CSR
 // ---------------------------------------------------------------------------------------
-__device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, int32_t ntiles2, int T2, int32_t rt) {
+__device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, int32_t ntiles2, int T2, int32_t rt,
+                          bool balanced) {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int t_lo = blockIdx.x * T2, t_hi = min(ntiles2, t_lo + T2);
     if (t_lo >= t_hi) return;
@@ -1143,7 +1148,14 @@ __device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, i
         const int32_t total = __ldcg(a.ttot + t);
         for (int32_t c = r0 + lane; c < r1; c += 32) a.cadjp[c] = p + __ldcg(a.lofs + c);
         bool big = false;
-        if (r0 < r1 && total > kBigTile) {
+        if (balanced && r0 < r1 && total > kBigTile) {
+            // listed for phase_c2b_big: its entries are copied by all CTAs in equal shares
+            if (lane == 0) {
+                const unsigned i = atomicAdd(&a.ctl->big_ctr, 1u);
+                a.seg[i] = make_int4(p, total, __ldcg(a.off + r0), 0);  // seg is idle after C2a
+            }
+            big = true;
+        } else if (r0 < r1 && total > kBigTile) {
             int slot = 0;
             if (lane == 0) slot = atomicAdd(&sm.len, 1);
             slot = __shfl_sync(0xffffffffu, slot, 0);
@@ -1178,7 +1190,7 @@ __device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, i
         }
     }
     __syncthreads();
-    const int nbig = min(sm.len, kCNT);
+    const int nbig = balanced ? 0 : min(sm.len, kCNT);
     for (int b = 0; b < nbig; ++b) {  // whole-CTA copies, 8 keys per thread in flight
         const int t = sm.lead[b];
         const int32_t p = tp[t - s_lo];
@@ -1204,6 +1216,55 @@ __device__ void phase_c2b(const ContractArgs &a, ContractSmem &sm, int32_t nc, i
         }
     }
     __syncthreads();
+    }
+}
+
+// ---------------------------------------------------------------------------------------
+// C2b, big tiles (R-MAT: tiles holding hub rows, clustered at the low coarse ids, so the
+// static tile chunks of C2b left one CTA copying ~10^8 entries -- 18-33 ms per C4 level): the
+// listed tiles' entries are concatenated and every CTA copies an equal share
+// ---------------------------------------------------------------------------------------
+__device__ void phase_c2b_big(const ContractArgs &a, ContractSmem &sm) {
+    const int32_t nb = (int32_t)*(volatile unsigned *)&a.ctl->big_ctr;
+    int32_t *pre = reinterpret_cast<int32_t *>(sm.buf);  // exclusive prefix of the chunk's totals
+    constexpr int kCap = 2 * kBuf - 1;
+    for (int32_t c0 = 0; c0 < nb; c0 += kCap) {
+        const int cnt = min(kCap, nb - c0);
+        const int32_t T = block_scan_list(sm, reinterpret_cast<const int32_t *>(a.seg + c0), 4, 1, cnt, 0, pre);
+        if (threadIdx.x == 0) pre[cnt] = T;
+        __syncthreads();
+        const long long e0 = (long long)T * blockIdx.x / g_cact, e1 = (long long)T * (blockIdx.x + 1) / g_cact;
+        // first listed tile holding entry e0: the last i with pre[i] <= e0
+        int lo = 0, hi = cnt - 1;
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (pre[mid] <= e0) lo = mid;
+            else hi = mid - 1;
+        }
+        for (int i = lo; i < cnt && pre[i] < e1; ++i) {
+            const int4 b = __ldcg(a.seg + c0 + i);  // {p, total, tout offset}
+            const int32_t j0 = (int32_t)max((long long)pre[i], e0) - pre[i];
+            const int32_t j1 = (int32_t)(min((long long)pre[i] + b.y, e1) - pre[i]);
+            const unsigned long long *src = a.tout + b.z;
+            constexpr int kB = 8;
+            for (int32_t jb = j0; jb < j1; jb += kCNT * kB) {
+                unsigned long long k[kB];
+#pragma unroll
+                for (int q = 0; q < kB; ++q) {
+                    const int32_t j = jb + q * kCNT + threadIdx.x;
+                    k[q] = j < j1 ? __ldcs(src + j) : 0ull;
+                }
+#pragma unroll
+                for (int q = 0; q < kB; ++q) {
+                    const int32_t j = jb + q * kCNT + threadIdx.x;
+                    if (j < j1) {
+                        a.cadjncy[b.x + j] = (int32_t)(k[q] >> 32);
+                        a.cadjwgt[b.x + j] = (int32_t)(uint32_t)k[q];
+                    }
+                }
+            }
+        }
+        __syncthreads();  // pre[] is rebuilt for the next chunk
     }
 }
 
@@ -1295,7 +1356,12 @@ __global__ void __launch_bounds__(kCNT, kMinB) k_contract_level(const __grid_con
         if (!single_pass) {
             grid_barrier(ctl->bar, bar_epoch, g_cact);
             trace_mark(ctl->trace, 7);
-            phase_c2b(a, sm, nc, ntiles2, T2, rt);
+            const bool balanced = *(volatile int32_t *)&ctl->big_flag != 0;  // uniform after the barrier
+            phase_c2b(a, sm, nc, ntiles2, T2, rt, balanced);
+            if (balanced) {
+                grid_barrier(ctl->bar, bar_epoch, g_cact);
+                phase_c2b_big(a, sm);
+            }
         }
     } else {  // no arcs: every coarse row is empty
         for (long long c = (long long)blockIdx.x * kCNT + threadIdx.x; c <= nc; c += (long long)g_cact * kCNT)

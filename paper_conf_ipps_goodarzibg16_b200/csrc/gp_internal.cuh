@@ -73,6 +73,8 @@ struct ContractCtl {
     unsigned blocks_done;
     unsigned tile_ctr;  // dynamic C2a warp-tile claims
     unsigned hub_ctr;   // dynamic C1h row claims
+    unsigned big_ctr;   // C2b: tiles of > kBigTile merged entries listed for the balanced copy
+    int32_t big_flag;   // C2a: some tile has > kBigTile merged entries
     int32_t chunk1[2 * kMaxContractCtas];  // C1 chunk sums {#leaders, sum ub} per owner CTA
     int32_t chunk2[kMaxContractCtas];      // C2 chunk sums of merged entries per owner CTA
     unsigned long long dbg[8];             // debug: slowest C2a warp tile (ns<<32 | tile), paths
