@@ -710,6 +710,16 @@ gp_status coarsen_single(Graph *g, const gp_coarsen_opts *opts, Hier **out) {
         sl.max_rounds = opts->max_rounds;
         if (small_use(n_b, m_b)) {
             s2 = enqueue_small(ctx, sl);
+        } else if (part_use(ctx, n_b, m_b) && !medium_use(n_b, m_b)) {  // all SMs, shared-memory partitions
+            PartLaunch pl;
+            static_cast<SmallLaunch &>(pl) = sl;
+            void *scr = nullptr;
+            s2 = dev_alloc(ctx, &scr, part_scratch_bytes(n_b, m_b));
+            if (s2 == GP_OK) {
+                h->arenas.push_back(scr);
+                pl.scratch = scr;
+                s2 = enqueue_part(ctx, pl);
+            }
         } else {  // one thread-block cluster, state in global memory
             MediumLaunch ml;
             static_cast<SmallLaunch &>(ml) = sl;
@@ -729,7 +739,7 @@ gp_status coarsen_single(Graph *g, const gp_coarsen_opts *opts, Hier **out) {
     bool stop_seen = false;
     while (st == GP_OK) {
         while (st == GP_OK && !stop_seen && enq < max_levels && enq - obs < kAhead) {
-            if (small_use(tight_n, tight_m) || medium_use(tight_n, tight_m)) {
+            if (small_use(tight_n, tight_m) || medium_use(tight_n, tight_m) || part_use(ctx, tight_n, tight_m)) {
                 GP_DBG("enqueue tail levels %d.. in one CTA / cluster (bounds n=%d nnz=%d)\n", enq, tight_n, tight_m);
                 st = enqueue_tail(enq);
                 enq = max_levels;
@@ -814,6 +824,9 @@ gp_status coarsen_single(Graph *g, const gp_coarsen_opts *opts, Hier **out) {
                     }
                     fprintf(stderr, "\n");
                 }
+                if (hd[l].match.barr[0][0])  // the partitioned grid tail (part.cu, GP_PROF=1)
+                    fprintf(stderr, "[gp]   part: slowest CTA round-1 proposals %.1f us, merges %.1f us, copy %.1f us\n",
+                            hd[l].match.wmax[0] * 1e-3, hd[l].match.barr[0][0] * 1e-3, hd[l].match.barr[0][1] * 1e-3);
                 if (hd[l].match.lens[1]) {
                     fprintf(stderr, "[gp]   per round (live | slowest warp us | rows rescanned thread / warp):");
                     for (int k = 1; k < 16 && hd[l].match.lens[k]; ++k)

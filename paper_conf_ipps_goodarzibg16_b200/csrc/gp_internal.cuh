@@ -329,6 +329,15 @@ struct MediumLaunch : SmallLaunch {
 bool medium_use(int32_t n_bound, int32_t nnz_bound);
 size_t medium_scratch_bytes(int32_t n, int32_t nnz);
 gp_status enqueue_medium(Ctx *ctx, const MediumLaunch &L);
+// partitioned grid tail (part.cu): every remaining level in one cooperative launch over all SMs,
+// each CTA's vertex range and rows in shared memory; same per-level outputs as small.cu
+struct PartLaunch : SmallLaunch {
+    void *scratch;  // part_scratch_bytes(cap_n, cap_nnz)
+};
+bool part_fits(Ctx *ctx, int32_t n, int32_t nnz);
+bool part_use(Ctx *ctx, int32_t n_bound, int32_t nnz_bound);
+size_t part_scratch_bytes(int32_t n, int32_t nnz);
+gp_status enqueue_part(Ctx *ctx, const PartLaunch &L);
 
 // refinement of un-coarsening (refine.cu)
 gp_status refine_graph(Ctx *ctx, const Graph *g, int32_t *d_part, const gp_refine_opts &o, int32_t *moves_out,

@@ -1,11 +1,17 @@
 """Coarse-level tail, -m gpu: once the level bounds are small, ONE launch runs
 every remaining level -- one CTA with the graph in shared memory (csrc/small.cu) when it fits one
-SM, else one thread-block cluster with the graph in L2 (csrc/medium.cu).  Each hierarchy must be
-bit-identical to the oracle and to the level kernels, in all three modes:
-  small   (default)                  single CTA when it fits, else the level kernels
-  medium  (GP_SMALL=0, GP_MEDIUM=1)  the cluster kernel (opt-in: measured slower)
-                                     even for graphs that fit one SM
-  levels  (GP_SMALL=0, GP_MEDIUM=0)  the grid-wide level kernels only."""
+SM, else every SM with its vertex range and rows in shared memory (csrc/part.cu), or (opt-in)
+one thread-block cluster with the graph in L2 (csrc/medium.cu).  Each hierarchy must be
+bit-identical to the oracle and to the level kernels, in every mode:
+  small    (default)                  single CTA when it fits, else the partitioned grid tail
+                                      when it fits, else the level kernels
+  part     (GP_SMALL=0)               the partitioned grid tail even for graphs that fit one SM
+  part_many (GP_SMALL=0, GP_PART_W=256)  ... on many CTAs (ranges of a few vertices: most pairs
+                                      and arcs cross CTA ranges)
+  part_global (+ GP_PART_GARCS=1, GP_PART_WCAP=64)  rows and most window lookups read from
+                                      global memory (the paths of graphs that do not fit)
+  medium   (GP_SMALL=0, GP_MEDIUM=1)  the cluster kernel (opt-in: measured slower)
+  levels   (GP_SMALL=0, GP_MEDIUM=0, GP_PART=0)  the grid-wide level kernels only."""
 import os
 
 import numpy as np
@@ -31,12 +37,20 @@ def ctx(gp):
     c.close()
 
 
-MODES = {"small": {}, "medium": {"GP_SMALL": "0", "GP_MEDIUM": "1"}, "levels": {"GP_SMALL": "0", "GP_MEDIUM": "0"}}
+MODES = {
+    "small": {},
+    "part": {"GP_SMALL": "0"},
+    "part_many": {"GP_SMALL": "0", "GP_PART_W": "256"},
+    "part_global": {"GP_SMALL": "0", "GP_PART_W": "256", "GP_PART_GARCS": "1", "GP_PART_WCAP": "64"},
+    "medium": {"GP_SMALL": "0", "GP_MEDIUM": "1"},
+    "levels": {"GP_SMALL": "0", "GP_MEDIUM": "0", "GP_PART": "0"},
+}
+KNOBS = ("GP_SMALL", "GP_MEDIUM", "GP_PART", "GP_PART_W", "GP_PART_GARCS", "GP_PART_WCAP")
 
 
 def _run(gp, ctx, g, mode, **kw):
     env = MODES[mode]
-    old = {k: os.environ.get(k) for k in ("GP_SMALL", "GP_MEDIUM")}
+    old = {k: os.environ.get(k) for k in KNOBS}
     for k in old:
         os.environ.pop(k, None)
     os.environ.update(env)
@@ -68,6 +82,7 @@ CASES = {
     "delaunay_40": (lambda: G.delaunay_like(40), dict(threshold=10)),
     "rmat10_shuf_vw": (lambda: G.varied_vwgt(G.shuffle_rows(G.rmat(10), 3)), dict(threshold=10)),
     "star1500": (lambda: _star(1500), dict(threshold=2)),
+    "star5000": (lambda: _star(5000), dict(threshold=2)),  # a merged row > 2048 keys (global staging)
     "road_48": (lambda: G.road_like(48), dict(threshold=5)),
     "isolated": (lambda: G.from_edge_list(300, []), dict(threshold=0)),
     "one_edge20": (lambda: G.from_edge_list(20, [(3, 11, 5)]), dict(threshold=1)),
@@ -88,6 +103,7 @@ def test_tail_equals_oracle_and_level_kernels(gp, ctx, name):
         assert_levels_equal(got, ref, f"{name} {mode}")
     if len(ref) > 1:  # the tail really ran (fewer launches than the level kernels)
         assert launches["medium"] < launches["levels"], launches
+        assert launches["part"] < launches["levels"], launches
         if g["n"] <= 8192:
             assert launches["small"] < launches["levels"], launches
 
@@ -100,10 +116,10 @@ def test_tail_is_one_launch_on_c1(gp, ctx):
 
 @pytest.mark.parametrize("name", ["C3_512", "C2_2^16", "road_256", "rmat14_w4"])
 def test_medium_tail_mid_hierarchy(gp, ctx, name):
-    """Graphs whose hierarchies enter the cluster tail after a few level kernels."""
+    """Graphs whose hierarchies enter the grid / cluster tail after a few level kernels."""
     g = {"C3_512": lambda: G.delaunay_like(512), "C2_2^16": lambda: G.rgg(1 << 16),
          "road_256": lambda: G.road_like(256), "rmat14_w4": lambda: G.rmat(14, wmax=4)}[name]()
     ref = oracle.coarsen_to(g, threshold=100)
-    for mode in ("small", "medium", "levels"):
+    for mode in ("small", "part_many", "part_global", "medium", "levels"):
         got, _ = _run(gp, ctx, g, mode, threshold=100)
         assert_levels_equal(got, ref, f"{name} {mode}")
