@@ -87,4 +87,39 @@ __device__ __forceinline__ void cx_sort16(uint32_t (&cx)[16], int32_t (&w)[16]) 
 #undef GP_CE
 }
 
+// Batcher odd-even merge sort network for 8 inputs (19 comparators; checked exhaustively on
+// 0-1 inputs), for rows of <= 8 merged entries (part.cu)
+__device__ __forceinline__ void cx_sort8(uint32_t (&cx)[8], int32_t (&w)[8]) {
+#define GP_CE(i, j)                                                      \
+    {                                                                    \
+        const bool sw = cx[i] > cx[j];                                   \
+        const uint32_t c0 = sw ? cx[j] : cx[i], c1 = sw ? cx[i] : cx[j]; \
+        const int32_t w0 = sw ? w[j] : w[i], w1 = sw ? w[i] : w[j];      \
+        cx[i] = c0;                                                      \
+        cx[j] = c1;                                                      \
+        w[i] = w0;                                                       \
+        w[j] = w1;                                                       \
+    }
+    GP_CE(0, 1)
+    GP_CE(2, 3)
+    GP_CE(4, 5)
+    GP_CE(6, 7)
+    GP_CE(0, 2)
+    GP_CE(1, 3)
+    GP_CE(4, 6)
+    GP_CE(5, 7)
+    GP_CE(1, 2)
+    GP_CE(5, 6)
+    GP_CE(0, 4)
+    GP_CE(1, 5)
+    GP_CE(2, 6)
+    GP_CE(3, 7)
+    GP_CE(2, 4)
+    GP_CE(3, 5)
+    GP_CE(1, 2)
+    GP_CE(3, 4)
+    GP_CE(5, 6)
+#undef GP_CE
+}
+
 }  // namespace gp

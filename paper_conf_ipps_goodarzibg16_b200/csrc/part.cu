@@ -250,6 +250,59 @@ __device__ __forceinline__ int32_t part_best(const PartView &V, const int32_t *P
     return key_vertex<H>(seed, best);
 }
 
+// Heaviest (free, when TEST) neighbour for every lane of the warp with `need`, the rows of the
+// needing lanes flattened over the lanes 32 arcs at a time: a lane finds its arc's row by a
+// shuffle search over the rows' exclusive degree prefix, and per-row maxima are a segmented
+// shuffle max whose segment tails update the row's slot.  Coarse levels have a heavy degree
+// tail (C3 level 8: mean 3.6, p99 19): a row per lane made every warp as slow as its longest
+// row.  All 32 lanes call (warp-uniform); `slot` = 32 entries of this warp.
+template <bool H, bool TEST>
+__device__ __forceinline__ int32_t warp_flat_best(const PartView &V, const int32_t *Pk, uint32_t seed, bool need,
+                                                  int32_t i, unsigned long long *slot) {
+    const int lane = threadIdx.x & 31;
+    const int32_t s = need ? V.rs(i) : 0;
+    const int32_t deg = need ? V.rs(i + 1) - s : 0;
+    const int32_t incl = warp_incl_scan(deg), excl = incl - deg;
+    const int32_t T = __shfl_sync(0xffffffffu, incl, 31);
+    slot[lane] = 0;
+    __syncwarp();
+    for (int32_t base = 0; base < T; base += 32) {
+        const int32_t e = base + lane;
+        const bool valid = e < T;
+        int o = 0;  // the last lane whose exclusive prefix is <= e (a lane with a positive degree)
+#pragma unroll
+        for (int step = 16; step > 0; step >>= 1) {
+            const int32_t ex = __shfl_sync(0xffffffffu, excl, o + step);
+            if (ex <= e) o += step;
+        }
+        const int32_t so = __shfl_sync(0xffffffffu, s, o), eo = __shfl_sync(0xffffffffu, excl, o);
+        unsigned long long key = 0;
+        if (valid) {
+            const int32_t j = so + (e - eo);
+            const int32_t x = V.arc(j), w = V.wgt(j);
+            bool f = true;
+            if (TEST) {
+                const int32_t c = V.wget(Pk, x);
+                f = !(c >= 0 && V.wget(Pk, c) == x);
+            }
+            if (f) key = pack_key<H>(seed, w, x);
+        }
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {  // segmented inclusive max over equal owners
+            const unsigned long long ok = __shfl_up_sync(0xffffffffu, key, d);
+            const int oo = __shfl_up_sync(0xffffffffu, o, d);
+            if (lane >= d && oo == o) key = umax64(key, ok);
+        }
+        const int no = __shfl_down_sync(0xffffffffu, o, 1);
+        const bool nvalid = __shfl_down_sync(0xffffffffu, valid ? 1 : 0, 1) != 0;
+        if (valid && (lane == 31 || no != o || !nvalid)) slot[o] = umax64(slot[o], key);
+        __syncwarp();
+    }
+    const unsigned long long bk = slot[lane];
+    __syncwarp();
+    return need ? key_vertex<H>(seed, bk) : kNone;
+}
+
 // the two fine rows of coarse row c (leader u = lo + i, partner v): arc e of the merged row
 struct RowSrc {
     int32_t su, du, sv, dv;  // starts (own rows: local arc index; foreign v: global) and degrees
@@ -314,15 +367,16 @@ __device__ __forceinline__ KeyAcc stage_of(const PartView &V, const RowSrc &r, u
     return s;
 }
 
-// ---- merged rows of <= 16 entries: one thread, register network ----
+// ---- merged rows of <= N (8 or 16) entries: one thread, register network ----
+template <int N>
 __device__ __forceinline__ int32_t merge_thread(const PartView &V, const int32_t *CMg, const RowSrc &r, int32_t c,
                                                 const KeyAcc &st) {
     const uint32_t kDrop = 0xFFFFFFFFu;
-    uint32_t kc[16];
-    int32_t kw[16];
+    uint32_t kc[N];
+    int32_t kw[N];
     const int32_t ub = r.du + r.dv;
 #pragma unroll
-    for (int q = 0; q < 16; ++q) {
+    for (int q = 0; q < N; ++q) {
         kc[q] = kDrop;
         kw[q] = 0;
         if (q < ub) {
@@ -333,12 +387,13 @@ __device__ __forceinline__ int32_t merge_thread(const PartView &V, const int32_t
             }
         }
     }
-    cx_sort16(kc, kw);
+    if constexpr (N == 8) cx_sort8(kc, kw);
+    else cx_sort16(kc, kw);
     int32_t cnt = 0;
     uint32_t prev = kDrop;
     int32_t acc = 0;
 #pragma unroll
-    for (int q = 0; q < 16; ++q) {
+    for (int q = 0; q < N; ++q) {
         if (kc[q] == prev) {
             acc += kw[q];  // repeated coarse neighbour: weights summed (R8, P12.s28)
         } else {
@@ -664,6 +719,8 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
 #endif
         {  // round-1 proposals: every vertex is free (phase g)
             int32_t mylive = 0;
+            // one row per thread: no freedom test in round 1, so a row is a short chain of
+            // shared loads (the flattened scan of the later rounds measured slower here)
             for (int32_t i = t; i < V.nv; i += kPT) {
                 const int32_t u = V.lo + i;
                 const int32_t p = part_best<H>(V, a.P1, a.tie_seed, i, false);
@@ -702,30 +759,34 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             if (k == 1) PT_DD();
             PT_MARK();
             int32_t mylive = 0, mypairs = 0;
-#define PT_CK() do { } while (0)
-#ifdef GP_PART_DBG
-            __syncwarp();
-            const long long wc0 = clock64();
-#endif
-            for (int32_t i = t; i < V.nv; i += kPT) {
-                if (V.M[i] != kFree) continue;
+            unsigned long long *slot = skeys + wid * 32;
+            for (int32_t ib = t - lane; ib < V.nv; ib += kPT) {  // warp-uniform
+                const int32_t i = ib + lane;
                 const int32_t u = V.lo + i;
-                const int32_t p = V.wget(Pk, u);
-                PT_CK();
-                if (p < 0) continue;  // dead: no free neighbour (stays free: leftover)
-                ++visits;
-                const int32_t q = V.wget(Pk, p);
-                PT_CK();
-                if (q == u) {  // handshake (P18.s10-12): matched in round k
+                int32_t p = -1, q = -1;
+                bool live = false, need = false;
+                if (i < V.nv && V.M[i] == kFree) {
+                    p = V.wget(Pk, u);
+                    live = p >= 0;  // else dead: no free neighbour (stays free: leftover)
+                }
+                if (live) {
+                    ++visits;
+                    q = V.wget(Pk, p);
+                    // q == u: handshake (P18.s10-12); else p keeps being the heaviest free
+                    // neighbour while it is free after round k, and u rescans if p matched q
+                    need = q != u && q >= 0 && V.wget(Pk, q) == p;
+                }
+                const int32_t b2 = warp_flat_best<H, true>(V, Pk, a.tie_seed, need, i, slot);
+                if (!live) continue;
+                if (q == u) {  // matched in round k
                     V.M[i] = p;
                     Pn[u] = p;  // both parity buffers now hold the partner
                     mypairs += u < p;
                     continue;
                 }
-                int32_t np = p;  // p still free after round k: still the heaviest free neighbour
-                if (q >= 0 && V.wget(Pk, q) == p) {  // p matched q this round: rescan
-                    np = part_best<H>(V, Pk, a.tie_seed, i, true);
-                    PT_CK();
+                int32_t np = p;
+                if (need) {
+                    np = b2;
                     ++rows;
                     arcs += (unsigned long long)(V.rs(i + 1) - V.rs(i));
                 }
@@ -735,27 +796,7 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
                 // completes a handshake or a "matched" test)
                 if (np < 0) Pk[u] = kNone;
                 mylive += np >= 0;
-                PT_CK();
             }
-#ifdef GP_PART_DBG
-            __syncwarp();
-            const long long wc1 = clock64();
-            {  // dry pass: the same lookups again (no writes), warm caches
-                unsigned long long dummy = 0;
-                for (int32_t i = t; i < V.nv; i += kPT) {
-                    const int32_t u = V.lo + i;
-                    const int32_t p = V.wget(Pk, u);
-                    if (p < 0) continue;
-                    const int32_t q = V.wget(Pk, p);
-                    dummy += (unsigned)part_best<H>(V, Pk, a.tie_seed, i, true) + (unsigned)q;
-                }
-                __syncwarp();
-                const long long wc2 = clock64();
-                if (k == 1 && level == 4 && b < 4 && lane == 0)
-                    printf("PW b=%d w=%d real %lld dry %lld (%llu)\n", b, wid, wc1 - wc0, wc2 - wc1, dummy & 1);
-            }
-#endif
-#undef PT_CK
             PT_MARK();
             if (k == 1) PT_DD();
 #ifdef GP_PART_DBG
@@ -819,25 +860,48 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
         // rows of > 16 merged entries, in sweeps over windows of kPT vertices: 17..32 by half
         // warps, 33..64 by warps, longer by the whole CTA
         PT_DD();
+#ifdef GP_PART_DBG
+        long long sw_c[4] = {0, 0, 0, 0};
+        int sw_n[4] = {0, 0, 0, 0};
+        long long swc = clock64();
+#define SW_CK(q) do { const long long c_ = clock64(); sw_c[q] += c_ - swc; swc = c_; } while (0)
+#else
+#define SW_CK(q) do { } while (0)
+#endif
         for (int32_t r0 = 0; r0 < V.nv; r0 += kPT) {
             if (t == 0) s_cnt3[0] = s_cnt3[1] = s_cnt3[2] = s_cnt3[3] = 0;
             __syncthreads();
             {
                 const int32_t i = r0 + t;
+                int which = -1;
                 if (i < V.nv) {
                     const int32_t m = V.M[i];
                     if (V.lo + i <= m) {
                         const RowSrc r = row_src(V, i, m);
                         const int32_t ub = r.du + r.dv;
-                        if (ub > 16) {
-                            const int which = ub <= 32 ? 0 : ub <= 64 ? 1 : ub <= 256 ? 2 : 3;
-                            s_lists[which][atomicAdd(&s_cnt3[which], 1)] = i;
-                        }
+                        if (ub > 16) which = ub <= 32 ? 0 : ub <= 64 ? 1 : ub <= 256 ? 2 : 3;
+                    }
+                }
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {  // warp-aggregated appends (one shared atomic per warp and list)
+                    const unsigned bq = __ballot_sync(0xffffffffu, which == q);
+                    if (bq) {
+                        int32_t base = 0;
+                        if (lane == __ffs(bq) - 1) base = atomicAdd(&s_cnt3[q], __popc(bq));
+                        base = __shfl_sync(0xffffffffu, base, __ffs(bq) - 1);
+                        if (which == q) s_lists[q][base + __popc(bq & lanemask_lt())] = i;
                     }
                 }
             }
             __syncthreads();
             const int32_t nA = s_cnt3[0], nB = s_cnt3[1], nW = s_cnt3[2], nC = s_cnt3[3];
+            SW_CK(0);
+#ifdef GP_PART_DBG
+            sw_n[0] += nA;
+            sw_n[1] += nB;
+            sw_n[2] += nW;
+            sw_n[3] += nC;
+#endif
             if (nA + nB + nW + nC == 0) continue;
             unsigned long long *wbuf = skeys + wid * 256;  // this warp's shared-memory keys
             for (int32_t q = 2 * wid; q < nA; q += 2 * kPW) {  // two 17..32-entry rows per warp
@@ -860,6 +924,7 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
                 const int32_t k2 = merge_seg(V, o.CM, r, cc, st, wbuf + half * 32);
                 if (ii >= 0 && (lane & 15) == 0) V.cnt[ii] = k2;
             }
+            SW_CK(1);
             for (int32_t q = wid; q < nB; q += kPW) {
                 const int32_t ii = s_lists[1][q];
                 const RowSrc r = row_src(V, ii, V.M[ii]);
@@ -874,6 +939,7 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
                 if (lane == 0) V.cnt[ii] = k2;
             }
             __syncthreads();
+            SW_CK(2);
             for (int32_t q = 0; q < nC; ++q) {
                 const int32_t ii = s_lists[3][q];
                 const RowSrc r = row_src(V, ii, V.M[ii]);
@@ -884,15 +950,41 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             }
         }
         PT_MARK();
+        SW_CK(3);
+#ifdef GP_PART_DBG
+        if (t == 0 && level == 4 && b < 8)
+            printf("PSW b=%d classify %lld seg %lld warp+ %lld cta %lld | rows %d %d %d %d\n", b, sw_c[0], sw_c[1], sw_c[2],
+                   sw_c[3], sw_n[0], sw_n[1], sw_n[2], sw_n[3]);
+#endif
+#undef SW_CK
         PT_DD();
         // rows of <= 16 entries by their thread (contiguous blocks = coarse id order)
+        // (warp-uniform steps: the 8-entry network runs when every merging lane's row fits it,
+        // else all merging lanes run the 16-entry one -- divergent networks would run both)
         int32_t mine = 0;
-        for (int32_t i = i0; i < i1; ++i) {
-            const int32_t u = V.lo + i, m = V.M[i];
-            if (u > m) continue;
-            const RowSrc r = row_src(V, i, m);
-            if (r.du + r.dv <= 16) V.cnt[i] = merge_thread(V, o.CM, r, V.wget(o.CM, u), stage_of(V, r, a.wkeys));
-            mine += V.cnt[i];
+        for (int32_t r0 = 0; r0 < per; ++r0) {
+            const int32_t i = i0 + r0;
+            int32_t ub = 0, m = 0;
+            RowSrc r;
+            r.du = r.dv = r.su = r.sv = 0;
+            r.vglob = false;
+            bool lead = false;
+            if (i < i1) {
+                m = V.M[i];
+                lead = V.lo + i <= m;
+                if (lead) {
+                    r = row_src(V, i, m);
+                    ub = r.du + r.dv;
+                }
+            }
+            const bool narrow = lead && ub <= 16;
+            const bool all8 = __all_sync(0xffffffffu, !narrow || ub <= 8);
+            if (narrow) {
+                const KeyAcc st = stage_of(V, r, a.wkeys);
+                const int32_t cu = V.wget(o.CM, V.lo + i);
+                V.cnt[i] = all8 ? merge_thread<8>(V, o.CM, r, cu, st) : merge_thread<16>(V, o.CM, r, cu, st);
+            }
+            if (lead) mine += V.cnt[i];
         }
         int32_t ctot;
         PT_DD();

@@ -68,7 +68,16 @@ __global__ void __launch_bounds__(512, 1) k_round(const int32_t *Pg, int32_t *Pn
             continue;
         }
         int32_t np = p;
-        if (VAR == 1 || (q >= 0 && V.wget(Pk, q) == p)) np = part_best<false>(V, Pk, 0u, i, true);
+        if (VAR == 2) {  // pure shared lookups (no predicated global fallback)
+            if (q >= 0 && V.win[q - V.wlo] == p) {
+                unsigned long long best = 0;
+                for (int32_t j = V.rs(i); j < V.rs(i + 1); ++j) {
+                    const int32_t x = V.sadj[j], c = V.win[x - V.wlo];
+                    if (!(c >= 0 && V.win[c - V.wlo] == x)) best = umax64(best, pack_key<false>(0u, V.swgt[j], x));
+                }
+                np = key_vertex<false>(0u, best);
+            }
+        } else if (VAR == 1 || (q >= 0 && V.wget(Pk, q) == p)) np = part_best<false>(V, Pk, 0u, i, true);
         Pn[u] = np;
         live += np >= 0;
     }
@@ -108,5 +117,6 @@ int main() {
     };
     run(k_round<0>, "keep + rescans");
     run(k_round<1>, "rescan every live vertex");
+    run(k_round<2>, "keep + rescans, pure LDS");
     return 0;
 }
