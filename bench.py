@@ -269,31 +269,18 @@ def run_ours(args, rank, world, local_rank):
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         ms_step = float(t.item())
 
-    # roofline of the dominant kernel family
-    fam_bytes = {}
-    for l in levels:
-        for k, v in level_bytes(l).items():
-            fam_bytes[k] = fam_bytes.get(k, 0) + v
-    if sharded:  # global sizes / world: the bytes one rank's kernels move (rows split evenly)
-        fam_bytes = {k: v / world for k, v in fam_bytes.items()}
-    kfam = {"match": "propose", "contract": "contract"}   # gp_kernel_kind of each family
-    fam_ms = {k: kstats[kfam[k]]["ms"] / args.steps for k in fam_bytes}
-    dom = max(fam_ms, key=lambda k: fam_ms[k])
-    peak, peak_kind = peaks()
-    achieved = fam_bytes[dom] / (fam_ms[dom] / 1e3) / 1e9 if fam_ms[dom] > 0 else 0.0
-    step_bytes = sum(fam_bytes.values())
-    traffic = ncu_traffic(args.config, {"match": "k_match_level", "contract": "k_contract_level"}[dom])
-
     # per-level rows (BASELINE metric "fine edges coarsened/sec per level"): each step enqueues
     # level l's matching then its contraction (speculative levels after the stop come last);
     # the median over the timed steps of each launch's CUDA-event time
+    peak, peak_kind = peaks()
     per_step = len(ltimes) // args.steps if args.steps else 0
     level_rows, tail = [], None
+    nreg, nreg_known = len(levels), False
     if not sharded and args.loopback <= 1 and per_step >= 1:
         # levels on the level kernels: 2 launches each (propose = k_match_level, contract =
         # k_contract_level); the coarse-level tail (one 'other' launch) runs the rest
         step0 = ltimes[:per_step]
-        nreg = 0
+        nreg, nreg_known = 0, True
         while 2 * nreg + 1 < per_step and nreg < len(levels) and step0[2 * nreg][0] == "propose" \
                 and step0[2 * nreg + 1][0] == "contract":
             nreg += 1
@@ -315,11 +302,34 @@ def run_ours(args, rank, world, local_rank):
         if nreg < len(levels) and 2 * nreg < per_step and step0[2 * nreg][0] == "other":
             tus = 1e3 * statistics.median(ltimes[st * per_step + 2 * nreg][1] for st in range(args.steps))
             rest = levels[nreg:]
+            tb = sum(sum(level_bytes(l).values()) for l in rest)  # §8(d) bytes of the tail's levels
             tail = {"levels": [nreg, len(levels) - 1], "launches": 1, "us": round(tus, 2),
                     "n_first": rest[0]["n"], "edges": sum(l["nnz"] // 2 for l in rest),
                     "rounds": [l["rounds"] for l in rest],
                     "edges_per_s": sum(l["nnz"] // 2 for l in rest) / (tus / 1e6),
-                    "kernel": "coarse-level tail: k_small (one CTA, shared memory) or k_medium (one cluster, L2)"}
+                    "bytes": tb, "GBps": tb / (tus / 1e6) / 1e9,
+                    "kernel": ("coarse-level tail: k_part (every SM, each CTA's vertex range and rows in shared "
+                               "memory) when the level fits the SMs' shared memory, k_small (one CTA) when it fits one "
+                               "SM, k_medium (one cluster, opt-in)")}
+
+    # roofline of the dominant kernel family
+    # (the levels the two level kernels ran; the coarse-level tail's levels are one other launch)
+    fam_bytes = {}
+    for l in (levels[:nreg] if nreg_known else levels):
+        for k, v in level_bytes(l).items():
+            fam_bytes[k] = fam_bytes.get(k, 0) + v
+    if sharded:  # global sizes / world: the bytes one rank's kernels move (rows split evenly)
+        fam_bytes = {k: v / world for k, v in fam_bytes.items()}
+    kfam = {"match": "propose", "contract": "contract"}   # gp_kernel_kind of each family
+    fam_ms = {k: kstats[kfam[k]]["ms"] / args.steps for k in fam_bytes}
+    if tail is not None:  # the coarse-level tail is one launch: its own family
+        fam_bytes["tail"] = tail["bytes"]
+        fam_ms["tail"] = tail["us"] / 1e3
+    dom = max(fam_ms, key=lambda k: fam_ms[k])
+    achieved = fam_bytes[dom] / (fam_ms[dom] / 1e3) / 1e9 if fam_ms[dom] > 0 else 0.0
+    step_bytes = sum(fam_bytes.values())
+    traffic = ncu_traffic(args.config, {"match": "k_match_level", "contract": "k_contract_level",
+                                        "tail": "k_part"}[dom])
 
     # projection: a synthetic labelling of the coarsest graph (c mod 64)
     # carried down to level 0 in one launch; algorithmic bytes = CM_0 read + labels written +
@@ -433,7 +443,8 @@ def run_ours(args, rank, world, local_rank):
                      "traffic_source": traffic[1] if traffic else None,
                      "bytes_per_step": fam_bytes[dom], "ms_per_step": fam_ms[dom]},
         "kernels": {k: {"ms_per_step": fam_ms[k], "GB/s": (fam_bytes[k] / (fam_ms[k] / 1e3) / 1e9) if fam_ms[k] else None,
-                        "launches_per_step": kstats[kfam[k]]["launches"] / args.steps} for k in fam_bytes},
+                        "launches_per_step": (kstats[kfam[k]]["launches"] / args.steps) if k in kfam else 1.0}
+                    for k in fam_bytes},
         "e2e": {"value": edges_per_step / (e2e_step / 1e3), "unit": UNIT, "ms_per_step": e2e_step,
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
         "gpu_launches": launches,
