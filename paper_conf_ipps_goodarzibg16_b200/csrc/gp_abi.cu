@@ -174,7 +174,9 @@ gp_status alloc_graph_arrays(Ctx *ctx, Graph *g, int32_t n_bound, int32_t nnz_bo
 }
 
 gp_status level_scratch(Ctx *ctx, int32_t n, int32_t nnz, LevelBufs *lb) {
-    const size_t nn = (size_t)(n > 0 ? n : 1);
+    // per-vertex arrays: a multiple of 4 ints, padded by >= 4 (16-byte aligned TMA windows that
+    // may round up past n, match_win.cu)
+    const size_t nn = ((size_t)(n > 0 ? n : 1) + 7) & ~(size_t)3;
     const size_t tiles = contract_tiles(n, nnz);
     const size_t ints = 14 * nn + 1 + 3 * tiles + 32;
     const size_t ibytes = ((ints * 4 + 255) / 256) * 256;
@@ -618,6 +620,13 @@ gp_status coarsen_single(Graph *g, const gp_coarsen_opts *opts, Hier **out) {
     if (st == GP_OK) st = fresh_sizes(ctx, g, in0);
     for (int i = 0; i < max_levels; ++i) ctx->reports[i].ready = 0;
 
+    // id locality of the input graph (measured once per graph; coarse graphs keep it: coarse ids
+    // follow the leaders' id order)
+    bool use_win = false;
+    if (st == GP_OK && win_enabled() && g->n >= win_min_n()) {  // opt-in (GP_WIN=1)
+        if (g->locality < 0) st = graph_locality(ctx, g, &g->locality);
+        use_win = g->locality == 1;
+    }
     auto enqueue_level = [&](int l) -> gp_status {
         const Graph *in = (l == 0) ? g : lv[l - 1].coarse;
         const int32_t n_b = tight_n, m_b = tight_m;
@@ -640,7 +649,10 @@ gp_status coarsen_single(Graph *g, const gp_coarsen_opts *opts, Hier **out) {
         LevelBufs b = lb;
         set_graph_bufs(&b, in);
         b.in = (l == 0) ? in0 : in->sizes;
-        s2 = enqueue_match(ctx, b, L.match, &h->levdev[l].match, opts->max_rounds, false, avg_degree(n_b, m_b));
+        if (use_win && n_b >= win_min_n())  // windowed rounds for graphs with local ids (match_win.cu)
+            s2 = enqueue_match_win(ctx, b, L.match, &h->levdev[l].match, opts->max_rounds);
+        else
+            s2 = enqueue_match(ctx, b, L.match, &h->levdev[l].match, opts->max_rounds, false, avg_degree(n_b, m_b));
         if (s2 != GP_OK) return s2;
         ContractParams prm{true, opts->threshold, pct, l, max_levels, n_b, m_b};
         return enqueue_contract(ctx, b, L.match, L.cmap, cg, &h->levdev[l].contract, &h->levdev[l].out,

@@ -148,6 +148,7 @@ struct gp_graph_s {
     gp::SizeRec *sizes = nullptr;  // device copy of {n, nnz, stop}
     bool owns_sizes = true;
     bool borrowed = false;  // owned by a hierarchy
+    int locality = -1;      // ids local (1) or not (0), measured on first use (match_win.cu)
     // sharded graphs (NCCL contexts): this rank's rows are the global vertices
     // [vbase, vbase + n); ranges[r] .. ranges[r+1] is rank r's range; adjncy holds global ids
     bool dist = false;
@@ -329,6 +330,11 @@ struct MediumLaunch : SmallLaunch {
 bool medium_use(int32_t n_bound, int32_t nnz_bound);
 size_t medium_scratch_bytes(int32_t n, int32_t nnz);
 gp_status enqueue_medium(Ctx *ctx, const MediumLaunch &L);
+// windowed matching rounds for graphs with local ids (match_win.cu)
+gp_status enqueue_match_win(Ctx *ctx, const LevelBufs &lb, int32_t *M, MatchCtl *ctl, int32_t max_rounds);
+gp_status graph_locality(Ctx *ctx, Graph *g, int *out);
+bool win_enabled();
+int32_t win_min_n();
 // partitioned grid tail (part.cu): every remaining level in one cooperative launch over all SMs,
 // each CTA's vertex range and rows in shared memory; same per-level outputs as small.cu
 struct PartLaunch : SmallLaunch {

@@ -123,3 +123,27 @@ def test_medium_tail_mid_hierarchy(gp, ctx, name):
     for mode in ("small", "part_many", "part_global", "medium", "levels"):
         got, _ = _run(gp, ctx, g, mode, threshold=100)
         assert_levels_equal(got, ref, f"{name} {mode}")
+
+
+@pytest.mark.parametrize("name", ["C3_512", "rgg_2^16", "road_256", "grid_shuf_vw"])
+def test_windowed_match_opt_in(gp, ctx, name):
+    """The opt-in windowed big-level matching (csrc/match_win.cu, GP_WIN=1), forced onto small
+    levels (GP_WIN_N), with and without the grid tail: bit-identical to the oracle."""
+    g = {"C3_512": lambda: G.delaunay_like(512), "rgg_2^16": lambda: G.rgg(1 << 16),
+         "road_256": lambda: G.road_like(256),
+         "grid_shuf_vw": lambda: G.varied_vwgt(G.shuffle_rows(G.grid2d(200, 200), 5))}[name]()
+    ref = oracle.coarsen_to(g, threshold=100)
+    old = {k: os.environ.get(k) for k in ("GP_WIN", "GP_WIN_N", "GP_PART")}
+    try:
+        os.environ["GP_WIN"] = "1"
+        os.environ["GP_WIN_N"] = "2000"
+        for part in ("1", "0"):
+            os.environ["GP_PART"] = part
+            got = gpu_coarsen(gp, ctx, g, threshold=100)
+            assert_levels_equal(got, ref, f"{name} windowed part={part}")
+    finally:
+        for k, v in old.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
