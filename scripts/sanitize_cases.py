@@ -1,6 +1,7 @@
 """Small coarsen_to runs for compute-sanitizer (memcheck / racecheck / synccheck), each checked
 bit for bit against the oracle so that a sanitizer run also proves the results:
-    python scripts/sanitize_cases.py c3_256 | star5000 | loopback3"""
+    python scripts/sanitize_cases.py c3_256 | star5000 | loopback3 | c1_tail | medium_tail |
+                                     part_tail | part_many | win | refine"""
 import os
 import sys
 
@@ -24,6 +25,19 @@ elif case == "c1_tail":  # the coarse-level tail kernel (csrc/small.cu) runs eve
 elif case == "medium_tail":  # the cluster tail (csrc/medium.cu): forced for a 16 K-vertex mesh
     os.environ["GP_SMALL"] = "0"
     os.environ["GP_MEDIUM"] = "1"
+    ctx, g, thr = gp.Context(0), G.delaunay_like(128), 100
+elif case == "part_tail":  # the partitioned grid tail (csrc/part.cu) for every level of a mesh
+    os.environ["GP_SMALL"] = "0"
+    ctx, g, thr = gp.Context(0), G.delaunay_like(128), 100
+elif case == "part_many":  # ... on many CTAs with rows and window lookups from global memory
+    os.environ["GP_SMALL"] = "0"
+    os.environ["GP_PART_W"] = "256"
+    os.environ["GP_PART_GARCS"] = "1"
+    os.environ["GP_PART_WCAP"] = "64"
+    ctx, g, thr = gp.Context(0), G.varied_vwgt(G.shuffle_rows(G.rmat(12), 3)), 10
+elif case == "win":  # the opt-in windowed big-level matching (csrc/match_win.cu)
+    os.environ["GP_WIN"] = "1"
+    os.environ["GP_WIN_N"] = "2000"
     ctx, g, thr = gp.Context(0), G.delaunay_like(128), 100
 elif case == "refine":  # gp_uncoarsen: projection + refinement kernels (csrc/refine.cu)
     import numpy as np
