@@ -572,6 +572,7 @@ gp_status gp_contract_level(gp_graph g, const gp_vid *d_match, gp_vid *d_cmap, g
 // stop (threshold / stall / max_levels) exits immediately and is discarded.
 // ---------------------------------------------------------------------------------------
 constexpr int kAhead = 2;
+constexpr int kTailSlots = 12;  // levels per coarse-level tail launch (arena slots)
 
 static bool debug_on() {
     static int on = -1;
@@ -663,9 +664,19 @@ gp_status coarsen_single(Graph *g, const gp_coarsen_opts *opts, Hier **out) {
     // shared memory, ONE launch of one CTA runs every remaining level.  The host creates the
     // levels up front (arrays in one arena slot per level) and reads their reports as usual.
     std::vector<std::vector<unsigned char>> keep_host;
+    // at most kTailSlots levels per tail launch (each slot is sized by the first level's
+    // bounds): a hierarchy that goes deeper continues with another launch from the last tail
+    // level's output, so the arena stays small (60 slots of C3's level-5 bounds were 1.6 GB,
+    // re-mapped per call when the sharded ranks fold onto this pipeline: loopback 13 -> 25 ms)
+    auto tail_slots = [&](int l0) -> int {
+        int ns = max_levels - l0;
+        const char *e = getenv("GP_TAIL_SLOTS");  // tuning knob (results never depend on it)
+        const int cap = e && atoi(e) > 0 ? atoi(e) : kTailSlots;
+        return cap < ns ? cap : ns;
+    };
     auto enqueue_tail = [&](int l0) -> gp_status {
         const int32_t n_b = tight_n, m_b = tight_m;
-        const int ns = max_levels - l0;
+        const int ns = tail_slots(l0);
         const size_t slot = small_slot_ints(n_b, m_b);
         void *arena = nullptr, *desc = nullptr;
         gp_status s2 = dev_alloc(ctx, &arena, sizeof(int32_t) * slot * (size_t)ns);
@@ -753,8 +764,9 @@ gp_status coarsen_single(Graph *g, const gp_coarsen_opts *opts, Hier **out) {
         while (st == GP_OK && !stop_seen && enq < max_levels && enq - obs < kAhead) {
             if (small_use(tight_n, tight_m) || medium_use(tight_n, tight_m) || part_use(ctx, tight_n, tight_m)) {
                 GP_DBG("enqueue tail levels %d.. in one CTA / cluster (bounds n=%d nnz=%d)\n", enq, tight_n, tight_m);
+                const int ns = tail_slots(enq);
                 st = enqueue_tail(enq);
-                enq = max_levels;
+                enq += ns;
                 break;
             }
             GP_DBG("enqueue level %d (bounds n=%d nnz=%d)\n", enq, tight_n, tight_m);

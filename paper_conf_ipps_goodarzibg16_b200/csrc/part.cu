@@ -82,6 +82,7 @@ struct PartArgs {
     int32_t wmin;                    // words of work per active CTA (fewer CTAs on small levels)
     int32_t force_garcs;             // test knob: arcs always read from global memory
     int32_t wcap_max;                // test knob: window capacity cap (words; 0 = none)
+    int32_t force_gstage;            // test knob: contraction staging in global memory
     int32_t prof;                    // GP_PROF=1: slowest CTA per round / contraction step
     int32_t trace;                   // GP_DEBUG: phase timestamps of block 0 (globaltimer reads cost)
 };
@@ -200,6 +201,10 @@ struct PartView {
     int32_t *sap, *M, *cnt, *sadj, *swgt, *win;
     int32_t loff, aoff;
     int32_t wlo, wlen;
+    // contraction staging in shared memory (after the window) when it fits: row i's merged
+    // entries at sst[cnt[i]] (cnt holds the rows' upper-bound offsets while merging)
+    unsigned long long *sst;
+    bool sstage;
     // row start of own vertex i relative to a0 (i in [0, nv])
     __device__ __forceinline__ int32_t rs(int32_t i) const { return sap[i + loff] - a0; }
     __device__ __forceinline__ int32_t arc(int32_t j) const { return garcs ? pld(gadjncy + a0 + j) : sadj[j + aoff]; }
@@ -363,6 +368,16 @@ __device__ __forceinline__ KeyAcc stage_of(const PartView &V, const RowSrc &r, u
     KeyAcc s;
     s.base0 = gkeys + V.a0 + r.su;
     s.base1 = gkeys + (r.vglob ? r.sv : V.a0 + r.sv);
+    s.d0 = r.du;
+    return s;
+}
+
+// where own row i (leader, sources r) stages its merged entries
+__device__ __forceinline__ KeyAcc stage_at(const PartView &V, const RowSrc &r, unsigned long long *gkeys, int32_t i) {
+    if (!V.sstage) return stage_of(V, r, gkeys);
+    KeyAcc s;
+    s.base0 = V.sst + V.cnt[i];
+    s.base1 = s.base0 + r.du;
     s.d0 = r.du;
     return s;
 }
@@ -856,6 +871,31 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
         // then copied to its final offset ----
         t0 = prof_now(a);
         part_fetch(&s_mbar, mph, V.win, o.CM + V.wlo, V.wlen);
+        {  // staging: shared memory after the window when the rows' upper bounds fit, else global
+            int32_t myub = 0;
+            for (int32_t i = i0; i < i1; ++i) {
+                const int32_t m = V.M[i];
+                if (V.lo + i <= m) {
+                    const RowSrc r = row_src(V, i, m);
+                    myub += r.du + r.dv;
+                }
+            }
+            int32_t ubtot;
+            int32_t ro = block_excl_scan<kPT>(myub, s_scan, ubtot);
+            int32_t *sb = V.win + ((V.wlen + 3) & ~3);
+            V.sst = reinterpret_cast<unsigned long long *>(sb);
+            V.sstage = !a.force_gstage && 2LL * ubtot + 4 <= (long long)(kPartBudget - (int32_t)(sb - sw));
+            if (V.sstage)
+                for (int32_t i = i0; i < i1; ++i) {
+                    const int32_t m = V.M[i];
+                    if (V.lo + i <= m) {
+                        const RowSrc r = row_src(V, i, m);
+                        V.cnt[i] = ro;  // this row's upper-bound offset in the staging
+                        ro += r.du + r.dv;
+                    }
+                }
+            __syncthreads();
+        }
         PT_MARK();
         // rows of > 16 merged entries, in sweeps over windows of kPT vertices: 17..32 by half
         // warps, 33..64 by warps, longer by the whole CTA
@@ -914,12 +954,12 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
                     ii = s_lists[0][qi];
                     r = row_src(V, ii, V.M[ii]);
                     cc = V.wget(o.CM, V.lo + ii);
-                    st = stage_of(V, r, a.wkeys);
+                    st = stage_at(V, r, a.wkeys, ii);
                 } else {
                     r.du = r.dv = 0;  // idle segment: all padding
                     r.su = r.sv = 0;
                     r.vglob = false;
-                    st = stage_of(V, r, a.wkeys);
+                    st = stage_of(V, r, a.wkeys);  // (unused: no entries)
                 }
                 const int32_t k2 = merge_seg(V, o.CM, r, cc, st, wbuf + half * 32);
                 if (ii >= 0 && (lane & 15) == 0) V.cnt[ii] = k2;
@@ -928,14 +968,14 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             for (int32_t q = wid; q < nB; q += kPW) {
                 const int32_t ii = s_lists[1][q];
                 const RowSrc r = row_src(V, ii, V.M[ii]);
-                const int32_t k2 = merge_warp(V, o.CM, r, V.wget(o.CM, V.lo + ii), stage_of(V, r, a.wkeys), wbuf);
+                const int32_t k2 = merge_warp(V, o.CM, r, V.wget(o.CM, V.lo + ii), stage_at(V, r, a.wkeys, ii), wbuf);
                 if (lane == 0) V.cnt[ii] = k2;
             }
             for (int32_t q = wid; q < nW; q += kPW) {
                 const int32_t ii = s_lists[2][q];
                 const RowSrc r = row_src(V, ii, V.M[ii]);
                 const int32_t k2 =
-                    merge_warp_smem(V, o.CM, r, V.wget(o.CM, V.lo + ii), stage_of(V, r, a.wkeys), wbuf);
+                    merge_warp_smem(V, o.CM, r, V.wget(o.CM, V.lo + ii), stage_at(V, r, a.wkeys, ii), wbuf);
                 if (lane == 0) V.cnt[ii] = k2;
             }
             __syncthreads();
@@ -944,7 +984,7 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
                 const int32_t ii = s_lists[3][q];
                 const RowSrc r = row_src(V, ii, V.M[ii]);
                 const int32_t k2 =
-                    merge_cta(V, o.CM, r, V.wget(o.CM, V.lo + ii), stage_of(V, r, a.wkeys), skeys, s_scan);
+                    merge_cta(V, o.CM, r, V.wget(o.CM, V.lo + ii), stage_at(V, r, a.wkeys, ii), skeys, s_scan);
                 if (t == 0) V.cnt[ii] = k2;
                 __syncthreads();
             }
@@ -980,7 +1020,7 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             const bool narrow = lead && ub <= 16;
             const bool all8 = __all_sync(0xffffffffu, !narrow || ub <= 8);
             if (narrow) {
-                const KeyAcc st = stage_of(V, r, a.wkeys);
+                const KeyAcc st = stage_at(V, r, a.wkeys, i);
                 const int32_t cu = V.wget(o.CM, V.lo + i);
                 V.cnt[i] = all8 ? merge_thread<8>(V, o.CM, r, cu, st) : merge_thread<16>(V, o.CM, r, cu, st);
             }
@@ -1025,7 +1065,59 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             ctl->bnd[0] = 0;
             ctl->bnd[nnext] = nc;
         }
-        {
+        if (V.sstage) {
+            // cadjp, bounds, and per vertex: M := the row's staging offset, cnt := its output
+            // offset in the CTA's range (running, so non-leaders keep offsets monotone); then the
+            // CTA's output copied in one coalesced sweep (an element's row: the last vertex
+            // whose output offset is <= the element's, by binary search)
+            int32_t ru = 0, ro = cex;
+            {
+                int32_t myub = 0;  // this thread's staging base = the exclusive scan of upper bounds
+                for (int32_t i = i0; i < i1; ++i) {
+                    const int32_t m = V.M[i];
+                    if (V.lo + i <= m) {
+                        const RowSrc r = row_src(V, i, m);
+                        myub += r.du + r.dv;
+                    }
+                }
+                int32_t ubtot;
+                ru = block_excl_scan<kPT>(myub, s_scan, ubtot);
+            }
+            for (int32_t i = i0; i < i1; ++i) {
+                const int32_t u = V.lo + i, m = V.M[i];
+                if (u > m) {
+                    V.cnt[i] = ro;
+                    continue;
+                }
+                const RowSrc r = row_src(V, i, m);
+                const int32_t cc = V.wget(o.CM, u), k2 = V.cnt[i];
+                const int32_t pos = s_b[4] + ro;
+                o.cadjp[cc] = pos;
+                if (nnext > 1) {
+                    const long long W0 = 2LL * pos + 5LL * cc, W1 = W0 + 2LL * k2 + 5;
+                    long long j = (W0 * nnext + Wt - 1) / Wt;
+                    if (j < 1) j = 1;
+                    for (; j < nnext && (j * Wt) / nnext < W1; ++j) ctl->bnd[j] = cc;
+                }
+                V.M[i] = ru;
+                V.cnt[i] = ro;
+                ru += r.du + r.dv;
+                ro += k2;
+            }
+            __syncthreads();
+            const int32_t gbase = s_b[4];
+            for (int32_t e = t; e < ctot; e += kPT) {
+                int32_t lo2 = 0, hi2 = V.nv;  // last i with cnt[i] <= e
+                while (hi2 - lo2 > 1) {
+                    const int32_t mid = (lo2 + hi2) >> 1;
+                    if (V.cnt[mid] <= e) lo2 = mid;
+                    else hi2 = mid;
+                }
+                const unsigned long long kv = V.sst[V.M[lo2] + (e - V.cnt[lo2])];
+                __stcg(o.cadjncy + gbase + e, (int32_t)(kv >> 32));
+                __stcg(o.cadjwgt + gbase + e, (int32_t)(uint32_t)kv);
+            }
+        } else {
             int32_t pos = s_b[4] + cex;
             for (int32_t i = i0; i < i1; ++i) {
                 const int32_t u = V.lo + i, m = V.M[i];
@@ -1178,6 +1270,7 @@ gp_status enqueue_part(Ctx *ctx, const PartLaunch &L) {
     a.wmin = part_wmin();
     a.force_garcs = part_knob("GP_PART_GARCS");
     a.wcap_max = part_knob("GP_PART_WCAP");
+    a.force_gstage = part_knob("GP_PART_GSTAGE");
     a.prof = part_knob("GP_PROF") == 1 ? 1 : 0;
     a.trace = getenv("GP_DEBUG") ? 1 : 0;
     {

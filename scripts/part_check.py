@@ -18,8 +18,9 @@ MODES = {
     "part": {"GP_SMALL": "0"},
     "part_many": {"GP_SMALL": "0", "GP_PART_W": "256"},
     "part_global": {"GP_SMALL": "0", "GP_PART_W": "256", "GP_PART_GARCS": "1", "GP_PART_WCAP": "64"},
+    "part_gstage": {"GP_SMALL": "0", "GP_PART_GSTAGE": "1"},
 }
-KN = ("GP_SMALL", "GP_PART_W", "GP_PART_GARCS", "GP_PART_WCAP", "GP_PART")
+KN = ("GP_SMALL", "GP_PART_W", "GP_PART_GARCS", "GP_PART_WCAP", "GP_PART", "GP_PART_GSTAGE")
 
 
 def star(k, wmax=100):

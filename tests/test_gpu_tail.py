@@ -10,6 +10,8 @@ bit-identical to the oracle and to the level kernels, in every mode:
                                       and arcs cross CTA ranges)
   part_global (+ GP_PART_GARCS=1, GP_PART_WCAP=64)  rows and most window lookups read from
                                       global memory (the paths of graphs that do not fit)
+  part_gstage (GP_SMALL=0, GP_PART_GSTAGE=1)  merged rows staged in global memory (levels whose
+                                      merged rows do not fit shared memory) instead of shared
   medium   (GP_SMALL=0, GP_MEDIUM=1)  the cluster kernel (opt-in: measured slower)
   levels   (GP_SMALL=0, GP_MEDIUM=0, GP_PART=0)  the grid-wide level kernels only."""
 import os
@@ -42,10 +44,11 @@ MODES = {
     "part": {"GP_SMALL": "0"},
     "part_many": {"GP_SMALL": "0", "GP_PART_W": "256"},
     "part_global": {"GP_SMALL": "0", "GP_PART_W": "256", "GP_PART_GARCS": "1", "GP_PART_WCAP": "64"},
+    "part_gstage": {"GP_SMALL": "0", "GP_PART_GSTAGE": "1"},
     "medium": {"GP_SMALL": "0", "GP_MEDIUM": "1"},
     "levels": {"GP_SMALL": "0", "GP_MEDIUM": "0", "GP_PART": "0"},
 }
-KNOBS = ("GP_SMALL", "GP_MEDIUM", "GP_PART", "GP_PART_W", "GP_PART_GARCS", "GP_PART_WCAP")
+KNOBS = ("GP_SMALL", "GP_MEDIUM", "GP_PART", "GP_PART_W", "GP_PART_GARCS", "GP_PART_WCAP", "GP_PART_GSTAGE")
 
 
 def _run(gp, ctx, g, mode, **kw):
@@ -147,3 +150,24 @@ def test_windowed_match_opt_in(gp, ctx, name):
                 os.environ.pop(k, None)
             else:
                 os.environ[k] = v
+
+
+@pytest.mark.parametrize("mode", ["small", "part", "part_many"])
+@pytest.mark.parametrize("name", ["C1", "C3_128", "star1500"])
+def test_tail_continues_across_launches(gp, ctx, name, mode):
+    """A tail launch holds at most GP_TAIL_SLOTS levels (default 12); a deeper hierarchy
+    continues with further launches from the last tail level's output.  With 2 slots every
+    hierarchy here needs several launches: still bit-identical to the oracle."""
+    make, kw = CASES[name]
+    g = make()
+    ref = oracle.coarsen_to(g, **kw)
+    old = os.environ.get("GP_TAIL_SLOTS")
+    os.environ["GP_TAIL_SLOTS"] = "2"
+    try:
+        got, launches = _run(gp, ctx, g, mode, **kw)
+        assert_levels_equal(got, ref, f"{name} {mode} 2 slots")
+    finally:
+        if old is None:
+            os.environ.pop("GP_TAIL_SLOTS", None)
+        else:
+            os.environ["GP_TAIL_SLOTS"] = old
