@@ -83,11 +83,27 @@ struct PartArgs {
     int32_t force_garcs;             // test knob: arcs always read from global memory
     int32_t wcap_max;                // test knob: window capacity cap (words; 0 = none)
     int32_t force_gstage;            // test knob: contraction staging in global memory
+    int32_t cap_n, cap_nnz;          // slot / staging capacities (the first level's bounds)
     int32_t prof;                    // GP_PROF=1: slowest CTA per round / contraction step
     int32_t trace;                   // GP_DEBUG: phase timestamps of block 0 (globaltimer reads cost)
 };
 
 __device__ __forceinline__ int32_t pld(const int32_t *p) { return __ldcg(p); }
+// GP_PART_CHECK builds: every shared / staging / output index is range-checked (a violation
+// prints and traps) -- the memory-safety check of this kernel where compute-sanitizer is not
+// available (tests run under it: scripts/part_checked.sh)
+#ifdef GP_PART_CHECK
+#define PCHK(cond, what, v)                                                                        \
+    do {                                                                                           \
+        if (!(cond)) {                                                                             \
+            printf("k_part check failed: %s (%lld) block %d thread %d\n", what, (long long)(v),    \
+                   (int)blockIdx.x, (int)threadIdx.x);                                             \
+            __trap();                                                                              \
+        }                                                                                          \
+    } while (0)
+#else
+#define PCHK(cond, what, v) do { } while (0)
+#endif
 // v, or *gp (ld.global.cg) when useg: a predicated load instead of a branch
 __device__ __forceinline__ int32_t ld_or(int32_t v, const int32_t *gp, bool useg) {
     asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.global.cg.s32 %0, [%1];\n\t}"
@@ -205,10 +221,21 @@ struct PartView {
     // entries at sst[cnt[i]] (cnt holds the rows' upper-bound offsets while merging)
     unsigned long long *sst;
     bool sstage;
+    int32_t sstot;   // staging entries (upper bounds) in shared memory (checks)
+    int32_t capnnz;  // global staging / output capacity (checks)
     // row start of own vertex i relative to a0 (i in [0, nv])
-    __device__ __forceinline__ int32_t rs(int32_t i) const { return sap[i + loff] - a0; }
-    __device__ __forceinline__ int32_t arc(int32_t j) const { return garcs ? pld(gadjncy + a0 + j) : sadj[j + aoff]; }
-    __device__ __forceinline__ int32_t wgt(int32_t j) const { return garcs ? pld(gadjwgt + a0 + j) : swgt[j + aoff]; }
+    __device__ __forceinline__ int32_t rs(int32_t i) const {
+        PCHK(i >= 0 && i <= nv, "row index", i);
+        return sap[i + loff] - a0;
+    }
+    __device__ __forceinline__ int32_t arc(int32_t j) const {
+        PCHK(j >= 0 && j < na, "arc index", j);
+        return garcs ? pld(gadjncy + a0 + j) : sadj[j + aoff];
+    }
+    __device__ __forceinline__ int32_t wgt(int32_t j) const {
+        PCHK(j >= 0 && j < na, "arc index", j);
+        return garcs ? pld(gadjwgt + a0 + j) : swgt[j + aoff];
+    }
     // window lookup of a global array g (P_k or CM) at x
     // branch-free: the shared load always issues (at index 0 when outside), the global load is
     // predicated -- a branch per lookup serialised the unrolled lookups of a row (no ILP)
@@ -346,6 +373,8 @@ __device__ __forceinline__ unsigned long long row_key(const PartView &V, const i
         w = pld((g ? V.gadjwgt : V.gadjwgt + V.a0) + j);
     } else {
         const int32_t jl = g ? 0 : j + V.aoff;  // a valid shared index either way
+        PCHK(g || (j >= 0 && j < V.na), "own row arc", j);
+        PCHK(!g || (j >= 0 && j < V.capnnz), "foreign row arc", j);
         x = ld_or(V.sadj[jl], V.gadjncy + j, g);
         w = ld_or(V.swgt[jl], V.gadjwgt + j, g);
     }
@@ -361,6 +390,7 @@ struct KeyAcc {
     unsigned long long *base0, *base1;
     int32_t d0;
     __device__ __forceinline__ unsigned long long &operator()(int32_t e) const {
+        PCHK(e >= 0, "staging entry", e);
         return e < d0 ? base0[e] : base1[e - d0];
     }
 };
@@ -376,6 +406,7 @@ __device__ __forceinline__ KeyAcc stage_of(const PartView &V, const RowSrc &r, u
 __device__ __forceinline__ KeyAcc stage_at(const PartView &V, const RowSrc &r, unsigned long long *gkeys, int32_t i) {
     if (!V.sstage) return stage_of(V, r, gkeys);
     KeyAcc s;
+    PCHK(V.cnt[i] >= 0 && V.cnt[i] + r.du + r.dv <= V.sstot, "shared staging slot", V.cnt[i]);
     s.base0 = V.sst + V.cnt[i];
     s.base1 = s.base0 + r.du;
     s.d0 = r.du;
@@ -638,6 +669,10 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
         V.gadjp = gadjp;
         V.gadjncy = gadjncy;
         V.gadjwgt = gadjwgt;
+        V.capnnz = a.cap_nnz;
+        V.sstage = false;
+        V.sstot = 0;
+        PCHK(n <= a.cap_n && nnz <= a.cap_nnz, "level size within the slot bounds", nnz);
         if (level == 0) {
             const long long W = 2LL * nnz + 5LL * n;
             V.lo = b == 0 ? 0 : part_search(gadjp, n, (long long)b * W / nact);
@@ -716,6 +751,7 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             if (wh - wl > wcap) wh = wl + wcap;
             V.wlo = (int32_t)wl;
             V.wlen = (int32_t)(wh - wl) > 0 ? (int32_t)(wh - wl) : 0;
+            PCHK((int32_t)(V.win - sw) + V.wlen <= kPartBudget, "window in shared memory", V.wlen);
             __syncthreads();
         }
         PT_MARK();
@@ -885,6 +921,7 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             int32_t *sb = V.win + ((V.wlen + 3) & ~3);
             V.sst = reinterpret_cast<unsigned long long *>(sb);
             V.sstage = !a.force_gstage && 2LL * ubtot + 4 <= (long long)(kPartBudget - (int32_t)(sb - sw));
+            V.sstot = ubtot;
             if (V.sstage)
                 for (int32_t i = i0; i < i1; ++i) {
                     const int32_t m = V.M[i];
@@ -1114,6 +1151,8 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
                     else hi2 = mid;
                 }
                 const unsigned long long kv = V.sst[V.M[lo2] + (e - V.cnt[lo2])];
+                PCHK(V.M[lo2] >= 0 && V.M[lo2] + (e - V.cnt[lo2]) < V.sstot, "staged entry", e);
+                PCHK(gbase + e < V.capnnz, "coarse arc", gbase + e);
                 __stcg(o.cadjncy + gbase + e, (int32_t)(kv >> 32));
                 __stcg(o.cadjwgt + gbase + e, (int32_t)(uint32_t)kv);
             }
@@ -1133,6 +1172,7 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
 #pragma unroll
                     for (int q = 0; q < 16; ++q)
                         if (q0 + q < k2) {
+                            PCHK(pos + q0 + q < V.capnnz, "coarse arc", pos + q0 + q);
                             o.cadjncy[pos + q0 + q] = (int32_t)(kv[q] >> 32);
                             o.cadjwgt[pos + q0 + q] = (int32_t)(uint32_t)kv[q];
                         }
@@ -1271,6 +1311,8 @@ gp_status enqueue_part(Ctx *ctx, const PartLaunch &L) {
     a.force_garcs = part_knob("GP_PART_GARCS");
     a.wcap_max = part_knob("GP_PART_WCAP");
     a.force_gstage = part_knob("GP_PART_GSTAGE");
+    a.cap_n = L.cap_n;
+    a.cap_nnz = L.cap_nnz;
     a.prof = part_knob("GP_PROF") == 1 ? 1 : 0;
     a.trace = getenv("GP_DEBUG") ? 1 : 0;
     {
