@@ -80,6 +80,7 @@ struct ContractArgs {
     // single-pass coarse CSR assembly (single GPU): decoupled look-back over the C2 warp tiles
     unsigned long long *status;  // one status word per tile (ctx->status; epoch-tagged, never reset)
     uint32_t epoch;
+    int32_t warp_max;  // single GPU: rows up to this bound merged by a warp in C2a (kWB..2*kWB)
     int32_t knobs;  // bit 0: route 65..kWB rows of small levels to C1h (GP_C1H_SMALL=1); bit 1: two-pass only (GP_C2_SP=0)
 };
 __device__ __forceinline__ bool small_hub_on(const ContractArgs &a) { return a.knobs & 1; }
@@ -1051,8 +1052,11 @@ __global__ void __launch_bounds__(kCNT, kMinB) k_contract_level(const __grid_con
     // of small levels (about one C2 tile per warp) to C1h -- measured slower on C3 (C1h took
     // ~20 us at L10/L11 for a few rows per CTA), so off by default.  Sharded levels keep kWB
     // (dist.cu builds their C1h list).
-    const int32_t hub_ub =
-        (a.dist || (long long)n > 32LL * 2 * g_cact * kCW || !small_hub_on(a)) ? kWB : kWarpNet;
+    // Single-GPU levels route rows of up to 2*kWB entries (one row then fills a warp's slot
+    // area) to the warp merges: on R-MAT (C4) the C1h rows of 257..512 entries, one CTA each
+    // with a block-wide sort, were most of the contraction (31-38 ms of ~42 ms per level).
+    const int32_t hub_ub = a.dist ? kWB
+                           : ((long long)n > 32LL * 2 * g_cact * kCW || !small_hub_on(a)) ? a.warp_max : kWarpNet;
     const int T1 = (nt1 + g_cact - 1) / g_cact;            // C1b tiles per CTA
     trace_mark(ctl->trace, 0);
     if (n > 0 && !a.dist) {
@@ -1226,6 +1230,9 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
     {
         const char *e1 = getenv("GP_C1H_SMALL"), *e2 = getenv("GP_C2_SP");  // tuning knobs (results never depend on them)
         a.knobs = ((e1 && atoi(e1) == 1) ? 1 : 0) | ((e2 && atoi(e2) == 0) ? 2 : 0);
+        const char *e3 = getenv("GP_WARP_ROW_MAX");  // tuning knob (results never depend on it)
+        const int wm = e3 ? atoi(e3) : 2 * kWB;
+        a.warp_max = wm < kWarpNet ? kWarpNet : wm > 2 * kWB ? 2 * kWB : wm;
     }
     if (!prm.dist) {
         const size_t tiles = ((size_t)(prm.n_bound > 0 ? prm.n_bound : 1) + kRT - 1) / kRT + 1;
