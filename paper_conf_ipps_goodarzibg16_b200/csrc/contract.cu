@@ -81,6 +81,7 @@ struct ContractArgs {
     unsigned long long *status;  // one status word per tile (ctx->status; epoch-tagged, never reset)
     uint32_t epoch;
     int32_t warp_max;  // single GPU: rows up to this bound merged by a warp in C2a (kWB..2*kWB)
+    int32_t giant_ub;  // single GPU: C1h rows longer than this merged by the whole grid (0: off)
     int32_t knobs;  // bit 0: route 65..kWB rows of small levels to C1h (GP_C1H_SMALL=1); bit 1: two-pass only (GP_C2_SP=0)
 };
 __device__ __forceinline__ bool small_hub_on(const ContractArgs &a) { return a.knobs & 1; }
@@ -275,6 +276,10 @@ __device__ void phase_c1b(const ContractArgs &a, ContractSmem &sm, int32_t n, in
                 a.off[cc] = oo;
                 a.seg[cc] = make_int4(su[i], dl, sv[i], d - dl);
                 if (d > hub_ub) a.huge[atomicAdd(&a.ctl->n_huge, 1)] = cc;
+                if (a.giant_ub > 0 && d > a.giant_ub) {  // merged by the whole grid (phase_c1h_giant)
+                    const int32_t gi = atomicAdd(&a.ctl->n_giant, 1);
+                    if (gi < kMaxGiant) a.ctl->giant[gi] = cc;
+                }
             }
             c += __popc(bl);
             o += dtot;
@@ -442,15 +447,105 @@ __device__ int32_t long_runsum_compact(ContractSmem &sm, unsigned long long *key
 }
 
 // ---------------------------------------------------------------------------------------
+// C1h giant rows (single GPU, ub > giant_ub: R-MAT hubs of 10^5 arcs): merged by the WHOLE
+// grid one row at a time through a dense accumulator over the coarse ids (the idle `lofs`)
+// and a presence bitmap (the idle `tout`): every CTA adds its share of the row's arcs into
+// acc[CM[x]] (weights summed, R8; collapsed edge dropped, R9), the first add of an id sets its
+// bit; each CTA then counts the bits of its slice of the bitmap, and after a prefix over the
+// CTAs writes its ids in increasing order (rows come out sorted by coarse id, R10), resetting
+// both as it goes.  ~3 grid barriers and nc / 32 words per row, whatever the row length.
+// One CTA sorting a 400 K-key hub row took 25-29 ms and was the whole C1h phase on C4.
+// ---------------------------------------------------------------------------------------
+__device__ __noinline__ void phase_c1h_giant(const ContractArgs &a, ContractSmem &sm, int32_t ng, int32_t nc,
+                                             unsigned &bar_epoch) {
+    ContractCtl *ctl = a.ctl;
+    int32_t *acc = a.lofs;                                     // weights by coarse id
+    uint32_t *bm = reinterpret_cast<uint32_t *>(a.tout);       // presence bits (tout: idle until C2a)
+    const int32_t nw = (nc + 31) >> 5;
+    const long long gthreads = (long long)g_cact * kCNT, gtid = (long long)blockIdx.x * kCNT + threadIdx.x;
+    for (long long i = gtid; i < nc; i += gthreads) acc[i] = 0;
+    for (long long i = gtid; i < nw; i += gthreads) bm[i] = 0u;
+    grid_barrier(ctl->bar, bar_epoch, g_cact);
+    // this CTA's bitmap words [w0, w1) = coarse ids [32 w0, 32 w1)
+    const int32_t w0 = (int32_t)((long long)nw * blockIdx.x / g_cact);
+    const int32_t w1 = (int32_t)((long long)nw * (blockIdx.x + 1) / g_cact);
+    const int32_t per = (w1 - w0 + kCNT - 1) / kCNT;  // words per thread (contiguous: id order)
+    const int32_t t0w = min(w1, w0 + (int32_t)threadIdx.x * per), t1w = min(w1, t0w + per);
+    for (int32_t gi = 0; gi < ng; ++gi) {
+        const int32_t c = ctl->giant[gi];
+        const int32_t o0 = __ldcg(a.off + c);
+        const int32_t ub = __ldcg(a.off + c + 1) - o0;
+        const int4 sg = __ldcg(a.seg + c);
+        for (long long p = gtid; p < ub; p += gthreads) {
+            const int32_t pi = (int32_t)p;
+            const int32_t j = pi < sg.y ? sg.x + pi : sg.z + (pi - sg.y);
+            const int32_t cx = ldCM(a.CM + __ldcs(a.adjncy + j));
+            if (cx != c + a.cbase) {
+                if (atomicAdd(acc + cx, __ldcs(a.adjwgt + j)) == 0) atomicOr(bm + (cx >> 5), 1u << (cx & 31));
+            }
+        }
+        grid_barrier(ctl->bar, bar_epoch, g_cact);
+        int32_t mine = 0;
+        for (int32_t w = t0w; w < t1w; ++w) mine += __popc(__ldcg(bm + w));
+        int32_t tot;
+        const int32_t ex = block_excl_scan<kCNT>(mine, sm.scan, tot);
+        if (threadIdx.x == 0) ctl->chunk2[blockIdx.x] = tot;  // (C2's chunk sums: idle until C2)
+        grid_barrier(ctl->bar, bar_epoch, g_cact);
+        if (threadIdx.x < 32) {
+            int32_t pre = 0, all = 0;
+            for (int q = threadIdx.x; q < g_cact; q += 32) {
+                const int32_t x = __ldcg(ctl->chunk2 + q);
+                all += x;
+                pre += q < (int)blockIdx.x ? x : 0;
+            }
+            pre = warp_sum(pre);
+            all = warp_sum(all);
+            if (threadIdx.x == 0) {
+                sm.last = pre;
+                if (blockIdx.x == 0) a.cnt[c] = all;
+            }
+        }
+        __syncthreads();
+        unsigned long long *dst = a.gkeys + o0;
+        int32_t wr = sm.last + ex;
+        for (int32_t w = t0w; w < t1w; ++w) {  // ids in increasing order: rows sorted by coarse id (R10)
+            uint32_t bits = __ldcg(bm + w);
+            if (!bits) continue;
+            bm[w] = 0u;
+            while (bits) {
+                const int b = __ffs(bits) - 1;
+                bits &= bits - 1;
+                const int32_t cx = (w << 5) + b;
+                dst[wr++] = ckey(cx, __ldcg(acc + cx));  // summed weight (R8); fits int32 (R14)
+                acc[cx] = 0;
+            }
+        }
+        __syncthreads();
+        grid_barrier(ctl->bar, bar_epoch, g_cact);  // the accumulator is clean for the next row
+    }
+    // chunk2 accumulates C2's per-CTA sums by atomics from zero: clear this CTA's entry (made
+    // visible by the grid barrier that follows C1h)
+    if (ng > 0 && threadIdx.x == 0) ctl->chunk2[blockIdx.x] = 0;
+}
+
+// ---------------------------------------------------------------------------------------
 // C1h: rows with ub > kWB, one CTA each; result compacted at gkeys[off[c]], count cnt[c]
 // ---------------------------------------------------------------------------------------
-__device__ __noinline__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, int32_t nh) {
+__device__ __noinline__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, int32_t nh, bool giant_done) {
     // rows are claimed dynamically (first one static): a CTA busy with a 400 K-key hub row
     // takes no further rows, instead of a fixed 1/nact share of them
     for (int i = blockIdx.x; i < nh;) {
         const int32_t c = a.huge[i];
         const int32_t o0 = __ldcg(a.off + c);
         const int32_t ub = __ldcg(a.off + c + 1) - o0;
+        if (giant_done && ub > a.giant_ub) {  // merged by the whole grid already
+            if (threadIdx.x == 0) sm.last = g_cact + (int)atomicAdd(&a.ctl->hub_ctr, 1u);
+            __syncthreads();
+            i = sm.last;
+            __syncthreads();
+            continue;
+        }
+        const unsigned long long tc0 = a.prof ? globaltimer() : 0ull;
         unsigned long long *dst = a.gkeys + o0;
         unsigned long long *keys = (ub <= kCtaRow) ? sm.buf : dst;
         // gather at fixed positions (leader's arcs, then the partner's; 4 per thread in flight);
@@ -506,6 +601,10 @@ __device__ __noinline__ void phase_c1h(const ContractArgs &a, ContractSmem &sm, 
         if (threadIdx.x == 0) {
             a.cnt[c] = cnt;
             sm.last = g_cact + (int)atomicAdd(&a.ctl->hub_ctr, 1u);
+            if (a.prof) {  // GP_PROF=1: C1h rows: sum of upper bounds; slowest row (ns << 32 | ub)
+                atomicAdd(&a.ctl->dbg[6], (unsigned long long)ub);
+                atomicMax(&a.ctl->dbg[7], ((globaltimer() - tc0) << 24) | (unsigned long long)min(ub, (1 << 24) - 1));
+            }
         }
         __syncthreads();
         i = sm.last;
@@ -1072,7 +1171,11 @@ __global__ void __launch_bounds__(kCNT, kMinB) k_contract_level(const __grid_con
     const int32_t nc = *(volatile int32_t *)&ctl->n_coarse;
     const int32_t nh = *(volatile int32_t *)&ctl->n_huge;
     if (nh > 0) {
-        phase_c1h(a, sm, nh);
+        const int32_t ng = a.dist ? 0 : *(volatile int32_t *)&ctl->n_giant;
+        // (an overflowing list, or a bitmap larger than tout: every row per CTA)
+        const bool giant = ng > 0 && ng <= kMaxGiant && ((long long)nc + 31) / 32 <= 2LL * nnz_in;
+        if (giant) phase_c1h_giant(a, sm, ng, nc, bar_epoch);
+        phase_c1h(a, sm, nh, giant);
         grid_barrier(ctl->bar, bar_epoch, g_cact);
     }
     trace_mark(ctl->trace, 5);
@@ -1233,6 +1336,12 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
         const char *e3 = getenv("GP_WARP_ROW_MAX");  // tuning knob (results never depend on it)
         const int wm = e3 ? atoi(e3) : 2 * kWB;
         a.warp_max = wm < kWarpNet ? kWarpNet : wm > 2 * kWB ? 2 * kWB : wm;
+        // Opt-in (GP_GIANT_ROW=<ub>): bit-exact (tests/test_gpu_giant.py, C4 identical to the
+        // per-CTA path), but measured slower on C4 (contraction 122 -> 132 ms): ~140 rows per
+        // level over 65536 entries cost ~40 us each across the grid, and the rows of 8 K..64 K
+        // entries left to single CTAs (~4 s of CTA time per level) still set the phase's length.
+        const char *e4 = getenv("GP_GIANT_ROW");  // knob (results never depend on it)
+        a.giant_ub = prm.dist ? 0 : (e4 ? atoi(e4) : 0);
     }
     if (!prm.dist) {
         const size_t tiles = ((size_t)(prm.n_bound > 0 ? prm.n_bound : 1) + kRT - 1) / kRT + 1;

@@ -833,6 +833,11 @@ gp_status coarsen_single(Graph *g, const gp_coarsen_opts *opts, Hier **out) {
                 for (int q = 1; q < 9; ++q)
                     fprintf(stderr, " %.1f", ct[q] && ct[q - 1] ? ((long long)ct[q] - (long long)ct[q - 1]) * 1e-3 : 0.0);
                 fprintf(stderr, " | gap to contract %.1f us\n", ct[0] && mt[1] ? ((long long)ct[0] - (long long)mt[0]) * 1e-3 : 0.0);
+                if (hd[l].contract.dbg[6]) {
+                    const unsigned long long *d = hd[l].contract.dbg;
+                    fprintf(stderr, "[gp]   c1h rows: sum of upper bounds %llu, slowest row %.1f us (ub %llu)\n", d[6],
+                            (d[7] >> 24) * 1e-3, d[7] & 0xFFFFFFull);
+                }
                 if (hd[l].contract.dbg[4]) {
                     const unsigned long long *d = hd[l].contract.dbg;
                     fprintf(stderr, "[gp]   c2a tiles %llu: slowest %.1f us (tile %llu), mean %.2f us, max warp-merged rows %llu (tile %llu), max rows %llu, warp-merged rows %llu\n",
