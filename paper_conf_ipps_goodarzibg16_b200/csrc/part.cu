@@ -111,9 +111,6 @@ __device__ __forceinline__ int32_t ld_or(int32_t v, const int32_t *gp, bool useg
         : "l"(gp), "r"((unsigned)useg));
     return v;
 }
-#ifdef GP_PART_DBG
-__shared__ int32_t g_part_miss;  // window misses of this CTA (debug builds)
-#endif
 
 // grid barrier over the nact CTAs still running (the count only grows: a barrier completes at
 // the running sum of the participants of all barriers so far)
@@ -242,9 +239,6 @@ struct PartView {
     __device__ __forceinline__ int32_t wget(const int32_t *g, int32_t x) const {
         const unsigned d = (unsigned)(x - wlo);
         const bool out = d >= (unsigned)wlen;
-#ifdef GP_PART_DBG
-        if (out) atomicAdd(&g_part_miss, 1);
-#endif
         return ld_or(win[out ? 0u : d], g + x, out);
     }
 };
@@ -760,14 +754,6 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
         int32_t rounds = 0, maximal = 0;
         MatchCtl *mc = &a.levdev[gl].match;
         unsigned long long t0 = prof_now(a);
-#ifdef GP_PART_DBG
-        unsigned long long dd[20] = {};
-        int ndd = 0;
-        if (t == 0) g_part_miss = 0;
-#define PT_DD() do { if (ndd < 20) dd[ndd++] = globaltimer() - t0; } while (0)
-#else
-#define PT_DD() do { } while (0)
-#endif
         {  // round-1 proposals: every vertex is free (phase g)
             int32_t mylive = 0;
             // one row per thread: no freedom test in round 1, so a row is a short chain of
@@ -782,7 +768,6 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             }
             PT_MARK();
             prof_max(a, &mc->wmax[0], t0);
-            PT_DD();
             round_bar(ctl, btarget, nact, g, mylive, 0, s_scan);
             PT_MARK();
             ++g;
@@ -807,7 +792,6 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             int32_t *Pk = (k & 1) ? a.P1 : a.P0;
             int32_t *Pn = (k & 1) ? a.P0 : a.P1;
             part_fetch(&s_mbar, mph, V.win, Pk + V.wlo, V.wlen);
-            if (k == 1) PT_DD();
             PT_MARK();
             int32_t mylive = 0, mypairs = 0;
             unsigned long long *slot = skeys + wid * 32;
@@ -849,13 +833,7 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
                 mylive += np >= 0;
             }
             PT_MARK();
-            if (k == 1) PT_DD();
-#ifdef GP_PART_DBG
-            __syncthreads();
-            if (k == 1) PT_DD();
-#endif
             if (k < 16) prof_max(a, &mc->wmax[k], t0);
-            PT_DD();
             round_bar(ctl, btarget, nact, g, mylive, mypairs, s_scan);
             PT_MARK();
             ++g;
@@ -936,15 +914,6 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
         PT_MARK();
         // rows of > 16 merged entries, in sweeps over windows of kPT vertices: 17..32 by half
         // warps, 33..64 by warps, longer by the whole CTA
-        PT_DD();
-#ifdef GP_PART_DBG
-        long long sw_c[4] = {0, 0, 0, 0};
-        int sw_n[4] = {0, 0, 0, 0};
-        long long swc = clock64();
-#define SW_CK(q) do { const long long c_ = clock64(); sw_c[q] += c_ - swc; swc = c_; } while (0)
-#else
-#define SW_CK(q) do { } while (0)
-#endif
         for (int32_t r0 = 0; r0 < V.nv; r0 += kPT) {
             if (t == 0) s_cnt3[0] = s_cnt3[1] = s_cnt3[2] = s_cnt3[3] = 0;
             __syncthreads();
@@ -972,13 +941,6 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             }
             __syncthreads();
             const int32_t nA = s_cnt3[0], nB = s_cnt3[1], nW = s_cnt3[2], nC = s_cnt3[3];
-            SW_CK(0);
-#ifdef GP_PART_DBG
-            sw_n[0] += nA;
-            sw_n[1] += nB;
-            sw_n[2] += nW;
-            sw_n[3] += nC;
-#endif
             if (nA + nB + nW + nC == 0) continue;
             unsigned long long *wbuf = skeys + wid * 256;  // this warp's shared-memory keys
             for (int32_t q = 2 * wid; q < nA; q += 2 * kPW) {  // two 17..32-entry rows per warp
@@ -1001,7 +963,6 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
                 const int32_t k2 = merge_seg(V, o.CM, r, cc, st, wbuf + half * 32);
                 if (ii >= 0 && (lane & 15) == 0) V.cnt[ii] = k2;
             }
-            SW_CK(1);
             for (int32_t q = wid; q < nB; q += kPW) {
                 const int32_t ii = s_lists[1][q];
                 const RowSrc r = row_src(V, ii, V.M[ii]);
@@ -1016,7 +977,6 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
                 if (lane == 0) V.cnt[ii] = k2;
             }
             __syncthreads();
-            SW_CK(2);
             for (int32_t q = 0; q < nC; ++q) {
                 const int32_t ii = s_lists[3][q];
                 const RowSrc r = row_src(V, ii, V.M[ii]);
@@ -1027,14 +987,6 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             }
         }
         PT_MARK();
-        SW_CK(3);
-#ifdef GP_PART_DBG
-        if (t == 0 && level == 4 && b < 8)
-            printf("PSW b=%d classify %lld seg %lld warp+ %lld cta %lld | rows %d %d %d %d\n", b, sw_c[0], sw_c[1], sw_c[2],
-                   sw_c[3], sw_n[0], sw_n[1], sw_n[2], sw_n[3]);
-#endif
-#undef SW_CK
-        PT_DD();
         // rows of <= 16 entries by their thread (contiguous blocks = coarse id order)
         // (warp-uniform steps: the 8-entry network runs when every merging lane's row fits it,
         // else all merging lanes run the 16-entry one -- divergent networks would run both)
@@ -1064,15 +1016,9 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
             if (lead) mine += V.cnt[i];
         }
         int32_t ctot;
-        PT_DD();
-#ifdef GP_PART_DBG
-        __syncthreads();
-        PT_DD();
-#endif
         const int32_t cex = block_excl_scan<kPT>(mine, s_scan, ctot);
         if (t == 0) ctl->nA[b] = ctot;
         prof_max(a, &mc->barr[0][0], t0);
-        PT_DD();
         PT_MARK();
         pbar(&ctl->bar, btarget, nact);
         PT_MARK();
@@ -1188,14 +1134,6 @@ __global__ void __launch_bounds__(kPT, 1) k_part(const __grid_constant__ PartArg
         }
         if (b == nact - 1 && t == 0) o.cadjp[nc] = cnnz;
         prof_max(a, &mc->barr[0][1], t0);
-        PT_DD();
-#ifdef GP_PART_DBG
-        if (t == 0 && level == 4)
-            printf("PDBG b=%d nv=%d na=%d wlen=%d garcs=%d miss=%d | %llu %llu %llu %llu %llu %llu %llu %llu %llu %llu %llu %llu %llu %llu %llu %llu %llu\n", b,
-                   V.nv, V.na, V.wlen, (int)V.garcs, g_part_miss, dd[0], dd[1], dd[2], dd[3], dd[4], dd[5], dd[6], dd[7],
-                   dd[8], dd[9], dd[10], dd[11], dd[12], dd[13], dd[14], dd[15], dd[16]);
-#endif
-#undef PT_DD
         PT_MARK();
         pbar(&ctl->bar, btarget, nact);
         // ---- statistics, stop rule (R12, R13), report ----
