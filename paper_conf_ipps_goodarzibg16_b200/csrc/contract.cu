@@ -30,6 +30,8 @@
 //  Rows come out sorted by coarse id (R10) with repeated coarse neighbours summed (R8) and
 //  the collapsed edge dropped (R9).
 #include <cuda_runtime.h>
+
+#include <algorithm>
 #include <stdlib.h>
 
 #include "device_util.cuh"
@@ -447,31 +449,50 @@ __device__ int32_t long_runsum_compact(ContractSmem &sm, unsigned long long *key
 }
 
 // ---------------------------------------------------------------------------------------
-// C1h giant rows (single GPU, ub > giant_ub: R-MAT hubs of 10^5 arcs): merged by the WHOLE
-// grid one row at a time through a dense accumulator over the coarse ids (the idle `lofs`)
-// and a presence bitmap (the idle `tout`): every CTA adds its share of the row's arcs into
+// C1h giant rows (single GPU, ub > giant_ub: R-MAT hubs of 10^4-10^5 arcs): merged by GROUPS
+// of CTAs, one row per group at a time, through a dense accumulator over the coarse ids and a
+// presence bitmap (both in the idle `tout`): every CTA adds its share of the row's arcs into
 // acc[CM[x]] (weights summed, R8; collapsed edge dropped, R9), the first add of an id sets its
 // bit; each CTA then counts the bits of its slice of the bitmap, and after a prefix over the
 // CTAs writes its ids in increasing order (rows come out sorted by coarse id, R10), resetting
-// both as it goes.  ~3 grid barriers and nc / 32 words per row, whatever the row length.
+// both as it goes.  ~3 group barriers and nc / 32 words per row, whatever the row length.
 // One CTA sorting a 400 K-key hub row took 25-29 ms and was the whole C1h phase on C4.
 // ---------------------------------------------------------------------------------------
+// barrier of the CTAs of one group (a running count: completes at the sum of the group's
+// arrivals so far)
+__device__ __forceinline__ void group_barrier(unsigned *bar, unsigned &target, unsigned gs) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        target += gs;
+        red_release_add_u32(bar, 1u);
+        const long long guard = spin_start();
+        while ((int)(ld_acquire_u32(bar) - target) < 0) spin_check(guard);
+    }
+    __syncthreads();
+}
+
 __device__ __noinline__ void phase_c1h_giant(const ContractArgs &a, ContractSmem &sm, int32_t ng, int32_t nc,
-                                             unsigned &bar_epoch) {
+                                             int32_t G) {
+    // G independent groups of CTAs (b % G), each with its own accumulator + bitmap region of
+    // the idle tout and its own barrier; group gb takes giant rows gb, gb + G, ...
     ContractCtl *ctl = a.ctl;
-    int32_t *acc = a.lofs;                                     // weights by coarse id
-    uint32_t *bm = reinterpret_cast<uint32_t *>(a.tout);       // presence bits (tout: idle until C2a)
     const int32_t nw = (nc + 31) >> 5;
-    const long long gthreads = (long long)g_cact * kCNT, gtid = (long long)blockIdx.x * kCNT + threadIdx.x;
+    const int gb = (int)blockIdx.x % G, r = (int)blockIdx.x / G;
+    const unsigned gs = (unsigned)((g_cact - gb + G - 1) / G);  // CTAs in this group
+    const size_t stride = ((size_t)nc + (size_t)nw + 64) & ~(size_t)31;
+    int32_t *acc = reinterpret_cast<int32_t *>(a.tout) + stride * gb;  // weights by coarse id
+    uint32_t *bm = reinterpret_cast<uint32_t *>(acc + nc + 32);        // presence bits
+    unsigned *gbar = ctl->gbar + gb;
+    unsigned gtarget = 0;  // (thread 0)
+    const long long gthreads = (long long)gs * kCNT, gtid = (long long)r * kCNT + threadIdx.x;
     for (long long i = gtid; i < nc; i += gthreads) acc[i] = 0;
     for (long long i = gtid; i < nw; i += gthreads) bm[i] = 0u;
-    grid_barrier(ctl->bar, bar_epoch, g_cact);
-    // this CTA's bitmap words [w0, w1) = coarse ids [32 w0, 32 w1)
-    const int32_t w0 = (int32_t)((long long)nw * blockIdx.x / g_cact);
-    const int32_t w1 = (int32_t)((long long)nw * (blockIdx.x + 1) / g_cact);
-    const int32_t per = (w1 - w0 + kCNT - 1) / kCNT;  // words per thread (contiguous: id order)
+    group_barrier(gbar, gtarget, gs);
+    // this CTA's bitmap words [w0, w1) = coarse ids [32 w0, 32 w1), per thread contiguous
+    const int32_t w0 = (int32_t)((long long)nw * r / gs), w1 = (int32_t)((long long)nw * (r + 1) / gs);
+    const int32_t per = (w1 - w0 + kCNT - 1) / kCNT;
     const int32_t t0w = min(w1, w0 + (int32_t)threadIdx.x * per), t1w = min(w1, t0w + per);
-    for (int32_t gi = 0; gi < ng; ++gi) {
+    for (int32_t gi = gb; gi < ng; gi += G) {
         const int32_t c = ctl->giant[gi];
         const int32_t o0 = __ldcg(a.off + c);
         const int32_t ub = __ldcg(a.off + c + 1) - o0;
@@ -484,25 +505,25 @@ __device__ __noinline__ void phase_c1h_giant(const ContractArgs &a, ContractSmem
                 if (atomicAdd(acc + cx, __ldcs(a.adjwgt + j)) == 0) atomicOr(bm + (cx >> 5), 1u << (cx & 31));
             }
         }
-        grid_barrier(ctl->bar, bar_epoch, g_cact);
+        group_barrier(gbar, gtarget, gs);
         int32_t mine = 0;
         for (int32_t w = t0w; w < t1w; ++w) mine += __popc(__ldcg(bm + w));
         int32_t tot;
         const int32_t ex = block_excl_scan<kCNT>(mine, sm.scan, tot);
         if (threadIdx.x == 0) ctl->chunk2[blockIdx.x] = tot;  // (C2's chunk sums: idle until C2)
-        grid_barrier(ctl->bar, bar_epoch, g_cact);
-        if (threadIdx.x < 32) {
+        group_barrier(gbar, gtarget, gs);
+        if (threadIdx.x < 32) {  // prefix over the group's lower ranks
             int32_t pre = 0, all = 0;
-            for (int q = threadIdx.x; q < g_cact; q += 32) {
-                const int32_t x = __ldcg(ctl->chunk2 + q);
+            for (int q = threadIdx.x; q < (int)gs; q += 32) {
+                const int32_t x = __ldcg(ctl->chunk2 + gb + q * G);
                 all += x;
-                pre += q < (int)blockIdx.x ? x : 0;
+                pre += q < r ? x : 0;
             }
             pre = warp_sum(pre);
             all = warp_sum(all);
             if (threadIdx.x == 0) {
                 sm.last = pre;
-                if (blockIdx.x == 0) a.cnt[c] = all;
+                if (r == 0) a.cnt[c] = all;
             }
         }
         __syncthreads();
@@ -520,12 +541,11 @@ __device__ __noinline__ void phase_c1h_giant(const ContractArgs &a, ContractSmem
                 acc[cx] = 0;
             }
         }
-        __syncthreads();
-        grid_barrier(ctl->bar, bar_epoch, g_cact);  // the accumulator is clean for the next row
+        group_barrier(gbar, gtarget, gs);  // the accumulator is clean for the group's next row
     }
     // chunk2 accumulates C2's per-CTA sums by atomics from zero: clear this CTA's entry (made
     // visible by the grid barrier that follows C1h)
-    if (ng > 0 && threadIdx.x == 0) ctl->chunk2[blockIdx.x] = 0;
+    if (threadIdx.x == 0) ctl->chunk2[blockIdx.x] = 0;
 }
 
 // ---------------------------------------------------------------------------------------
@@ -1172,9 +1192,15 @@ __global__ void __launch_bounds__(kCNT, kMinB) k_contract_level(const __grid_con
     const int32_t nh = *(volatile int32_t *)&ctl->n_huge;
     if (nh > 0) {
         const int32_t ng = a.dist ? 0 : *(volatile int32_t *)&ctl->n_giant;
-        // (an overflowing list, or a bitmap larger than tout: every row per CTA)
-        const bool giant = ng > 0 && ng <= kMaxGiant && ((long long)nc + 31) / 32 <= 2LL * nnz_in;
-        if (giant) phase_c1h_giant(a, sm, ng, nc, bar_epoch);
+        // groups of >= 16 CTAs, as many as the idle tout holds accumulators + bitmaps for (none:
+        // an overflowing list or no room -- every row per CTA)
+        const long long per_group = (long long)nc + ((long long)nc + 31) / 32 + 96;
+        int32_t G = g_cact / 16 < 32 ? g_cact / 16 : 32;
+        const long long room = 2LL * nnz_in / per_group;
+        if (G > room) G = (int32_t)room;
+        if (G > ng) G = ng;
+        const bool giant = ng > 0 && ng <= kMaxGiant && G >= 1;
+        if (giant) phase_c1h_giant(a, sm, ng, nc, G);
         phase_c1h(a, sm, nh, giant);
         grid_barrier(ctl->bar, bar_epoch, g_cact);
     }
@@ -1336,12 +1362,15 @@ gp_status enqueue_contract(Ctx *ctx, const LevelBufs &lb, int32_t *M, int32_t *C
         const char *e3 = getenv("GP_WARP_ROW_MAX");  // tuning knob (results never depend on it)
         const int wm = e3 ? atoi(e3) : 2 * kWB;
         a.warp_max = wm < kWarpNet ? kWarpNet : wm > 2 * kWB ? 2 * kWB : wm;
-        // Opt-in (GP_GIANT_ROW=<ub>): bit-exact (tests/test_gpu_giant.py, C4 identical to the
-        // per-CTA path), but measured slower on C4 (contraction 122 -> 132 ms): ~140 rows per
-        // level over 65536 entries cost ~40 us each across the grid, and the rows of 8 K..64 K
-        // entries left to single CTAs (~4 s of CTA time per level) still set the phase's length.
+        // Opt-in (GP_GIANT_ROW=<ub>, at most kCtaRow): bit-exact (tests/test_gpu_giant.py, C4
+        // identical to the per-CTA path), but measured slower on C4: every row scans the whole
+        // presence bitmap (nc / 32 words), so thousands of rows over 4096 entries per level cost
+        // more than one CTA per row (contraction 124 -> 435 ms at 4096; the grid-wide variant
+        // over 65536 entries: 122 -> 132 ms, the shorter rows left to single CTAs still set
+        // the phase).
         const char *e4 = getenv("GP_GIANT_ROW");  // knob (results never depend on it)
-        a.giant_ub = prm.dist ? 0 : (e4 ? atoi(e4) : 0);
+        // (<= kCtaRow: the per-CTA rows then never use tout, which holds the groups' accumulators)
+        a.giant_ub = prm.dist ? 0 : (e4 ? std::min(std::max(atoi(e4), 0), kCtaRow) : 0);
     }
     if (!prm.dist) {
         const size_t tiles = ((size_t)(prm.n_bound > 0 ? prm.n_bound : 1) + kRT - 1) / kRT + 1;

@@ -65,7 +65,7 @@ struct MatchCtl {
 };
 
 constexpr int kMaxContractCtas = 1024;  // grid cap of the contraction kernel
-constexpr int kMaxGiant = 2048;         // C1h rows merged by the whole grid per level (contract.cu)
+constexpr int kMaxGiant = 16384;        // C1h rows merged by CTA groups per level (contract.cu)
 
 struct ContractCtl {
     unsigned long long trace[kTrace];
@@ -79,7 +79,8 @@ struct ContractCtl {
     int32_t chunk1[2 * kMaxContractCtas];  // C1 chunk sums {#leaders, sum ub} per owner CTA
     int32_t chunk2[kMaxContractCtas];      // C2 chunk sums of merged entries per owner CTA
     unsigned long long dbg[8];             // debug: slowest C2a warp tile (ns<<32 | tile), paths
-    int32_t n_giant;                       // C1h rows merged by the whole grid (ub > giant_ub)
+    int32_t n_giant;                       // C1h rows merged by CTA groups (ub > giant_ub)
+    unsigned gbar[32];                     // their group barriers
     int32_t giant[kMaxGiant];
 };
 
