@@ -65,7 +65,7 @@ struct MatchCtl {
 };
 
 constexpr int kMaxContractCtas = 1024;  // grid cap of the contraction kernel
-constexpr int kMaxGiant = 16384;        // C1h rows merged by CTA groups per level (contract.cu)
+constexpr int kMaxGiant = 4096;         // C1h rows merged by CTA groups per level (contract.cu)
 
 struct ContractCtl {
     unsigned long long trace[kTrace];
